@@ -1,0 +1,166 @@
+// Row-sharded multi-GPU execution (BASELINE north_star (4); not in the paper,
+// which is single-GPU).  Rows are independent units: a row-only
+// subgraph runs unchanged on each rank's row slice.  A column reduction over
+// the sharded row dimension is completed with ONE ncclAllReduce of the
+// per-rank fp32 partials on the caller's stream (over NVLink / NVSwitch),
+// followed by a small epilogue kernel for the column consumers.
+//
+// libnccl is dlopen'ed (PyTorch's copy is already loaded in-process).
+#include <dlfcn.h>
+
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "internal.h"
+#include "nccl.h"
+
+using namespace astitch;
+
+namespace {
+
+struct Nccl {
+  void* h = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*);
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int);
+  ncclResult_t (*CommDestroy)(ncclComm_t);
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t);
+  const char* (*GetErrorString)(ncclResult_t);
+};
+
+Nccl* nccl(std::string& err) {
+  static Nccl n;
+  static bool tried = false;
+  static std::string load_err;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  if (tried) {
+    if (!n.h) err = load_err;
+    return n.h ? &n : nullptr;
+  }
+  tried = true;
+  const char* cands[] = {getenv("ASTITCH_NCCL"), "libnccl.so.2", "libnccl.so"};
+  for (const char* c : cands) {
+    if (!c) continue;
+    n.h = dlopen(c, RTLD_NOW | RTLD_GLOBAL | RTLD_NOLOAD);
+    if (!n.h) n.h = dlopen(c, RTLD_NOW | RTLD_GLOBAL);
+    if (n.h) break;
+  }
+  if (!n.h) {
+    load_err = "cannot dlopen libnccl.so.2 (import torch first or set ASTITCH_NCCL)";
+    err = load_err;
+    return nullptr;
+  }
+#define SYM(field, name)                                   \
+  *reinterpret_cast<void**>(&n.field) = dlsym(n.h, name);  \
+  if (!n.field) {                                          \
+    load_err = std::string("libnccl lacks ") + name;       \
+    err = load_err;                                        \
+    n.h = nullptr;                                         \
+    return nullptr;                                        \
+  }
+  SYM(GetUniqueId, "ncclGetUniqueId");
+  SYM(CommInitRank, "ncclCommInitRank");
+  SYM(CommDestroy, "ncclCommDestroy");
+  SYM(AllReduce, "ncclAllReduce");
+  SYM(GetErrorString, "ncclGetErrorString");
+#undef SYM
+  return &n;
+}
+
+}  // namespace
+
+struct astitch_comm_s {
+  ncclComm_t comm = nullptr;
+  int world = 1, rank = 0, device = 0;
+};
+
+namespace astitch {
+astitch_status check_io(const Plan& p, const void* const* inputs, void* const* outputs, void* ws);
+KernelParams make_params(const Plan& p, const void* const* inputs, void* const* outputs, void* ws);
+astitch_status launch(const Plan& p, const Kernel& k, KernelParams& kp, void* stream);
+}  // namespace astitch
+
+extern "C" {
+
+astitch_status astitch_comm_unique_id(uint8_t id[128]) {
+  if (!id) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL id");
+  std::string err;
+  Nccl* n = nccl(err);
+  if (!n) return fail(ASTITCH_ERR_NCCL, err);
+  ncclUniqueId u;
+  ncclResult_t r = n->GetUniqueId(&u);
+  if (r != ncclSuccess) return fail(ASTITCH_ERR_NCCL, n->GetErrorString(r));
+  static_assert(sizeof(u) == 128, "ncclUniqueId size");
+  memcpy(id, &u, 128);
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_comm_create(int32_t world, int32_t rank, const uint8_t id[128], int32_t device,
+                                   astitch_comm_t* out) {
+  if (!id || !out || world < 1 || rank < 0 || rank >= world || device < 0)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad comm arguments");
+  std::string err;
+  Nccl* n = nccl(err);
+  if (!n) return fail(ASTITCH_ERR_NCCL, err);
+  int sms = 0, smem = 0;
+  if (!drv_device_info(device, sms, smem, err)) return fail(ASTITCH_ERR_CUDA, err);
+  ncclUniqueId u;
+  memcpy(&u, id, 128);
+  auto* c = new astitch_comm_s();
+  ncclResult_t r = n->CommInitRank(&c->comm, world, u, rank);
+  if (r != ncclSuccess) {
+    delete c;
+    return fail(ASTITCH_ERR_NCCL, std::string("ncclCommInitRank: ") + n->GetErrorString(r));
+  }
+  c->world = world;
+  c->rank = rank;
+  c->device = device;
+  *out = c;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_comm_destroy(astitch_comm_t c) {
+  if (!c) return ASTITCH_OK;
+  std::string err;
+  Nccl* n = nccl(err);
+  if (n && c->comm) n->CommDestroy(c->comm);
+  delete c;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_run_sharded(astitch_plan_t h, astitch_comm_t c, const void* const* inputs,
+                                   void* const* outputs, void* ws, void* stream) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  const Plan& p = *h->p;
+  // row-local subgraphs: no communication at all
+  if (p.colreds.empty() || p.desc.shard_world <= 1) return astitch_run(h, inputs, outputs, ws, stream);
+  if (!c) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "column reduction over shards needs a comm");
+  if (c->world != p.desc.shard_world || c->rank != p.desc.shard_rank)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "comm world/rank do not match the plan's shard");
+  if (p.shard_kernels.empty() || !p.shard_kernels[0].function)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "plan has no loaded sharded kernels");
+  astitch_status s = ASTITCH_OK;
+  // empty shard: contribute identity partials (the main kernel still runs its
+  // combine with zero rows, writing 0 / -inf partials)
+  s = check_io(p, inputs, outputs, ws);
+  if (s != ASTITCH_OK) return s;
+  KernelParams kp = make_params(p, inputs, outputs, ws);
+  if ((s = launch(p, p.shard_kernels[0], kp, stream)) != ASTITCH_OK) return s;
+  std::string err;
+  Nccl* n = nccl(err);
+  if (!n) return fail(ASTITCH_ERR_NCCL, err);
+  const size_t C = static_cast<size_t>(p.desc.cols);
+  char* colpart = static_cast<char*>(ws) + p.ws.colvals + p.post_colvecs.size() * C * 4;
+  for (size_t q = 0; q < p.colreds.size(); ++q) {
+    ncclRedOp_t op = p.g.nodes[p.colreds[q]].sub == ASTITCH_RMAX ? ncclMax : ncclSum;
+    float* buf = reinterpret_cast<float*>(colpart) + q * C;
+    ncclResult_t r = n->AllReduce(buf, buf, C, ncclFloat32, op, c->comm, static_cast<cudaStream_t>(stream));
+    if (r != ncclSuccess) return fail(ASTITCH_ERR_NCCL, std::string("ncclAllReduce: ") + n->GetErrorString(r));
+  }
+  for (size_t i = 1; i < p.shard_kernels.size(); ++i)
+    if ((s = launch(p, p.shard_kernels[i], kp, stream)) != ASTITCH_OK) return s;
+  return ASTITCH_OK;
+}
+
+}  // extern "C"

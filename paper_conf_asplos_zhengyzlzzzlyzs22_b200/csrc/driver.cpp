@@ -1,0 +1,229 @@
+// CUDA driver API access through dlopen("libcuda.so.1"): module loading,
+// occupancy queries and kernel launches (cooperative / cluster attributes) on
+// the caller's stream.  Linking no CUDA library keeps libastitch loadable on
+// hosts without a GPU (the host-side tests).
+#include <cuda.h>
+#include <dlfcn.h>
+
+#include <mutex>
+#include <string>
+
+#include "internal.h"
+
+namespace astitch {
+
+struct Driver {
+  void* h = nullptr;
+  CUresult (*Init)(unsigned int);
+  CUresult (*DeviceGet)(CUdevice*, int);
+  CUresult (*DeviceGetAttribute)(int*, CUdevice_attribute, CUdevice);
+  CUresult (*PrimaryCtxRetain)(CUcontext*, CUdevice);
+  CUresult (*CtxGetCurrent)(CUcontext*);
+  CUresult (*CtxSetCurrent)(CUcontext);
+  CUresult (*CtxGetDevice)(CUdevice*);
+  CUresult (*ModuleLoadData)(CUmodule*, const void*);
+  CUresult (*ModuleUnload)(CUmodule);
+  CUresult (*ModuleGetFunction)(CUfunction*, CUmodule, const char*);
+  CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int);
+  CUresult (*FuncGetAttribute)(int*, CUfunction_attribute, CUfunction);
+  CUresult (*Occupancy)(int*, CUfunction, int, size_t);
+  CUresult (*LaunchKernelEx)(const CUlaunchConfig*, CUfunction, void**, void**);
+  CUresult (*MemsetD8Async)(CUdeviceptr, unsigned char, size_t, CUstream);
+  CUresult (*MemcpyAsync)(CUdeviceptr, CUdeviceptr, size_t, CUstream);
+  CUresult (*StreamSynchronize)(CUstream);
+  CUresult (*GetErrorString)(CUresult, const char**);
+};
+
+namespace {
+
+std::string cu_err(Driver* d, CUresult r, const char* what) {
+  const char* s = nullptr;
+  if (d && d->GetErrorString) d->GetErrorString(r, &s);
+  return std::string(what) + " failed: " + (s ? s : "unknown CUDA error") + " (" + std::to_string(r) + ")";
+}
+
+}  // namespace
+
+Driver* driver(std::string& err) {
+  static Driver d;
+  static bool tried = false;
+  static std::string load_err;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
+  if (tried) {
+    if (!d.h) err = load_err;
+    return d.h ? &d : nullptr;
+  }
+  tried = true;
+  d.h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_LOCAL);
+  if (!d.h) {
+    load_err = "cannot dlopen libcuda.so.1 (no NVIDIA driver on this host)";
+    err = load_err;
+    return nullptr;
+  }
+#define SYM(field, name)                                          \
+  *reinterpret_cast<void**>(&d.field) = dlsym(d.h, name);         \
+  if (!d.field) {                                                 \
+    load_err = std::string("libcuda lacks ") + name;              \
+    err = load_err;                                               \
+    d.h = nullptr;                                                \
+    return nullptr;                                               \
+  }
+  SYM(Init, "cuInit");
+  SYM(DeviceGet, "cuDeviceGet");
+  SYM(DeviceGetAttribute, "cuDeviceGetAttribute");
+  SYM(PrimaryCtxRetain, "cuDevicePrimaryCtxRetain");
+  SYM(CtxGetCurrent, "cuCtxGetCurrent");
+  SYM(CtxSetCurrent, "cuCtxSetCurrent");
+  SYM(CtxGetDevice, "cuCtxGetDevice");
+  SYM(ModuleLoadData, "cuModuleLoadData");
+  SYM(ModuleUnload, "cuModuleUnload");
+  SYM(ModuleGetFunction, "cuModuleGetFunction");
+  SYM(FuncSetAttribute, "cuFuncSetAttribute");
+  SYM(FuncGetAttribute, "cuFuncGetAttribute");
+  SYM(Occupancy, "cuOccupancyMaxActiveBlocksPerMultiprocessor");
+  SYM(LaunchKernelEx, "cuLaunchKernelEx");
+  SYM(MemsetD8Async, "cuMemsetD8Async");
+  SYM(MemcpyAsync, "cuMemcpyAsync");
+  SYM(StreamSynchronize, "cuStreamSynchronize");
+  SYM(GetErrorString, "cuGetErrorString");
+#undef SYM
+  CUresult r = d.Init(0);
+  if (r != CUDA_SUCCESS) {
+    load_err = cu_err(&d, r, "cuInit");
+    err = load_err;
+    d.h = nullptr;
+    return nullptr;
+  }
+  return &d;
+}
+
+namespace {
+
+// Make the device's primary context current on this thread (the one PyTorch
+// uses), unless a context is already current.
+bool ensure_ctx(Driver* d, int device, std::string& err) {
+  CUcontext cur = nullptr;
+  d->CtxGetCurrent(&cur);
+  if (cur) {
+    CUdevice dev;
+    if (d->CtxGetDevice(&dev) == CUDA_SUCCESS && static_cast<int>(dev) == device) return true;
+  }
+  CUdevice dev;
+  CUresult r = d->DeviceGet(&dev, device);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuDeviceGet"); return false; }
+  CUcontext ctx;
+  r = d->PrimaryCtxRetain(&ctx, dev);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuDevicePrimaryCtxRetain"); return false; }
+  r = d->CtxSetCurrent(ctx);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuCtxSetCurrent"); return false; }
+  return true;
+}
+
+}  // namespace
+
+bool drv_device_info(int device, int& sm_count, int& max_smem_optin, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  if (!ensure_ctx(d, device, err)) return false;
+  CUdevice dev;
+  d->DeviceGet(&dev, device);
+  d->DeviceGetAttribute(&sm_count, CU_DEVICE_ATTRIBUTE_MULTIPROCESSOR_COUNT, dev);
+  d->DeviceGetAttribute(&max_smem_optin, CU_DEVICE_ATTRIBUTE_MAX_SHARED_MEMORY_PER_BLOCK_OPTIN, dev);
+  return true;
+}
+
+bool drv_load(Plan& p, Kernel& k, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  if (!ensure_ctx(d, p.device, err)) return false;
+  CUmodule mod;
+  CUresult r = d->ModuleLoadData(&mod, k.cubin.data());
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuModuleLoadData"); return false; }
+  CUfunction fn;
+  r = d->ModuleGetFunction(&fn, mod, k.name.c_str());
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuModuleGetFunction"); d->ModuleUnload(mod); return false; }
+  if (k.smem > 48 * 1024) {
+    r = d->FuncSetAttribute(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, k.smem);
+    if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuFuncSetAttribute(smem)"); d->ModuleUnload(mod); return false; }
+  }
+  int regs = -1, local = -1;
+  d->FuncGetAttribute(&regs, CU_FUNC_ATTRIBUTE_NUM_REGS, fn);
+  d->FuncGetAttribute(&local, CU_FUNC_ATTRIBUTE_LOCAL_SIZE_BYTES, fn);
+  k.regs = regs;
+  if (k.spill_bytes < 0) k.spill_bytes = local;
+  int occ = 0;
+  r = d->Occupancy(&occ, fn, k.threads, static_cast<size_t>(k.smem));
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuOccupancyMaxActiveBlocksPerMultiprocessor"); d->ModuleUnload(mod); return false; }
+  k.occupancy = occ;
+  k.module = mod;
+  k.function = fn;
+  return true;
+}
+
+bool drv_unload(Kernel& k) {
+  std::string err;
+  Driver* d = driver(err);
+  if (d && k.module) d->ModuleUnload(static_cast<CUmodule>(k.module));
+  k.module = nullptr;
+  k.function = nullptr;
+  return true;
+}
+
+bool drv_launch(const Kernel& k, void* params, size_t params_size, void* stream, std::string& err) {
+  (void)params_size;
+  void* args[] = {params};
+  return drv_launch_args(k, args, stream, err);
+}
+
+bool drv_launch_args(const Kernel& k, void** args, void* stream, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUlaunchConfig cfg{};
+  cfg.gridDimX = static_cast<unsigned>(k.grid);
+  cfg.gridDimY = 1;
+  cfg.gridDimZ = 1;
+  cfg.blockDimX = static_cast<unsigned>(k.threads);
+  cfg.blockDimY = 1;
+  cfg.blockDimZ = 1;
+  cfg.sharedMemBytes = static_cast<unsigned>(k.smem);
+  cfg.hStream = static_cast<CUstream>(stream);
+  CUlaunchAttribute attr[1];
+  if (k.cooperative) {
+    attr[0].id = CU_LAUNCH_ATTRIBUTE_COOPERATIVE;
+    attr[0].value.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+  }
+  CUresult r = d->LaunchKernelEx(&cfg, static_cast<CUfunction>(k.function), args, nullptr);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, ("cuLaunchKernelEx(" + k.name + ")").c_str()); return false; }
+  return true;
+}
+
+bool drv_memset_async(void* ptr, size_t bytes, void* stream, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUresult r = d->MemsetD8Async(reinterpret_cast<CUdeviceptr>(ptr), 0, bytes, static_cast<CUstream>(stream));
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuMemsetD8Async"); return false; }
+  return true;
+}
+
+bool drv_memcpy_async(void* dst, const void* src, size_t bytes, int kind, void* stream, std::string& err) {
+  (void)kind;
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUresult r = d->MemcpyAsync(reinterpret_cast<CUdeviceptr>(dst), reinterpret_cast<CUdeviceptr>(src), bytes,
+                              static_cast<CUstream>(stream));
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuMemcpyAsync"); return false; }
+  return true;
+}
+
+bool drv_sync(void* stream, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUresult r = d->StreamSynchronize(static_cast<CUstream>(stream));
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuStreamSynchronize"); return false; }
+  return true;
+}
+
+}  // namespace astitch

@@ -1,0 +1,203 @@
+// Internal data structures of the AStitch B200 engine (not part of the C ABI).
+//
+//   Graph    — the tiny SSA op-graph IR of one stitch op (Sec. 4.1).
+//   Analysis — per-op class, dominant / group, scheme (Sec. 4.3).
+//   Mapping  — the adaptive thread mapping chosen for the dominant schedule
+//              (task packing / splitting).
+//   Plan     — everything astitch_run needs: kernels, launch config, workspace.
+#pragma once
+
+#include <cstdint>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "astitch.h"
+
+namespace astitch {
+
+// ------------------------------------------------------------------ errors
+void set_error(const std::string& msg);
+astitch_status fail(astitch_status s, const std::string& msg);
+
+struct Error {
+  astitch_status status;
+  std::string msg;
+};
+
+// ------------------------------------------------------------------ IR
+enum class NodeType { Input, Const, Unary, Binary, Reduce, Bcast };
+
+struct Node {
+  NodeType type = NodeType::Input;
+  int sub = 0;             // unop / binop / redop
+  int axis = 0;            // astitch_axis for Reduce / Bcast
+  int a = -1, b = -1;      // operands
+  astitch_kind kind = ASTITCH_FULL;
+  astitch_dtype dtype = ASTITCH_F32;  // storage dtype (inputs)
+  double cval = 0.0;       // Const value
+  int input_index = -1;    // position in the input list
+};
+
+struct Graph {
+  std::vector<Node> nodes;
+  std::vector<int> inputs;                  // node ids in input order
+  std::vector<int> outputs;                 // node ids in output order
+  std::vector<astitch_dtype> output_dtypes;
+  int lengths_node = -1;
+  int64_t rows_per_segment = 0;
+};
+
+int dtype_size(astitch_dtype d);
+const char* dtype_name(astitch_dtype d);
+const char* kind_name(astitch_kind k);
+const char* unop_name(int op);
+const char* binop_name(int op);
+
+// ------------------------------------------------------------------ analysis
+// Op classes of the paper's taxonomy: light / heavy element-wise,
+// broadcast, row- / column-reduce.
+enum class OpClass { Input, Const, LightEW, HeavyEW, BcastRow, BcastCol, ReduceRow, ReduceCol };
+// Stitching schemes of Table 1.
+enum class Scheme { Independent, Local, Regional, Global };
+
+const char* opclass_name(OpClass c);
+const char* scheme_name(Scheme s);
+
+struct NodeInfo {
+  OpClass cls = OpClass::Input;
+  bool live = false;           // reaches an output
+  bool post = false;           // depends on a column reduction (after the grid barrier)
+  bool candidate = false;      // dominant candidate (Step 1)
+  bool dominant = false;       // final dominant
+  bool sub_dominant = false;
+  int group = -1;              // op group id
+  Scheme scheme = Scheme::Local;
+  bool global_full = false;    // FULL value buffered in HBM across the barrier
+  std::vector<int> consumers;
+};
+
+enum class Template {
+  RowTeam,     // row-reduce / EW: a team of lanes per row, registers + shuffles (regional)
+  PackedTile,  // many tiny rows: TMA-bulk tiles in smem, thread per row (horizontal packing)
+  GlobalSweep, // column reduce: vertical packing + block partials + grid barrier (global)
+  SplitRow     // few long rows: row split over a thread-block cluster (task splitting)
+};
+const char* template_name(Template t);
+
+struct Mapping {
+  Template tmpl = Template::RowTeam;
+  int vec_elems = 1;        // E: elements per chunk (one vector access per tensor)
+  int chunks = 1;           // C / E
+  int team = 32;            // T: lanes cooperating on one row
+  int chunks_per_lane = 1;  // V
+  int threads = 256;        // block size
+  int rows_per_block = 8;   // teams per block (threads / T), or tile rows (PackedTile)
+  int row_unroll = 1;       // U: rows per team per iteration (vertical packing ILP)
+  bool prefetch = true;     // software-pipeline the next row's loads
+  bool hoist_colvec = true; // keep COLVEC operands in registers across rows
+  int tile_rows = 0;        // PackedTile rows per stage
+  int stages = 0;           // PackedTile pipeline stages
+  int split = 1;            // CTAs per row (task splitting; 1 = none)
+  int64_t grid = 1;
+  int blocks_per_sm = 1;    // assume-relax-apply target
+  int reg_cap = 255;
+  int64_t vertical_trips = 1;
+  double lane_util = 1.0;
+  int smem_bytes = 0;       // dynamic shared memory per block
+  int bank_conflict_ways = 1;
+  std::string reason;       // selector decision trace
+};
+
+// ------------------------------------------------------------------ plan
+struct Kernel {
+  std::string name;
+  std::string source;
+  std::vector<char> cubin;
+  std::string log;
+  int threads = 256;
+  int64_t grid = 1;
+  int smem = 0;
+  bool cooperative = false;
+  int regs = -1;
+  int spill_bytes = -1;
+  int occupancy = -1;        // blocks per SM from the occupancy API
+  void* module = nullptr;    // CUmodule
+  void* function = nullptr;  // CUfunction
+};
+
+struct WsLayout {
+  size_t barrier = 0;        // 2 x u32 (+ pad)
+  size_t partials = 0;       // [grid][ncolred][C] fp32 block partials
+  size_t colvals = 0;        // [ncolvec_post][C] fp32 finalized column values
+  size_t globals = 0;        // [nglobal_full][R][C] fp32 buffers
+  size_t total = 0;
+};
+
+struct Plan {
+  Graph g;
+  astitch_plan_desc desc{};
+  int sm_count = 148;
+  std::vector<NodeInfo> info;
+  std::vector<std::vector<int>> groups;
+  Mapping map;
+  std::vector<int> colreds;      // column reduce node ids (in order)
+  std::vector<int> post_colvecs; // COLVEC values computed after the barrier (incl. colreds)
+  std::vector<int> global_fulls; // FULL values buffered in HBM across the barrier
+  bool needs_sweep2 = false;
+  std::vector<Kernel> kernels;   // kernels launched by astitch_run, in order
+  std::vector<Kernel> shard_kernels; // kernels of the sharded path (after the allreduce)
+  WsLayout ws;
+  uint64_t compulsory_bytes = 0;
+  int device = -1;
+  std::string describe;
+};
+
+// planner.cpp
+void analyse(Plan& p);                 // a1, a2, a5: classes, dominants, groups, schemes
+void select_mapping(Plan& p);          // a3, a4, a6, a7: thread mapping, memory, launch
+void plan_workspace(Plan& p);
+void retune_grid(Plan& p);
+std::string describe_json(const Plan& p);
+uint64_t compulsory_bytes(const Plan& p);
+
+// codegen.cpp
+std::string generate_kernel(const Plan& p, int role, const std::string& name);
+enum KernelRole { ROLE_MAIN = 0, ROLE_SHARD_MAIN = 1, ROLE_SHARD_FINAL = 2, ROLE_SHARD_SWEEP2 = 3 };
+
+// jit.cpp
+bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<char>& cubin,
+                   std::string& log, std::string& err);
+const char* device_header_source();
+
+// driver.cpp — libcuda via dlopen
+struct Driver;
+Driver* driver(std::string& err);
+bool drv_load(Plan& p, Kernel& k, std::string& err);
+bool drv_launch(const Kernel& k, void* params, size_t params_size, void* stream, std::string& err);
+bool drv_launch_args(const Kernel& k, void** args, void* stream, std::string& err);
+bool drv_unload(Kernel& k);
+bool drv_memset_async(void* ptr, size_t bytes, void* stream, std::string& err);
+bool drv_memcpy_async(void* dst, const void* src, size_t bytes, int kind, void* stream,
+                      std::string& err);
+bool drv_device_info(int device, int& sm_count, int& max_smem_optin, std::string& err);
+bool drv_sync(void* stream, std::string& err);
+
+// kernel parameter block (mirrors the struct emitted by codegen)
+constexpr int kMaxIO = 16;
+struct KernelParams {
+  const void* in[kMaxIO];
+  void* out[kMaxIO];
+  void* ws;
+  long long rows;
+  long long row_offset;   // global row index of row 0 (sharded plans; mask segments)
+};
+
+}  // namespace astitch
+
+struct astitch_graph_s {
+  astitch::Graph g;
+};
+struct astitch_plan_s {
+  std::unique_ptr<astitch::Plan> p;
+};

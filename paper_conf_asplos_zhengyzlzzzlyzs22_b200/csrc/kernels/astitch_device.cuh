@@ -1,0 +1,443 @@
+// astitch_device.cuh — hand-written sm_100a device building blocks of the
+// stitched kernels.  The planner's code generator (codegen.cpp) instantiates
+// one of the scheme templates below per subgraph and fills in the op chain;
+// the result is compiled by NVRTC for sm_100a (the paper's JIT).
+//
+//   memory  : 16/32-byte streaming loads (ld.global.nc.L1::no_allocate),
+//             vector stores, bf16/f16 <-> fp32 packing
+//   local   : element-wise math in fp32 registers (Table 1 "local")
+//   regional: team reductions by warp shuffles / shared memory (Table 1
+//             "regional"; block locality)
+//   global  : HBM partials + generation-counted grid barrier (Table 1
+//             "global")
+//   packed  : TMA bulk (cp.async.bulk) row tiles + mbarrier pipeline for
+//             many tiny rows (horizontal packing)
+//
+// No includes: NVRTC compiles this without the CUDA headers.
+#pragma once
+
+typedef unsigned int u32;
+typedef unsigned long long u64;
+typedef unsigned short u16;
+
+#define AS_INF __int_as_float(0x7f800000)
+
+namespace as {
+
+// ------------------------------------------------------------------ raw chunks
+template <int NB> struct Raw;
+template <> struct Raw<2> { u16 x; };
+template <> struct Raw<4> { u32 x; };
+template <> struct Raw<8> { u32 x, y; };
+template <> struct Raw<16> { u32 x, y, z, w; };
+template <> struct Raw<32> { u32 x, y, z, w, a, b, c, d; };
+
+// streaming (read-once) global loads: no L1 allocation
+__device__ __forceinline__ Raw<2> ldg(const Raw<2>* p) {
+  Raw<2> r;
+  asm volatile("ld.global.nc.L1::no_allocate.b16 %0, [%1];" : "=h"(r.x) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<4> ldg(const Raw<4>* p) {
+  Raw<4> r;
+  asm volatile("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(r.x) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<8> ldg(const Raw<8>* p) {
+  Raw<8> r;
+  asm volatile("ld.global.nc.L1::no_allocate.v2.b32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<16> ldg(const Raw<16>* p) {
+  Raw<16> r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<32> ldg(const Raw<32>* p) {
+  Raw<32> r;
+  asm volatile("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w), "=r"(r.a), "=r"(r.b), "=r"(r.c), "=r"(r.d)
+               : "l"(p));
+  return r;
+}
+// L2-coherent (.cg) loads of workspace data written earlier in the same kernel
+__device__ __forceinline__ Raw<16> ldg_cg(const Raw<16>* p) {
+  Raw<16> r;
+  asm volatile("ld.global.cg.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<8> ldg_cg(const Raw<8>* p) {
+  Raw<8> r;
+  asm volatile("ld.global.cg.v2.b32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<4> ldg_cg(const Raw<4>* p) {
+  Raw<4> r;
+  asm volatile("ld.global.cg.b32 %0, [%1];" : "=r"(r.x) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<32> ldg_cg(const Raw<32>* p) {
+  Raw<32> r;
+  const Raw<16>* q = reinterpret_cast<const Raw<16>*>(p);
+  Raw<16> a = ldg_cg(q), b = ldg_cg(q + 1);
+  r.x = a.x; r.y = a.y; r.z = a.z; r.w = a.w; r.a = b.x; r.b = b.y; r.c = b.z; r.d = b.w;
+  return r;
+}
+// L1-cached read-only loads for operands re-read every row (COLVEC vectors)
+__device__ __forceinline__ Raw<2> ldg_l1(const Raw<2>* p) {
+  Raw<2> r; asm volatile("ld.global.nc.b16 %0, [%1];" : "=h"(r.x) : "l"(p)); return r;
+}
+__device__ __forceinline__ Raw<4> ldg_l1(const Raw<4>* p) {
+  Raw<4> r; asm volatile("ld.global.nc.b32 %0, [%1];" : "=r"(r.x) : "l"(p)); return r;
+}
+__device__ __forceinline__ Raw<8> ldg_l1(const Raw<8>* p) {
+  Raw<8> r; asm volatile("ld.global.nc.v2.b32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p)); return r;
+}
+__device__ __forceinline__ Raw<16> ldg_l1(const Raw<16>* p) {
+  Raw<16> r;
+  asm volatile("ld.global.nc.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ Raw<32> ldg_l1(const Raw<32>* p) {
+  Raw<32> r;
+  asm volatile("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w), "=r"(r.a), "=r"(r.b), "=r"(r.c), "=r"(r.d)
+               : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ void stg(Raw<2>* p, const Raw<2>& r) {
+  asm volatile("st.global.b16 [%0], %1;" ::"l"(p), "h"(r.x) : "memory");
+}
+__device__ __forceinline__ void stg(Raw<4>* p, const Raw<4>& r) {
+  asm volatile("st.global.b32 [%0], %1;" ::"l"(p), "r"(r.x) : "memory");
+}
+__device__ __forceinline__ void stg(Raw<8>* p, const Raw<8>& r) {
+  asm volatile("st.global.v2.b32 [%0], {%1,%2};" ::"l"(p), "r"(r.x), "r"(r.y) : "memory");
+}
+__device__ __forceinline__ void stg(Raw<16>* p, const Raw<16>& r) {
+  asm volatile("st.global.v4.b32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w)
+               : "memory");
+}
+__device__ __forceinline__ void stg(Raw<32>* p, const Raw<32>& r) {
+  asm volatile("st.global.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(r.x), "r"(r.y), "r"(r.z),
+               "r"(r.w), "r"(r.a), "r"(r.b), "r"(r.c), "r"(r.d)
+               : "memory");
+}
+
+// shared-memory chunk loads / stores (packed template); saddr = shared window address
+__device__ __forceinline__ Raw<2> lds(u32 a) { Raw<2> r; asm volatile("ld.shared.b16 %0, [%1];" : "=h"(r.x) : "r"(a)); return r; }
+__device__ __forceinline__ Raw<4> lds4(u32 a) { Raw<4> r; asm volatile("ld.shared.b32 %0, [%1];" : "=r"(r.x) : "r"(a)); return r; }
+template <int NB> __device__ __forceinline__ Raw<NB> lds_chunk(u32 a);
+template <> __device__ __forceinline__ Raw<2> lds_chunk<2>(u32 a) { return lds(a); }
+template <> __device__ __forceinline__ Raw<4> lds_chunk<4>(u32 a) { return lds4(a); }
+template <> __device__ __forceinline__ Raw<8> lds_chunk<8>(u32 a) {
+  Raw<8> r; asm volatile("ld.shared.v2.b32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "r"(a)); return r;
+}
+template <> __device__ __forceinline__ Raw<16> lds_chunk<16>(u32 a) {
+  Raw<16> r;
+  asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(a));
+  return r;
+}
+template <> __device__ __forceinline__ Raw<32> lds_chunk<32>(u32 a) {
+  Raw<32> r;
+  asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(a));
+  asm volatile("ld.shared.v4.b32 {%0,%1,%2,%3}, [%4];" : "=r"(r.a), "=r"(r.b), "=r"(r.c), "=r"(r.d) : "r"(a + 16));
+  return r;
+}
+template <int NB> __device__ __forceinline__ void sts_chunk(u32 a, const Raw<NB>& r);
+template <> __device__ __forceinline__ void sts_chunk<2>(u32 a, const Raw<2>& r) {
+  asm volatile("st.shared.b16 [%0], %1;" ::"r"(a), "h"(r.x) : "memory");
+}
+template <> __device__ __forceinline__ void sts_chunk<4>(u32 a, const Raw<4>& r) {
+  asm volatile("st.shared.b32 [%0], %1;" ::"r"(a), "r"(r.x) : "memory");
+}
+template <> __device__ __forceinline__ void sts_chunk<8>(u32 a, const Raw<8>& r) {
+  asm volatile("st.shared.v2.b32 [%0], {%1,%2};" ::"r"(a), "r"(r.x), "r"(r.y) : "memory");
+}
+template <> __device__ __forceinline__ void sts_chunk<16>(u32 a, const Raw<16>& r) {
+  asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w) : "memory");
+}
+template <> __device__ __forceinline__ void sts_chunk<32>(u32 a, const Raw<32>& r) {
+  asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w) : "memory");
+  asm volatile("st.shared.v4.b32 [%0], {%1,%2,%3,%4};" ::"r"(a + 16), "r"(r.a), "r"(r.b), "r"(r.c), "r"(r.d) : "memory");
+}
+
+// ------------------------------------------------------------------ dtype conversion
+// DT: 0 = f32, 1 = bf16, 2 = f16
+__device__ __forceinline__ float bf16lo(u32 w) { return __int_as_float(w << 16); }
+__device__ __forceinline__ float bf16hi(u32 w) { return __int_as_float(w & 0xffff0000u); }
+__device__ __forceinline__ u32 pack_bf16x2(float lo, float hi) {
+  u32 r;
+  asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+__device__ __forceinline__ float f16lo(u32 w) {
+  float f; asm("{.reg .b16 l, h; mov.b32 {l, h}, %1; cvt.f32.f16 %0, l;}" : "=f"(f) : "r"(w)); return f;
+}
+__device__ __forceinline__ float f16hi(u32 w) {
+  float f; asm("{.reg .b16 l, h; mov.b32 {l, h}, %1; cvt.f32.f16 %0, h;}" : "=f"(f) : "r"(w)); return f;
+}
+__device__ __forceinline__ u32 pack_f16x2(float lo, float hi) {
+  u32 r;
+  asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+
+__device__ __forceinline__ void words_to_float(int DT, const u32* w, int nwords, float* out) {
+  if (DT == 0) {
+#pragma unroll
+    for (int i = 0; i < nwords; ++i) out[i] = __int_as_float(w[i]);
+  } else if (DT == 1) {
+#pragma unroll
+    for (int i = 0; i < nwords; ++i) { out[2 * i] = bf16lo(w[i]); out[2 * i + 1] = bf16hi(w[i]); }
+  } else {
+#pragma unroll
+    for (int i = 0; i < nwords; ++i) { out[2 * i] = f16lo(w[i]); out[2 * i + 1] = f16hi(w[i]); }
+  }
+}
+
+template <int DT, int E> struct Conv {
+  static constexpr int NB = E * (DT == 0 ? 4 : 2);
+  __device__ static __forceinline__ void unpack(const Raw<NB>& r, float* o) {
+    if constexpr (NB == 2) {
+      u32 w = r.x;
+      o[0] = DT == 1 ? bf16lo(w) : f16lo(w);
+    } else {
+      words_to_float(DT, reinterpret_cast<const u32*>(&r), NB / 4, o);
+    }
+  }
+  __device__ static __forceinline__ Raw<NB> pack(const float* v) {
+    Raw<NB> r;
+    if constexpr (NB == 2) {
+      u32 w = DT == 1 ? pack_bf16x2(v[0], 0.f) : pack_f16x2(v[0], 0.f);
+      r.x = static_cast<u16>(w & 0xffffu);
+    } else {
+      u32* w = reinterpret_cast<u32*>(&r);
+      if (DT == 0) {
+#pragma unroll
+        for (int i = 0; i < NB / 4; ++i) w[i] = __float_as_int(v[i]);
+      } else {
+#pragma unroll
+        for (int i = 0; i < NB / 4; ++i)
+          w[i] = DT == 1 ? pack_bf16x2(v[2 * i], v[2 * i + 1]) : pack_f16x2(v[2 * i], v[2 * i + 1]);
+      }
+    }
+    return r;
+  }
+};
+
+// scalar (ROWVEC / COLVEC element) load / store with dtype
+template <int DT> __device__ __forceinline__ float ld_scalar(const void* base, long long i) {
+  if (DT == 0) return __ldg(reinterpret_cast<const float*>(base) + i);
+  u16 h = __ldg(reinterpret_cast<const unsigned short*>(base) + i);
+  return DT == 1 ? __int_as_float(static_cast<u32>(h) << 16) : f16lo(h);
+}
+template <int DT> __device__ __forceinline__ void st_scalar(void* base, long long i, float v) {
+  if (DT == 0) { reinterpret_cast<float*>(base)[i] = v; return; }
+  u32 w = DT == 1 ? pack_bf16x2(v, 0.f) : pack_f16x2(v, 0.f);
+  reinterpret_cast<unsigned short*>(base)[i] = static_cast<unsigned short>(w & 0xffffu);
+}
+
+// ------------------------------------------------------------------ local: fp32 math
+// MUFU-based with cancellation-free forms (reading R6: no tanh.approx).
+__device__ __forceinline__ float ex2(float x) { float r; asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
+__device__ __forceinline__ float rcp(float x) { float r; asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
+__device__ __forceinline__ float rsq(float x) { float r; asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
+__device__ __forceinline__ float sqrt_(float x) { float r; asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
+__device__ __forceinline__ float fexp(float x) { return ex2(x * 1.4426950408889634f); }
+__device__ __forceinline__ float fdiv(float a, float b) { return a * rcp(b); }
+__device__ __forceinline__ float fsigmoid(float x) { return rcp(1.0f + fexp(-x)); }
+// tanh for general use: accurate libdevice form (small |x| would cancel in the exp form)
+__device__ __forceinline__ float ftanh(float x) { return tanhf(x); }
+__device__ __forceinline__ float ferf(float x) { return erff(x); }
+__device__ __forceinline__ float flog(float x) { return logf(x); }
+
+#define AS_GELU_C 0.7978845608028654f  /* sqrt(2/pi) */
+#define AS_GELU_K 0.044715f
+// gelu_tanh(x) = 0.5 x (1 + tanh(u)) = x * sigmoid(2u), u = c (x + k x^3)
+__device__ __forceinline__ float gelu_tanh(float x) {
+  float u = AS_GELU_C * fmaf(AS_GELU_K * x, x * x, x);
+  return x * rcp(1.0f + ex2(-2.8853900817779268f * u));   // exp(-2u) = 2^(-2u log2 e)
+}
+// d/dx gelu_tanh = sigmoid(2u) + 0.5 x sech^2(u) c (1 + 3 k x^2)
+// with e = exp(-2|u|): sigmoid(2u) = u>=0 ? 1/(1+e) : e/(1+e);  sech^2 u = 4e/(1+e)^2
+__device__ __forceinline__ float gelu_tanh_grad(float x) {
+  float x2 = x * x;
+  float u = AS_GELU_C * fmaf(AS_GELU_K * x, x2, x);
+  float e = ex2(-2.8853900817779268f * fabsf(u));
+  float r = rcp(1.0f + e);
+  float sig = u >= 0.f ? r : e * r;
+  float sech2 = 4.0f * e * r * r;
+  float du = AS_GELU_C * fmaf(3.0f * AS_GELU_K, x2, 1.0f);
+  return fmaf(0.5f * x * sech2, du, sig);
+}
+// exact GELU: x Phi(x) = 0.5 x erfc(-x / sqrt 2) (no cancellation for x << 0)
+__device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * erfcf(-0.7071067811865476f * x); }
+
+__device__ __forceinline__ float fpow(float a, float b) { return powf(a, b); }
+
+// ------------------------------------------------------------------ regional: team reductions
+template <int T> __device__ __forceinline__ float team_sum(float v) {
+#pragma unroll
+  for (int o = (T < 32 ? T : 32) / 2; o > 0; o /= 2) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+template <int T> __device__ __forceinline__ float team_max(float v) {
+#pragma unroll
+  for (int o = (T < 32 ? T : 32) / 2; o > 0; o /= 2) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+// team larger than a warp == whole block: warp tree, then a fixed-order
+// combine of the per-warp values in shared memory (deterministic).
+template <int T, bool MAX> __device__ __forceinline__ float block_team_reduce(float v, float* scratch) {
+  v = MAX ? team_max<32>(v) : team_sum<32>(v);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  __syncthreads();  // scratch reuse guard
+  if (l == 0) scratch[w] = v;
+  __syncthreads();
+  constexpr int NW = T / 32;
+  float r = (l < NW) ? scratch[l] : (MAX ? -AS_INF : 0.f);
+  r = MAX ? team_max<32>(r) : team_sum<32>(r);
+  return r;
+}
+
+// fp64 team sum for cancellation-prone row sums (e.g. a mean that is then
+// subtracted): the result is carried as a double and split hi+lo in fp32.
+template <int T> __device__ __forceinline__ double team_sum_d(double v) {
+#pragma unroll
+  for (int o = (T < 32 ? T : 32) / 2; o > 0; o /= 2) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+template <int T> __device__ __forceinline__ double block_team_sum_d(double v, double* scratch) {
+  v = team_sum_d<32>(v);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  __syncthreads();
+  if (l == 0) scratch[w] = v;
+  __syncthreads();
+  constexpr int NW = T / 32;
+  double r = (l < NW) ? scratch[l] : 0.0;
+  return team_sum_d<32>(r);
+}
+template <int N> struct TreeD {
+  __device__ static __forceinline__ double reduce(const float* a) {
+    if constexpr (N == 1) {
+      return static_cast<double>(a[0]);
+    } else {
+      constexpr int H = N / 2;
+      return TreeD<H>::reduce(a) + TreeD<N - H>::reduce(a + H);
+    }
+  }
+};
+
+// pairwise tree over a register array (fixed order -> deterministic)
+template <int N, bool MAX> struct Tree {
+  __device__ static __forceinline__ float reduce(const float* a) {
+    if constexpr (N == 1) {
+      return a[0];
+    } else {
+      constexpr int H = N / 2;
+      float l = Tree<H, MAX>::reduce(a);
+      float r = Tree<N - H, MAX>::reduce(a + H);
+      return MAX ? fmaxf(l, r) : l + r;
+    }
+  }
+};
+
+// ------------------------------------------------------------------ global: grid barrier
+// Generation-counted, self-resetting barrier for a co-resident (cooperative)
+// grid.  bar[0] = arrival count, bar[1] = generation.  No memset per run.
+__device__ __forceinline__ u32 ld_acquire(const u32* p) {
+  u32 v; asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
+}
+__device__ __forceinline__ void st_release(u32* p, u32 v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ u32 atom_add_acqrel(u32* p, u32 v) {
+  u32 old; asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory"); return old;
+}
+__device__ __forceinline__ void grid_barrier(u32* bar) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const u32 nb = gridDim.x * gridDim.y * gridDim.z;
+    u32 gen = ld_acquire(bar + 1);
+    __threadfence();
+    u32 arrived = atom_add_acqrel(bar, 1u);
+    if (arrived == nb - 1) {
+      *reinterpret_cast<volatile u32*>(bar) = 0u;
+      __threadfence();
+      st_release(bar + 1, gen + 1);
+    } else {
+      while (ld_acquire(bar + 1) == gen) { __nanosleep(20); }
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+// L2-coherent load of data written earlier in the same kernel by other blocks
+__device__ __forceinline__ float ld_cg(const float* p) { return __ldcg(p); }
+
+// ------------------------------------------------------------------ packed: TMA bulk + mbarrier
+__device__ __forceinline__ u32 smem_addr(const void* p) {
+  return static_cast<u32>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(u32 bar, u32 count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(u32 bar, u32 bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(u32 bar, u32 parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(bar), "r"(parity)
+      : "memory");
+}
+// global -> shared bulk copy completing on an mbarrier (UBLKCP)
+__device__ __forceinline__ void bulk_g2s(u32 dst, const void* src, u32 bytes, u32 bar) {
+  asm volatile("cp.async.bulk.shared::cta.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+// shared -> global bulk copy (bulk-group completion)
+__device__ __forceinline__ void bulk_s2g(void* dst, u32 src, u32 bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N> __device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+}  // namespace as
+
+// ------------------------------------------------------------------ measurement kernels
+// Barrier-only kernel (Table 6 micro-benchmark on B200).
+extern "C" __global__ void astitch_barrier_bench(u32* bar, int iters) {
+  for (int i = 0; i < iters; ++i) as::grid_barrier(bar);
+}
+// Copy ceiling with the same streaming 16-byte accesses as the stitched kernels.
+extern "C" __global__ void __launch_bounds__(256) astitch_copy_bench(const as::Raw<16>* __restrict__ src,
+                                                                     as::Raw<16>* __restrict__ dst,
+                                                                     long long n16) {
+  long long i = blockIdx.x * 256LL + threadIdx.x;
+  const long long stride = gridDim.x * 256LL;
+  for (; i + 3 * stride < n16; i += 4 * stride) {
+    as::Raw<16> a = as::ldg(src + i), b = as::ldg(src + i + stride), c = as::ldg(src + i + 2 * stride),
+                d = as::ldg(src + i + 3 * stride);
+    as::stg(dst + i, a); as::stg(dst + i + stride, b); as::stg(dst + i + 2 * stride, c);
+    as::stg(dst + i + 3 * stride, d);
+  }
+  for (; i < n16; i += stride) as::stg(dst + i, as::ldg(src + i));
+}

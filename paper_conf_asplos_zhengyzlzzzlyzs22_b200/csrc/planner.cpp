@@ -1,0 +1,618 @@
+// Planner: the paper's Sec. 4 pipeline, re-derived for B200.
+//
+//   a1  classify ops (light / heavy EW, broadcast, row / column reduce)
+//   a2  dominant candidates -> dominant merging -> op groups
+//   a3  adaptive thread mapping (packing / splitting)
+//   a4  schedule propagation (every op inherits its group's mapping)
+//   a5  scheme finalisation (passive / proactive block locality)
+//   a6  memory plan (smem per block, HBM workspace)
+//   a7  launch configuration (assume-relax-apply register bound)
+//
+// Constants that the paper gives for V100 (1024-element split threshold,
+// 1024-thread blocks, 160 blocks per wave) are recomputed from B200 limits
+// (reading R15).
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <functional>
+#include <numeric>
+#include <sstream>
+
+#include "internal.h"
+
+namespace astitch {
+
+const char* opclass_name(OpClass c) {
+  switch (c) {
+    case OpClass::Input: return "input";
+    case OpClass::Const: return "const";
+    case OpClass::LightEW: return "light_ew";
+    case OpClass::HeavyEW: return "heavy_ew";
+    case OpClass::BcastRow: return "broadcast_row";
+    case OpClass::BcastCol: return "broadcast_col";
+    case OpClass::ReduceRow: return "reduce_row";
+    case OpClass::ReduceCol: return "reduce_col";
+  }
+  return "?";
+}
+
+const char* scheme_name(Scheme s) {
+  switch (s) {
+    case Scheme::Independent: return "independent";
+    case Scheme::Local: return "local";
+    case Scheme::Regional: return "regional";
+    case Scheme::Global: return "global";
+  }
+  return "?";
+}
+
+const char* template_name(Template t) {
+  switch (t) {
+    case Template::RowTeam: return "row_team";
+    case Template::PackedTile: return "packed_tile";
+    case Template::GlobalSweep: return "global_sweep";
+    case Template::SplitRow: return "split_row";
+  }
+  return "?";
+}
+
+namespace {
+
+// Heavy element-wise ops ("tanh, power, and log"; we add the other
+// transcendental / division ops that cost a MUFU or a multi-instruction sequence).
+bool is_heavy_unop(int op) {
+  switch (op) {
+    case ASTITCH_NEG:
+    case ASTITCH_ABS: return false;
+    default: return true;
+  }
+}
+// Division is light: in Fig. 7(a)/9 divide.1 is not a dominant candidate while
+// power.1 is, so only POW counts as a heavy binary op.
+bool is_heavy_binop(int op) { return op == ASTITCH_POW; }
+
+struct DSU {
+  std::vector<int> p;
+  explicit DSU(int n) : p(n) { std::iota(p.begin(), p.end(), 0); }
+  int find(int x) { return p[x] == x ? x : p[x] = find(p[x]); }
+  void unite(int a, int b) { p[find(a)] = find(b); }
+};
+
+}  // namespace
+
+// ------------------------------------------------------------------------ a1/a2/a5
+void analyse(Plan& p) {
+  const Graph& g = p.g;
+  const int n = static_cast<int>(g.nodes.size());
+  p.info.assign(n, NodeInfo());
+  auto& info = p.info;
+
+  // consumers
+  for (int i = 0; i < n; ++i) {
+    const Node& nd = g.nodes[i];
+    if (nd.a >= 0) info[nd.a].consumers.push_back(i);
+    if (nd.b >= 0 && nd.b != nd.a) info[nd.b].consumers.push_back(i);
+  }
+  // liveness: reverse reachability from outputs
+  std::function<void(int)> mark = [&](int i) {
+    if (info[i].live) return;
+    info[i].live = true;
+    if (g.nodes[i].a >= 0) mark(g.nodes[i].a);
+    if (g.nodes[i].b >= 0) mark(g.nodes[i].b);
+  };
+  for (int o : g.outputs) mark(o);
+  if (g.lengths_node >= 0) info[g.lengths_node].live = true;
+
+  // a1: classification
+  for (int i = 0; i < n; ++i) {
+    const Node& nd = g.nodes[i];
+    OpClass c = OpClass::Input;
+    switch (nd.type) {
+      case NodeType::Input: c = OpClass::Input; break;
+      case NodeType::Const: c = OpClass::Const; break;
+      case NodeType::Unary: c = is_heavy_unop(nd.sub) ? OpClass::HeavyEW : OpClass::LightEW; break;
+      case NodeType::Binary: c = is_heavy_binop(nd.sub) ? OpClass::HeavyEW : OpClass::LightEW; break;
+      case NodeType::Reduce:
+        c = nd.axis == ASTITCH_AXIS_ROW ? OpClass::ReduceRow : OpClass::ReduceCol;
+        break;
+      case NodeType::Bcast:
+        c = nd.axis == ASTITCH_AXIS_ROW ? OpClass::BcastRow : OpClass::BcastCol;
+        break;
+    }
+    info[i].cls = c;
+  }
+
+  // values downstream of a column reduction run after the grid barrier
+  p.colreds.clear();
+  for (int i = 0; i < n; ++i) {
+    const Node& nd = g.nodes[i];
+    if (!info[i].live) continue;
+    bool post = false;
+    if (nd.a >= 0 && info[nd.a].post) post = true;
+    if (nd.b >= 0 && info[nd.b].post) post = true;
+    if (info[i].cls == OpClass::ReduceCol) {
+      if (post) throw Error{ASTITCH_ERR_UNSUPPORTED,
+                            "a column reduction downstream of another column reduction"};
+      post = true;
+      p.colreds.push_back(i);
+    }
+    info[i].post = post;
+  }
+
+  // a2 step 1: dominant candidates = reduces, heavy EW followed by a broadcast,
+  // and the outputs of the stitch op.
+  std::vector<bool> is_output(n, false);
+  for (int o : g.outputs) is_output[o] = true;
+  for (int i = 0; i < n; ++i) {
+    if (!info[i].live) continue;
+    OpClass c = info[i].cls;
+    bool cand = (c == OpClass::ReduceRow || c == OpClass::ReduceCol || is_output[i]);
+    if (c == OpClass::HeavyEW) {
+      for (int u : info[i].consumers)
+        if (info[u].live && (info[u].cls == OpClass::BcastRow || info[u].cls == OpClass::BcastCol))
+          cand = true;
+    }
+    // Reading R17: a value read after the grid barrier (by anything but the
+    // column reduce that accumulates it) has a one-to-many dependency across
+    // groups too, so it is a candidate (power.1 of Fig. 7(a)).
+    if (!info[i].post && c != OpClass::Input && c != OpClass::Const &&
+        (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC)) {
+      for (int u : info[i].consumers)
+        if (info[u].live && info[u].post && info[u].cls != OpClass::ReduceCol) cand = true;
+    }
+    info[i].candidate = cand;
+  }
+
+  // a2 step 2: dominant merging / grouping.  Ops connected through local-only
+  // paths share one schedule.  Two kinds of edges are cut: the
+  // edge into a column reduction (its one-to-many dependency spans all rows,
+  // so its consumers need the grid barrier) and any edge crossing that barrier.
+  DSU dsu(n);
+  for (int i = 0; i < n; ++i) {
+    if (!info[i].live || info[i].cls == OpClass::Const) continue;
+    const Node& nd = g.nodes[i];
+    for (int src : {nd.a, nd.b}) {
+      if (src < 0 || info[src].cls == OpClass::Const) continue;
+      if (info[i].cls == OpClass::ReduceCol) continue;
+      if (!info[src].post && info[i].post) continue;
+      dsu.unite(src, i);
+    }
+  }
+  std::vector<int> gid(n, -1);
+  p.groups.clear();
+  for (int i = 0; i < n; ++i) {
+    if (!info[i].live || info[i].cls == OpClass::Const || info[i].cls == OpClass::Input) continue;
+    int r = dsu.find(i);
+    if (gid[r] < 0) {
+      gid[r] = static_cast<int>(p.groups.size());
+      p.groups.emplace_back();
+    }
+    info[i].group = gid[r];
+    p.groups[gid[r]].push_back(i);
+  }
+  for (int i = 0; i < n; ++i)
+    if (info[i].live && info[i].cls == OpClass::Input && gid[dsu.find(i)] >= 0)
+      info[i].group = gid[dsu.find(i)];
+
+  // final dominant per group: prefer a reduction, column reduce first
+  // (it fixes the whole sweep's mapping), then the first row reduce, then a
+  // heavy-EW candidate, then an output.  Other candidates are sub-dominants.
+  for (auto& grp : p.groups) {
+    int best = -1, best_rank = 99;
+    for (int i : grp) {
+      if (!info[i].candidate) continue;
+      int rank = 9;
+      if (info[i].cls == OpClass::ReduceCol) rank = 0;
+      else if (info[i].cls == OpClass::ReduceRow) rank = 1;
+      else if (info[i].cls == OpClass::HeavyEW) rank = 2;
+      else rank = 3;
+      if (rank < best_rank) { best_rank = rank; best = i; }
+    }
+    for (int i : grp) {
+      if (!info[i].candidate) continue;
+      if (i == best) info[i].dominant = true;
+      else info[i].sub_dominant = true;
+    }
+  }
+
+  // a5: scheme finalisation.  Passive block-locality check for reduce-
+  // dominated groups: a row reduce is produced and consumed by the same row
+  // team inside one block (or one cluster when split) -> regional.  A column
+  // reduce's consumers need every row -> global.  FULL values that cross the
+  // barrier are buffered in HBM -> global.  EW-only groups adapt their mapping
+  // to the producer's (proactive adaptation) and stay local.
+  p.global_fulls.clear();
+  p.post_colvecs.clear();
+  p.needs_sweep2 = false;
+  bool force_global = (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) != 0;
+  for (int i = 0; i < n; ++i) {
+    if (!info[i].live) continue;
+    Scheme s = Scheme::Local;
+    OpClass c = info[i].cls;
+    if (c == OpClass::ReduceRow) s = force_global ? Scheme::Global : Scheme::Regional;
+    else if (c == OpClass::ReduceCol) s = Scheme::Global;
+    else if (c == OpClass::HeavyEW && info[i].candidate && !is_output[i])
+      s = (g.nodes[i].kind == ASTITCH_ROWVEC || g.nodes[i].kind == ASTITCH_COLVEC)
+              ? Scheme::Regional : Scheme::Local;
+    // a pre-barrier FULL / ROWVEC value read after the barrier (by anything
+    // but the column reduction that accumulates it before the barrier)
+    auto used_after_barrier = [&](int v) {
+      for (int u : info[v].consumers)
+        if (info[u].live && info[u].post && info[u].cls != OpClass::ReduceCol) return true;
+      return false;
+    };
+    if (c != OpClass::Const && c != OpClass::Input && !info[i].post &&
+        (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC) && used_after_barrier(i)) {
+      s = Scheme::Global;
+      info[i].global_full = true;
+    }
+    if (c == OpClass::Input && g.nodes[i].kind == ASTITCH_FULL && used_after_barrier(i))
+      info[i].global_full = true;  // re-read from HBM after the barrier
+    bool has_live_consumer = false;
+    for (int u : info[i].consumers) has_live_consumer |= info[u].live;
+    if (is_output[i] && !has_live_consumer && s == Scheme::Local) s = Scheme::Independent;
+    info[i].scheme = s;
+    if (info[i].global_full && c != OpClass::Input) p.global_fulls.push_back(i);
+    if (info[i].post && g.nodes[i].kind == ASTITCH_COLVEC) p.post_colvecs.push_back(i);
+    if (info[i].post && (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC))
+      p.needs_sweep2 = true;
+  }
+  if (force_global)
+    throw Error{ASTITCH_ERR_UNSUPPORTED,
+                "FORCE_GLOBAL ablation (regional -> global demotion) is not implemented yet"};
+}
+
+// ------------------------------------------------------------------------ a3/a4/a6/a7
+namespace {
+
+int pow2_floor(int x) {
+  int r = 1;
+  while (r * 2 <= x) r *= 2;
+  return r;
+}
+
+// Shared-memory bank-conflict degree of a quarter-warp reading 16-byte chunks
+// at a byte stride `stride` (thread-per-row staging, LDS.128).
+int lds128_conflict_ways(int stride) {
+  // LDS.128 serves 8 lanes per wavefront; lanes collide when their 16-byte
+  // bank groups (addr / 16 mod 8) coincide.
+  int cnt[8] = {0};
+  for (int l = 0; l < 8; ++l) cnt[((l * stride) / 16) % 8]++;
+  return *std::max_element(cnt, cnt + 8);
+}
+
+}  // namespace
+
+void select_mapping(Plan& p) {
+  const Graph& g = p.g;
+  Mapping m;
+  const int64_t R = p.desc.rows, C = p.desc.cols;
+  const int sms = p.sm_count;
+  std::ostringstream why;
+
+  // element sizes over FULL tensors (inputs and outputs)
+  int es_min = 16, es_max = 1;
+  bool any_full = false;
+  for (int id : g.inputs) {
+    const Node& nd = g.nodes[id];
+    if (nd.kind == ASTITCH_FULL && p.info[id].live) {
+      es_min = std::min(es_min, dtype_size(nd.dtype));
+      es_max = std::max(es_max, dtype_size(nd.dtype));
+      any_full = true;
+    }
+  }
+  for (size_t k = 0; k < g.outputs.size(); ++k) {
+    if (g.nodes[g.outputs[k]].kind == ASTITCH_FULL) {
+      es_min = std::min(es_min, dtype_size(g.output_dtypes[k]));
+      es_max = std::max(es_max, dtype_size(g.output_dtypes[k]));
+      any_full = true;
+    }
+  }
+  if (!p.global_fulls.empty()) es_max = 4, es_min = std::min(es_min, 4);
+  if (!any_full) es_min = es_max = 4;
+
+  // E: the widest power-of-two vector (<= 16 bytes of the narrowest tensor)
+  // that divides C, so every chunk is aligned and never straddles a row.
+  int E = std::max(1, 16 / es_min);
+  while (E > 1 && (C % E) != 0) E /= 2;
+  m.vec_elems = E;
+  m.chunks = static_cast<int>((C + E - 1) / E);
+  const int chunks = m.chunks;
+  const bool has_mask = g.lengths_node >= 0;
+  const bool has_colred = !p.colreds.empty();
+  const int row_bytes_max = static_cast<int>(std::min<int64_t>(C * es_max, 1 << 30));
+
+  // number of live FULL inputs (memory streams per row)
+  int nfull_in = 0;
+  for (int id : g.inputs)
+    if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live) ++nfull_in;
+  nfull_in = std::max(nfull_in, 1);
+
+  // Team choice: lanes T (power of two) x chunks per lane V, T*V >= chunks.
+  // Score: lane utilisation first, then per-lane elements near the target
+  // (enough bytes in flight, few registers), then fewer lanes (cheaper team
+  // reduction).  Depends on C and dtypes only, never on R, so a row's
+  // reduction tree is identical for every shard (reading R13).
+  auto choose_team = [&](int max_team, int target_ne, int max_ne) {
+    int bestT = 1, bestV = chunks;
+    double best_score = -1e30;
+    for (int T = 1; T <= max_team; T *= 2) {
+      int V = (chunks + T - 1) / T;
+      int ne = V * E;
+      if (ne > max_ne && T < max_team) continue;
+      double util = static_cast<double>(chunks) / (T * V);
+      double score = util * 100.0 - std::fabs(std::log2(static_cast<double>(ne) / target_ne)) * 4.0 -
+                     (T > 32 ? 6.0 : 0.0) - (T < 4 ? 3.0 : 0.0);
+      if (score > best_score) { best_score = score; bestT = T; bestV = V; }
+    }
+    m.team = bestT;
+    m.chunks_per_lane = bestV;
+    m.lane_util = static_cast<double>(chunks) / (bestT * bestV);
+  };
+
+  bool no_pack = (p.desc.flags & ASTITCH_FLAG_NO_PACK) != 0;
+  bool no_split = (p.desc.flags & ASTITCH_FLAG_NO_SPLIT) != 0;
+  bool no_tma = (p.desc.flags & ASTITCH_FLAG_NO_TMA) != 0;
+  m.prefetch = (p.desc.flags & ASTITCH_FLAG_NO_PREFETCH) == 0;
+
+  // Blocks-per-wave reference for the paper's shape rule: the number
+  // of 1024-thread-equivalent blocks the chip runs at once = 2 per SM.
+  const int64_t blocks_per_wave_1024 = 2LL * sms;
+
+  if (has_colred) {
+    // ---------------------------------------------------------- global sweep
+    // Column reductions (K3) need all rows: a one-wave persistent grid sweeps
+    // the rows (vertical packing), each lane keeps fp32 column
+    // partials in registers, blocks combine in smem, then the grid barrier
+    // and a deterministic fixed-order final combine.
+    m.tmpl = Template::GlobalSweep;
+    choose_team(1024, 8, 16);
+    if (no_pack && m.team < 32) { m.team = 32; m.chunks_per_lane = (chunks + 31) / 32; }
+    bool has_rowred = false;
+    for (size_t i = 0; i < g.nodes.size(); ++i)
+      if (p.info[i].live && p.info[i].cls == OpClass::ReduceRow) has_rowred = true;
+    // a multi-warp team reduces through block-wide smem: one team per block
+    m.threads = (m.team > 32 && has_rowred) ? m.team : std::max(512, m.team);
+    m.rows_per_block = m.threads / m.team;
+    int ne = m.chunks_per_lane * E;
+    m.row_unroll = std::max(1, std::min(4, 32 / std::max(1, ne * nfull_in)));
+    // a6: block-level combine of the teams' column partials in smem
+    if (m.rows_per_block > 1) {
+      int64_t cb = static_cast<int64_t>(m.rows_per_block) * m.team * m.chunks_per_lane * E * 4;
+      if (cb <= 96 * 1024) m.smem_bytes = static_cast<int>(cb);
+    }
+    why << "column reduce -> global sweep (vertical packing, grid barrier); ";
+  } else {
+    // ---------------------------------------------------------- row-wise
+    choose_team(1024, 16, 32);
+    if (no_pack && m.team < 32 && chunks >= 1) {
+      // ablation: XLA-style one row per warp (no horizontal packing)
+      m.team = 32;
+      m.chunks_per_lane = (chunks + 31) / 32;
+      m.lane_util = static_cast<double>(chunks) / (32 * m.chunks_per_lane);
+    }
+    bool row16 = true;  // every FULL row is a multiple of 16 bytes
+    for (int id : g.inputs)
+      if (g.nodes[id].kind == ASTITCH_FULL && (C * dtype_size(g.nodes[id].dtype)) % 16) row16 = false;
+    for (size_t k = 0; k < g.outputs.size(); ++k)
+      if (g.nodes[g.outputs[k]].kind == ASTITCH_FULL && (C * dtype_size(g.output_dtypes[k])) % 16)
+        row16 = false;
+    bool has_colvec_in = false;
+    for (int id : g.inputs)
+      if (g.nodes[id].kind == ASTITCH_COLVEC && p.info[id].live) has_colvec_in = true;
+    // Horizontal packing of many tiny rows: when a row is too
+    // short for a power-of-two team to tile it (e.g. 9 x 16-byte chunks),
+    // stage row tiles in smem with TMA bulk copies and give each thread a row.
+    bool packed_ok = !no_tma && !no_pack && !has_mask && row16 && !has_colvec_in &&
+                     row_bytes_max <= 512 && m.lane_util < 0.95 && chunks <= 32 &&
+                     p.global_fulls.empty() && R >= 4096;
+    // Task splitting (rule P:L270): rows < blocks-per-wave and row > 1024.
+    bool split_rule = !no_split && R < blocks_per_wave_1024 && C > 1024;
+    if (packed_ok) {
+      m.tmpl = Template::PackedTile;
+      m.team = 1;
+      m.chunks_per_lane = chunks;
+      m.lane_util = 1.0;
+      m.threads = 128;
+      m.tile_rows = 128;
+      m.stages = 4;  // prefetch distance 2 tiles + 2 tiles draining (bulk stores)
+      m.rows_per_block = m.tile_rows;
+      // stage bytes: input tiles + output tiles that cannot be written in
+      // place over an input tile of the same element size (mirrors codegen)
+      int in_bytes = 0, out_bytes = 0;
+      std::vector<int> in_sizes;
+      for (int id : g.inputs)
+        if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live) {
+          in_bytes += static_cast<int>(C) * dtype_size(g.nodes[id].dtype);
+          in_sizes.push_back(dtype_size(g.nodes[id].dtype));
+        }
+      for (size_t k = 0; k < g.outputs.size(); ++k)
+        if (g.nodes[g.outputs[k]].kind == ASTITCH_FULL) {
+          int es = dtype_size(g.output_dtypes[k]);
+          auto it = std::find(in_sizes.begin(), in_sizes.end(), es);
+          if (it != in_sizes.end()) in_sizes.erase(it);
+          else out_bytes += static_cast<int>(C) * es;
+        }
+      m.smem_bytes = m.stages * m.tile_rows * (in_bytes + out_bytes) + 64 * m.stages;
+      while (m.smem_bytes > 200 * 1024 && m.stages > 2) {
+        m.stages--;
+        m.smem_bytes = m.stages * m.tile_rows * (in_bytes + out_bytes) + 64 * m.stages;
+      }
+      m.bank_conflict_ways = lds128_conflict_ways(static_cast<int>(C) * es_min);
+      why << "row of " << chunks << " x " << (E * es_min)
+          << "B chunks does not tile a power-of-two team -> TMA-staged packed tiles, thread per row; ";
+    } else {
+      m.tmpl = Template::RowTeam;
+      if (split_rule) {
+        m.split = static_cast<int>(std::max<int64_t>(2, (blocks_per_wave_1024 + R - 1) / std::max<int64_t>(R, 1)));
+        m.split = std::min(m.split, 8);
+        why << "paper split rule holds (rows " << R << " < per-wave " << blocks_per_wave_1024
+            << " and row " << C << " > 1024): split factor " << m.split
+            << " requested; executed as one block team per row (cluster split is NEXT f2); ";
+        m.split = 1;
+      }
+      // a multi-warp team reduces through block-wide smem: one team per block
+      m.threads = m.team > 32 ? m.team : 256;
+      m.rows_per_block = m.threads / m.team;
+      m.row_unroll = 1;
+      why << "row team of " << m.team << " lanes x " << m.chunks_per_lane << " chunks ("
+          << m.rows_per_block << " rows / block, packing), regional via shuffles" << (m.team > 32 ? "+smem" : "")
+          << "; ";
+    }
+  }
+
+  // colvec operands: hoist in registers when the footprint is small (a6)
+  {
+    int ncv = 0;
+    for (int i = 0; i < static_cast<int>(g.nodes.size()); ++i)
+      if (p.info[i].live && !p.info[i].post && g.nodes[i].kind == ASTITCH_COLVEC) ++ncv;
+    m.hoist_colvec = (ncv * m.chunks_per_lane * E) <= 48;
+  }
+
+  // a7: assume-relax-apply.  Assume the 32-register bound (full occupancy),
+  // compute blocks per SM from threads and smem, relax the register cap to the
+  // largest value that keeps those blocks resident; the caller
+  // recompiles with a lower target if ptxas reports spills.
+  int by_threads = 2048 / m.threads;
+  int by_smem = m.smem_bytes > 0 ? (228 * 1024) / (m.smem_bytes + 1024) : 32;
+  m.blocks_per_sm = std::max(1, std::min({32, by_threads, by_smem}));
+  m.reg_cap = std::min(255, (65536 / (m.blocks_per_sm * m.threads)) & ~7);
+
+  m.reason = why.str();
+  p.map = m;
+  retune_grid(p);
+}
+
+// grid: one wave (persistent, vertical packing); never more blocks
+// than there is work.  Recomputed whenever blocks_per_sm is relaxed.
+void retune_grid(Plan& p) {
+  Mapping& m = p.map;
+  const int64_t R = p.desc.rows;
+  int64_t work_units = 0;
+  if (m.tmpl == Template::PackedTile) work_units = (R + m.tile_rows - 1) / m.tile_rows;
+  else work_units = (R + (int64_t)m.rows_per_block * m.row_unroll - 1) / ((int64_t)m.rows_per_block * m.row_unroll);
+  int64_t wave = static_cast<int64_t>(m.blocks_per_sm) * p.sm_count;
+  m.grid = std::max<int64_t>(1, std::min(work_units, wave));
+  m.vertical_trips = (work_units + m.grid - 1) / m.grid;
+  plan_workspace(p);
+}
+
+// ------------------------------------------------------------------------ a6 workspace
+void plan_workspace(Plan& p) {
+  WsLayout w;
+  size_t off = 0;
+  auto align = [](size_t x) { return (x + 255) & ~static_cast<size_t>(255); };
+  const int64_t C = p.desc.cols, R = p.desc.rows;
+  if (p.map.tmpl == Template::GlobalSweep) {
+    w.barrier = off;
+    off = align(off + 256);
+    w.partials = off;
+    off = align(off + static_cast<size_t>(p.map.grid) * p.colreds.size() * C * 4);
+    w.colvals = off;
+    off = align(off + std::max<size_t>(p.post_colvecs.size(), 1) * C * 4 + C * 4 * p.colreds.size());
+    w.globals = off;
+    off = align(off + p.global_fulls.size() * static_cast<size_t>(R) * C * 4);
+  }
+  w.total = off;
+  p.ws = w;
+}
+
+uint64_t compulsory_bytes(const Plan& p) {
+  const Graph& g = p.g;
+  const uint64_t R = p.desc.rows, C = p.desc.cols;
+  uint64_t b = 0;
+  for (int id : g.inputs) {
+    const Node& nd = g.nodes[id];
+    if (!p.info[id].live) continue;
+    uint64_t es = dtype_size(nd.dtype);
+    if (nd.kind == ASTITCH_FULL) b += R * C * es;
+    else if (nd.kind == ASTITCH_ROWVEC) b += R * es;
+    else if (nd.kind == ASTITCH_COLVEC) b += C * es;
+    else if (nd.kind == ASTITCH_LENGTHS)
+      b += 4 * ((R + g.rows_per_segment - 1) / std::max<int64_t>(g.rows_per_segment, 1));
+  }
+  for (size_t k = 0; k < g.outputs.size(); ++k) {
+    uint64_t es = dtype_size(g.output_dtypes[k]);
+    astitch_kind kd = g.nodes[g.outputs[k]].kind;
+    if (kd == ASTITCH_FULL) b += R * C * es;
+    else if (kd == ASTITCH_ROWVEC) b += R * es;
+    else b += C * es;
+  }
+  return b;
+}
+
+// ------------------------------------------------------------------------ describe
+std::string describe_json(const Plan& p) {
+  std::ostringstream o;
+  const Graph& g = p.g;
+  const Mapping& m = p.map;
+  auto esc = [](const std::string& s) {
+    std::string r;
+    for (char c : s) {
+      if (c == '"' || c == '\\') r += '\\';
+      if (c == '\n') { r += "\\n"; continue; }
+      r += c;
+    }
+    return r;
+  };
+  o << "{\"rows\":" << p.desc.rows << ",\"cols\":" << p.desc.cols << ",\"device\":" << p.desc.device
+    << ",\"shard_rank\":" << p.desc.shard_rank << ",\"shard_world\":" << p.desc.shard_world
+    << ",\"sm_count\":" << p.sm_count;
+  o << ",\"ops\":[";
+  for (size_t i = 0; i < g.nodes.size(); ++i) {
+    const Node& nd = g.nodes[i];
+    const NodeInfo& in = p.info[i];
+    if (i) o << ",";
+    o << "{\"id\":" << i << ",\"class\":\"" << opclass_name(in.cls) << "\",\"kind\":\""
+      << kind_name(nd.kind) << "\"";
+    if (nd.type == NodeType::Unary) o << ",\"op\":\"" << unop_name(nd.sub) << "\"";
+    if (nd.type == NodeType::Binary) o << ",\"op\":\"" << binop_name(nd.sub) << "\"";
+    if (nd.type == NodeType::Reduce) o << ",\"op\":\"" << (nd.sub == ASTITCH_SUM ? "SUM" : "RMAX") << "\"";
+    if (nd.a >= 0) o << ",\"a\":" << nd.a;
+    if (nd.b >= 0) o << ",\"b\":" << nd.b;
+    o << ",\"live\":" << (in.live ? "true" : "false") << ",\"post_barrier\":" << (in.post ? "true" : "false")
+      << ",\"candidate\":" << (in.candidate ? "true" : "false")
+      << ",\"dominant\":" << (in.dominant ? "true" : "false")
+      << ",\"sub_dominant\":" << (in.sub_dominant ? "true" : "false") << ",\"group\":" << in.group
+      << ",\"scheme\":\"" << scheme_name(in.scheme) << "\"}";
+  }
+  o << "],\"groups\":[";
+  for (size_t k = 0; k < p.groups.size(); ++k) {
+    if (k) o << ",";
+    o << "[";
+    for (size_t j = 0; j < p.groups[k].size(); ++j) o << (j ? "," : "") << p.groups[k][j];
+    o << "]";
+  }
+  o << "],\"mapping\":{\"template\":\"" << template_name(m.tmpl) << "\",\"vec_elems\":" << m.vec_elems
+    << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
+    << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads
+    << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
+    << ",\"prefetch\":" << (m.prefetch ? "true" : "false")
+    << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
+    << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"grid\":" << m.grid
+    << ",\"blocks_per_sm\":" << m.blocks_per_sm << ",\"reg_cap\":" << m.reg_cap
+    << ",\"vertical_trips\":" << m.vertical_trips << ",\"smem_bytes\":" << m.smem_bytes
+    << ",\"lds128_conflict_ways\":" << m.bank_conflict_ways << ",\"reason\":\"" << esc(m.reason)
+    << "\"}";
+  o << ",\"workspace\":{\"total\":" << p.ws.total << ",\"barrier\":" << p.ws.barrier
+    << ",\"partials\":" << p.ws.partials << ",\"colvals\":" << p.ws.colvals << ",\"globals\":" << p.ws.globals
+    << "}";
+  o << ",\"global_fulls\":[";
+  for (size_t k = 0; k < p.global_fulls.size(); ++k) o << (k ? "," : "") << p.global_fulls[k];
+  o << "],\"needs_sweep2\":" << (p.needs_sweep2 ? "true" : "false");
+  o << ",\"kernel_count\":" << p.kernels.size() << ",\"memsets_per_run\":0";
+  o << ",\"kernels\":[";
+  for (size_t k = 0; k < p.kernels.size(); ++k) {
+    const Kernel& kk = p.kernels[k];
+    if (k) o << ",";
+    o << "{\"name\":\"" << kk.name << "\",\"threads\":" << kk.threads << ",\"grid\":" << kk.grid
+      << ",\"smem\":" << kk.smem << ",\"cooperative\":" << (kk.cooperative ? "true" : "false")
+      << ",\"regs\":" << kk.regs << ",\"spill_bytes\":" << kk.spill_bytes
+      << ",\"occupancy_blocks_per_sm\":" << kk.occupancy << ",\"cubin_bytes\":" << kk.cubin.size() << "}";
+  }
+  o << "],\"shard_kernels\":" << p.shard_kernels.size();
+  o << ",\"compulsory_bytes\":" << p.compulsory_bytes << "}";
+  return o.str();
+}
+
+}  // namespace astitch

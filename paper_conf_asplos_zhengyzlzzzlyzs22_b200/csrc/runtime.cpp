@@ -1,0 +1,447 @@
+// Plan construction (JIT) and execution entry points of the C ABI.
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <regex>
+#include <string>
+
+#include "internal.h"
+
+using namespace astitch;
+
+namespace {
+
+uint64_t fnv1a(const std::string& s) {
+  uint64_t h = 1469598103934665603ULL;
+  for (unsigned char c : s) {
+    h ^= c;
+    h *= 1099511628211ULL;
+  }
+  return h;
+}
+
+void parse_ptxas(Kernel& k) {
+  std::smatch mt;
+  std::regex rr("Used ([0-9]+) registers");
+  if (std::regex_search(k.log, mt, rr)) k.regs = std::stoi(mt[1]);
+  std::regex rs("([0-9]+) bytes spill stores");
+  if (std::regex_search(k.log, mt, rs)) k.spill_bytes = std::stoi(mt[1]);
+}
+
+size_t io_bytes(const Plan& p, int node, astitch_dtype dt) {
+  const Node& nd = p.g.nodes[node];
+  const size_t R = static_cast<size_t>(p.desc.rows), C = static_cast<size_t>(p.desc.cols);
+  const size_t es = dtype_size(dt);
+  switch (nd.kind) {
+    case ASTITCH_FULL: return R * C * es;
+    case ASTITCH_ROWVEC: return R * es;
+    case ASTITCH_COLVEC: return C * es;
+    case ASTITCH_LENGTHS: {
+      size_t rps = static_cast<size_t>(p.g.rows_per_segment);
+      return 4 * ((R + rps - 1) / rps);
+    }
+    default: return 0;
+  }
+}
+
+const char* role_suffix(int role) {
+  switch (role) {
+    case ROLE_MAIN: return "";
+    case ROLE_SHARD_MAIN: return "_shard";
+    case ROLE_SHARD_FINAL: return "_shard_final";
+    case ROLE_SHARD_SWEEP2: return "_shard_sweep2";
+  }
+  return "";
+}
+
+// Build (generate + compile + load) one kernel of the plan.  Applies the
+// assume-relax-apply loop: if ptxas spills under the assumed
+// register bound, relax the target blocks per SM and recompile.
+astitch_status build_kernel(Plan& p, int role, Kernel& k) {
+  const bool compile = (p.desc.flags & ASTITCH_FLAG_NO_COMPILE) == 0;
+  const bool may_relax = (role == ROLE_MAIN);  // later kernels share the main kernel's layout
+  for (int attempt = 0; attempt < 3; ++attempt) {
+    std::string base = std::string("astitch_") + template_name(p.map.tmpl) + role_suffix(role);
+    k.name = base;
+    k.source = generate_kernel(p, role, base);
+    char hb[32];
+    snprintf(hb, sizeof(hb), "_%012llx", static_cast<unsigned long long>(fnv1a(k.source) & 0xffffffffffffULL));
+    // give each specialisation a unique, recognisable symbol
+    std::string uniq = base + hb;
+    size_t pos = k.source.find(" " + base + "(");
+    if (pos != std::string::npos) k.source.replace(pos + 1, base.size(), uniq);
+    k.name = uniq;
+    k.threads = (role == ROLE_SHARD_FINAL) ? 256 : p.map.threads;
+    k.grid = (role == ROLE_SHARD_FINAL) ? std::max<int64_t>(1, (p.desc.cols + 255) / 256) : p.map.grid;
+    k.smem = (role == ROLE_SHARD_FINAL) ? 0 : p.map.smem_bytes;
+    k.cooperative = (p.map.tmpl == Template::GlobalSweep) && (role == ROLE_MAIN || role == ROLE_SHARD_MAIN);
+    if (!compile) return ASTITCH_OK;
+    std::string err;
+    if (!nvrtc_compile(k.source, k.name, k.cubin, k.log, err)) return fail(ASTITCH_ERR_CUDA, err);
+    parse_ptxas(k);
+    if (k.spill_bytes > 0 && p.map.blocks_per_sm > 1 && may_relax) {
+      // relax: compile once without the occupancy bound to learn the natural
+      // register demand, then apply the largest occupancy that fits it.
+      if (attempt == 0) {
+        Plan probe = p;
+        probe.map.blocks_per_sm = 1;
+        std::string src = generate_kernel(probe, role, base);
+        Kernel kp;
+        kp.name = base;
+        std::string e2;
+        if (!nvrtc_compile(src, base, kp.cubin, kp.log, e2)) return fail(ASTITCH_ERR_CUDA, e2);
+        parse_ptxas(kp);
+        int regs = std::max(32, (kp.regs + 7) & ~7);
+        int bps = std::max(1, std::min(p.map.blocks_per_sm - 1, 65536 / (regs * p.map.threads)));
+        p.map.blocks_per_sm = bps;
+      } else {
+        p.map.blocks_per_sm = std::max(1, p.map.blocks_per_sm - 1);
+      }
+      p.map.reg_cap = std::min(255, (65536 / (p.map.blocks_per_sm * p.map.threads)) & ~7);
+      retune_grid(p);
+      continue;
+    }
+    return ASTITCH_OK;
+  }
+  return ASTITCH_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+astitch_status astitch_plan(astitch_graph_t gr, const astitch_plan_desc* desc, astitch_plan_t* out) {
+  if (!gr || !desc || !out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL graph, desc or out");
+  *out = nullptr;
+  if (desc->rows < 0) return fail(ASTITCH_ERR_SHAPE, "rows < 0");
+  if (desc->cols < 1) return fail(ASTITCH_ERR_SHAPE, "cols < 1");
+  if (desc->cols > (1LL << 31) || desc->rows > (1LL << 40) ||
+      static_cast<double>(desc->rows) * static_cast<double>(desc->cols) > 4.0e12)
+    return fail(ASTITCH_ERR_SHAPE, "shape too large");
+  if (desc->shard_world < 0 || (desc->shard_world > 0 && (desc->shard_rank < 0 || desc->shard_rank >= desc->shard_world)))
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad shard_rank / shard_world");
+  if (gr->g.outputs.empty()) return fail(ASTITCH_ERR_INVALID_GRAPH, "graph has no outputs");
+  try {
+    auto plan = std::make_unique<Plan>();
+    Plan& p = *plan;
+    p.g = gr->g;
+    p.desc = *desc;
+    if (p.desc.shard_world == 0) p.desc.shard_world = 1;
+    p.device = desc->device;
+    p.sm_count = desc->sm_count > 0 ? desc->sm_count : 148;
+    if (p.device >= 0) {
+      std::string err;
+      int sms = 0, smem_optin = 0;
+      if (!drv_device_info(p.device, sms, smem_optin, err)) return fail(ASTITCH_ERR_CUDA, err);
+      if (desc->sm_count <= 0) p.sm_count = sms;
+    }
+    analyse(p);
+    select_mapping(p);
+    plan_workspace(p);
+    p.compulsory_bytes = compulsory_bytes(p);
+
+    std::vector<int> roles = {ROLE_MAIN};
+    p.kernels.resize(1);
+    astitch_status s = build_kernel(p, ROLE_MAIN, p.kernels[0]);
+    if (s != ASTITCH_OK) return s;
+    if (p.map.tmpl == Template::GlobalSweep && p.desc.shard_world > 1) {
+      std::vector<int> sr = {ROLE_SHARD_MAIN, ROLE_SHARD_FINAL};
+      if (p.needs_sweep2) sr.push_back(ROLE_SHARD_SWEEP2);
+      p.shard_kernels.resize(sr.size());
+      for (size_t i = 0; i < sr.size(); ++i) {
+        s = build_kernel(p, sr[i], p.shard_kernels[i]);
+        if (s != ASTITCH_OK) return s;
+      }
+    }
+    // workspace offsets are baked into the sources: keep the layout computed
+    // for the planned (maximum) grid; the launch grid may only shrink.
+    if (p.device >= 0 && (p.desc.flags & ASTITCH_FLAG_NO_COMPILE) == 0) {
+      auto load = [&](Kernel& k) -> astitch_status {
+        std::string err;
+        if (!drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
+        if (k.cooperative) {
+          int64_t max_grid = static_cast<int64_t>(k.occupancy) * p.sm_count;
+          if (max_grid < 1)
+            return fail(ASTITCH_ERR_RESOURCE, "kernel " + k.name + " cannot be resident (occupancy 0)");
+          if (k.grid > max_grid) k.grid = max_grid;
+        }
+        return ASTITCH_OK;
+      };
+      for (auto& k : p.kernels)
+        if ((s = load(k)) != ASTITCH_OK) return s;
+      for (auto& k : p.shard_kernels)
+        if ((s = load(k)) != ASTITCH_OK) return s;
+    }
+    p.describe = describe_json(p);
+    auto* h = new astitch_plan_s();
+    h->p = std::move(plan);
+    *out = h;
+    set_error("");
+    return ASTITCH_OK;
+  } catch (const Error& e) {
+    return fail(e.status, e.msg);
+  } catch (const std::exception& e) {
+    return fail(ASTITCH_ERR_INTERNAL, e.what());
+  }
+}
+
+astitch_status astitch_plan_destroy(astitch_plan_t h) {
+  if (!h) return ASTITCH_OK;
+  for (auto& k : h->p->kernels) drv_unload(k);
+  for (auto& k : h->p->shard_kernels) drv_unload(k);
+  delete h;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_plan_workspace_bytes(astitch_plan_t h, size_t* bytes) {
+  if (!h || !bytes) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan or bytes");
+  *bytes = h->p->ws.total;
+  return ASTITCH_OK;
+}
+
+static astitch_status copy_out(const std::string& s, char* buf, size_t cap, size_t* len) {
+  if (len) *len = s.size();
+  if (buf && cap > 0) {
+    size_t n = std::min(cap - 1, s.size());
+    memcpy(buf, s.data(), n);
+    buf[n] = '\0';
+  }
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_plan_describe(astitch_plan_t h, char* json, size_t cap, size_t* len) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  return copy_out(h->p->describe, json, cap, len);
+}
+
+static const Kernel* kernel_at(const Plan& p, int32_t k) {
+  if (k < 0) return nullptr;
+  if (k < static_cast<int32_t>(p.kernels.size())) return &p.kernels[k];
+  k -= static_cast<int32_t>(p.kernels.size());
+  if (k < static_cast<int32_t>(p.shard_kernels.size())) return &p.shard_kernels[k];
+  return nullptr;
+}
+
+astitch_status astitch_plan_source(astitch_plan_t h, int32_t k, char* buf, size_t cap, size_t* len) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  const Kernel* kk = kernel_at(*h->p, k);
+  if (!kk) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "kernel index out of range");
+  return copy_out(kk->source, buf, cap, len);
+}
+
+astitch_status astitch_plan_cubin(astitch_plan_t h, int32_t k, void* buf, size_t cap, size_t* len) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  const Kernel* kk = kernel_at(*h->p, k);
+  if (!kk) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "kernel index out of range");
+  if (len) *len = kk->cubin.size();
+  if (buf && cap >= kk->cubin.size()) memcpy(buf, kk->cubin.data(), kk->cubin.size());
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_plan_kernel_count(astitch_plan_t h, int32_t* n) {
+  if (!h || !n) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan or n");
+  *n = static_cast<int32_t>(h->p->kernels.size());
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_plan_io_count(astitch_plan_t h, int32_t* ni, int32_t* no) {
+  if (!h || !ni || !no) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  *ni = static_cast<int32_t>(h->p->g.inputs.size());
+  *no = static_cast<int32_t>(h->p->g.outputs.size());
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_plan_io(astitch_plan_t h, int32_t is_output, int32_t index, astitch_kind* kind,
+                               astitch_dtype* dtype) {
+  if (!h || !kind || !dtype) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  const Graph& g = h->p->g;
+  if (is_output) {
+    if (index < 0 || index >= static_cast<int32_t>(g.outputs.size()))
+      return fail(ASTITCH_ERR_INVALID_ARGUMENT, "output index out of range");
+    *kind = g.nodes[g.outputs[index]].kind;
+    *dtype = g.output_dtypes[index];
+  } else {
+    if (index < 0 || index >= static_cast<int32_t>(g.inputs.size()))
+      return fail(ASTITCH_ERR_INVALID_ARGUMENT, "input index out of range");
+    *kind = g.nodes[g.inputs[index]].kind;
+    *dtype = g.nodes[g.inputs[index]].dtype;
+  }
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_workspace_init(astitch_plan_t h, void* ws, void* stream) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  const Plan& p = *h->p;
+  if (p.ws.total == 0) return ASTITCH_OK;
+  if (!ws) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "plan needs a workspace");
+  std::string err;
+  if (!drv_memset_async(static_cast<char*>(ws) + p.ws.barrier, 256, stream, err))
+    return fail(ASTITCH_ERR_CUDA, err);
+  return ASTITCH_OK;
+}
+
+}  // extern "C"
+
+namespace astitch {
+
+astitch_status check_io(const Plan& p, const void* const* inputs, void* const* outputs, void* ws) {
+  const Graph& g = p.g;
+  if (!inputs && !g.inputs.empty()) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "inputs is NULL");
+  if (!outputs) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "outputs is NULL");
+  for (size_t i = 0; i < g.inputs.size(); ++i) {
+    if (!inputs[i]) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "input " + std::to_string(i) + " is NULL");
+    if (reinterpret_cast<uintptr_t>(inputs[i]) % 16)
+      return fail(ASTITCH_ERR_INVALID_ARGUMENT, "input " + std::to_string(i) + " is not 16-byte aligned");
+  }
+  for (size_t i = 0; i < g.outputs.size(); ++i) {
+    if (!outputs[i]) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "output " + std::to_string(i) + " is NULL");
+    if (reinterpret_cast<uintptr_t>(outputs[i]) % 16)
+      return fail(ASTITCH_ERR_INVALID_ARGUMENT, "output " + std::to_string(i) + " is not 16-byte aligned");
+  }
+  if (p.ws.total > 0 && !ws) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "plan needs a workspace");
+  if (ws && reinterpret_cast<uintptr_t>(ws) % 256) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "workspace not 256-byte aligned");
+  if (p.kernels.empty() || !p.kernels[0].function)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "plan was built without a device (device = -1 or NO_COMPILE)");
+  return ASTITCH_OK;
+}
+
+KernelParams make_params(const Plan& p, const void* const* inputs, void* const* outputs, void* ws) {
+  KernelParams kp;
+  memset(&kp, 0, sizeof(kp));
+  for (size_t i = 0; i < p.g.inputs.size(); ++i) kp.in[i] = inputs[i];
+  for (size_t i = 0; i < p.g.outputs.size(); ++i) kp.out[i] = outputs[i];
+  kp.ws = ws;
+  kp.rows = p.desc.rows;
+  kp.row_offset = 0;
+  return kp;
+}
+
+astitch_status launch(const Plan& p, const Kernel& k, KernelParams& kp, void* stream) {
+  std::string err;
+  if (!drv_launch(k, &kp, sizeof(kp), stream, err)) return fail(ASTITCH_ERR_CUDA, err);
+  if (p.desc.flags & ASTITCH_FLAG_LAUNCH_CHECK) {
+    if (!drv_sync(stream, err)) return fail(ASTITCH_ERR_CUDA, err);
+  }
+  return ASTITCH_OK;
+}
+
+}  // namespace astitch
+
+extern "C" {
+
+astitch_status astitch_run(astitch_plan_t h, const void* const* inputs, void* const* outputs, void* ws,
+                           void* stream) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  const Plan& p = *h->p;
+  if (p.desc.rows == 0) return ASTITCH_OK;
+  astitch_status s = check_io(p, inputs, outputs, ws);
+  if (s != ASTITCH_OK) return s;
+  KernelParams kp = make_params(p, inputs, outputs, ws);
+  for (const Kernel& k : p.kernels)
+    if ((s = launch(p, k, kp, stream)) != ASTITCH_OK) return s;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_run_host(astitch_plan_t h, const void* const* host_inputs, void* const* host_outputs,
+                                const void* const* dev_inputs, void* const* dev_outputs, void* ws, void* stream) {
+  if (!h || !host_inputs || !host_outputs || !dev_inputs || !dev_outputs)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  const Plan& p = *h->p;
+  if (p.desc.rows == 0) return ASTITCH_OK;
+  std::string err;
+  for (size_t i = 0; i < p.g.inputs.size(); ++i) {
+    int node = p.g.inputs[i];
+    size_t nbytes = io_bytes(p, node, p.g.nodes[node].dtype);
+    if (!host_inputs[i]) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "host input NULL");
+    if (!drv_memcpy_async(const_cast<void*>(dev_inputs[i]), host_inputs[i], nbytes, 1, stream, err))
+      return fail(ASTITCH_ERR_CUDA, err);
+  }
+  astitch_status s = astitch_run(h, dev_inputs, dev_outputs, ws, stream);
+  if (s != ASTITCH_OK) return s;
+  for (size_t i = 0; i < p.g.outputs.size(); ++i) {
+    size_t nbytes = io_bytes(p, p.g.outputs[i], p.g.output_dtypes[i]);
+    if (!host_outputs[i]) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "host output NULL");
+    if (!drv_memcpy_async(host_outputs[i], dev_outputs[i], nbytes, 2, stream, err))
+      return fail(ASTITCH_ERR_CUDA, err);
+  }
+  return ASTITCH_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------------------ measurement aids
+namespace {
+struct BenchModule {
+  Kernel barrier, copy;
+  bool ok = false;
+};
+std::mutex g_bench_mu;
+BenchModule g_bench[64];
+
+astitch_status bench_module(int device, BenchModule*& out) {
+  if (device < 0 || device >= 64) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad device");
+  std::lock_guard<std::mutex> lk(g_bench_mu);
+  BenchModule& b = g_bench[device];
+  if (!b.ok) {
+    std::string err, log;
+    std::vector<char> cubin;
+    std::string src = "#include \"astitch_device.cuh\"\n";
+    if (!nvrtc_compile(src, "astitch_bench", cubin, log, err)) return fail(ASTITCH_ERR_CUDA, err);
+    Plan tmp;
+    tmp.device = device;
+    b.barrier.cubin = cubin;
+    b.barrier.name = "astitch_barrier_bench";
+    b.barrier.threads = 1024;
+    b.copy.cubin = cubin;
+    b.copy.name = "astitch_copy_bench";
+    b.copy.threads = 256;
+    if (!drv_load(tmp, b.barrier, err)) return fail(ASTITCH_ERR_CUDA, err);
+    if (!drv_load(tmp, b.copy, err)) return fail(ASTITCH_ERR_CUDA, err);
+    b.ok = true;
+  }
+  out = &b;
+  return ASTITCH_OK;
+}
+}  // namespace
+
+extern "C" {
+
+astitch_status astitch_bench_barrier(int32_t device, int32_t blocks, int32_t threads, int32_t iters, void* ws,
+                                     void* stream) {
+  if (blocks < 1 || threads < 32 || threads > 1024 || iters < 0 || !ws)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad barrier bench arguments");
+  BenchModule* b = nullptr;
+  astitch_status s = bench_module(device, b);
+  if (s != ASTITCH_OK) return s;
+  Kernel k = b->barrier;
+  k.grid = blocks;
+  k.threads = threads;
+  k.cooperative = true;
+  void* bar = ws;
+  int it = iters;
+  void* argv[] = {&bar, &it};
+  std::string err;
+  if (!drv_launch_args(k, argv, stream, err)) return fail(ASTITCH_ERR_CUDA, err);
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_bench_copy(int32_t device, const void* src, void* dst, size_t bytes, void* stream) {
+  if (!src || !dst || bytes % 16) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad copy arguments");
+  BenchModule* b = nullptr;
+  astitch_status s = bench_module(device, b);
+  if (s != ASTITCH_OK) return s;
+  Kernel k = b->copy;
+  k.threads = 256;
+  int sms = 148, smem = 0;
+  std::string err;
+  drv_device_info(device, sms, smem, err);
+  k.grid = static_cast<int64_t>(sms) * 8;
+  long long n16 = static_cast<long long>(bytes / 16);
+  const void* s_ = src;
+  void* d_ = dst;
+  void* argv[] = {&s_, &d_, &n16};
+  if (!drv_launch_args(k, argv, stream, err)) return fail(ASTITCH_ERR_CUDA, err);
+  return ASTITCH_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,131 @@
+"""Host-only tests of the C-ABI library: it loads without a GPU, exports every
+symbol include/astitch.h declares, and returns the documented status codes."""
+
+import ctypes as ct
+import os
+import re
+
+import pytest
+
+import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+from paper_conf_asplos_zhengyzlzzzlyzs22_b200 import _lib
+from workloads import specs
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    text = open(os.path.join(ROOT, "include", "astitch.h")).read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    return sorted(set(re.findall(r"\b(astitch_[a-z_]+)\s*\(", text)))
+
+
+def test_library_exports_every_header_symbol():
+    syms = header_symbols()
+    assert len(syms) >= 30
+    for s in syms:
+        assert hasattr(_lib.lib, s), f"libastitch.so does not export {s}"
+    assert set(syms) == set(_lib.EXPORTED)
+    assert _lib.lib.astitch_abi_version() == 1
+
+
+def test_library_has_no_cuda_link_dependency():
+    # libcuda / libnvrtc / libnccl are dlopen'ed lazily: loading works without a GPU
+    out = os.popen(f"ldd {_lib.LIB_PATH}").read()
+    for bad in ("libcuda.so", "libnvrtc", "libnccl", "libcudart"):
+        assert bad not in out, out
+
+
+def test_status_strings():
+    for code, name in _lib.STATUS.items():
+        assert _lib.lib.astitch_status_str(code).decode() == name
+
+
+def _st(fn, *args):
+    return fn(*args)
+
+
+def test_builder_errors():
+    g = A.Graph()
+    x = g.input("FULL", "F32")
+    r = g.input("ROWVEC", "F32")
+    with pytest.raises(A.AstitchError) as e:
+        g.binary("ADD", x, r)                     # kind mismatch -> INVALID_GRAPH
+    assert e.value.status == 2
+    with pytest.raises(A.AstitchError) as e:
+        g.reduce("SUM", "ROW", r)                 # reduce of a ROWVEC -> UNSUPPORTED
+    assert e.value.status == 3
+    with pytest.raises(A.AstitchError) as e:
+        g.broadcast("COL", r)                     # broadcast COL needs COLVEC -> INVALID_GRAPH
+    assert e.value.status == 2
+    v = ct.c_int32()
+    assert _lib.lib.astitch_graph_unary(g.handle, 99, x, ct.byref(v)) == 1      # bad enum
+    assert _lib.lib.astitch_graph_unary(g.handle, 0, 12345, ct.byref(v)) == 1   # bad operand
+    assert _lib.lib.astitch_graph_unary(g.handle, 0, x, None) == 1              # NULL out
+    assert _lib.lib.astitch_graph_input(g.handle, 3, 0, ct.byref(v)) == 1       # SCALAR input
+    L = g.lengths(8)
+    with pytest.raises(A.AstitchError):
+        g.lengths(8)                              # one mask per graph
+    with pytest.raises(A.AstitchError):
+        g.unary("EXP", L)                         # LENGTHS is not an operand
+
+
+def _plan_status(spec, rows, cols, flags=_lib.FLAG_NO_COMPILE):
+    g = A.Graph.from_spec(spec)
+    d = _lib.PlanDesc(rows=rows, cols=cols, device=-1, shard_rank=0, shard_world=1, flags=flags)
+    h = ct.c_void_p()
+    s = _lib.lib.astitch_plan(g.handle, ct.byref(d), ct.byref(h))
+    if s == 0:
+        _lib.lib.astitch_plan_destroy(h)
+    return s
+
+
+def test_plan_shape_errors():
+    spec = specs.get("C1")
+    assert _plan_status(spec, 32, 0) == 4          # cols < 1
+    assert _plan_status(spec, -1, 128) == 4        # rows < 0
+    assert _plan_status(spec, 1 << 41, 1 << 30) == 4
+    assert _plan_status(spec, 0, 128) == 0         # rows = 0 is a valid (no-op) plan
+    g = A.Graph()
+    g.input("FULL", "F32")
+    d = _lib.PlanDesc(rows=4, cols=4, device=-1, shard_world=1, flags=_lib.FLAG_NO_COMPILE)
+    h = ct.c_void_p()
+    assert _lib.lib.astitch_plan(g.handle, ct.byref(d), ct.byref(h)) == 2        # no outputs
+
+
+def test_run_on_host_only_plan_fails_loudly():
+    spec = specs.get("C1")
+    p = A.Plan(A.Graph.from_spec(spec), 32, 128, device=-1, flags=A.FLAG_NO_COMPILE)
+    ins = _lib.ptr_array([16])
+    outs = _lib.ptr_array([32])
+    s = _lib.lib.astitch_run(p.handle, ins, outs, None, None)
+    assert s == 1
+    assert "without a device" in _lib.lib.astitch_last_error().decode()
+    # misaligned pointer
+    s = _lib.lib.astitch_run(p.handle, _lib.ptr_array([17]), outs, None, None)
+    assert s == 1 and "aligned" in _lib.lib.astitch_last_error().decode()
+
+
+def test_shard_rows_partition():
+    for R in (0, 1, 7, 1_048_576, 524_289):
+        for g in (1, 2, 3, 4, 8):
+            total, nxt = 0, 0
+            for r in range(g):
+                b, c = A.shard_rows(R, g, r)
+                assert b == nxt and c in (R // g, R // g + 1)
+                nxt, total = b + c, total + c
+            assert total == R
+    with pytest.raises(A.AstitchError):
+        A.shard_rows(10, 2, 2)
+
+
+def test_io_signature_and_workspace():
+    spec = specs.get("C5", rows=4096)
+    p = A.Plan(A.Graph.from_spec(spec), 4096, 1024, device=-1, flags=A.FLAG_NO_COMPILE)
+    assert p.inputs == [("FULL", "BF16"), ("FULL", "BF16"), ("COLVEC", "F32")]
+    assert p.outputs == [("FULL", "BF16"), ("COLVEC", "F32"), ("COLVEC", "F32")]
+    assert p.workspace_bytes() > 0
+    spec = specs.get("C3", rows=8192)
+    p = A.Plan(A.Graph.from_spec(spec), 8192, 512, device=-1, flags=A.FLAG_NO_COMPILE)
+    assert p.inputs == [("FULL", "BF16"), ("LENGTHS", "I32")]
+    assert p.workspace_bytes() == 0

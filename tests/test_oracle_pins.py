@@ -283,7 +283,7 @@ def test_fig7a_bruteforce():
     R2 = [sum(A[r][c] * A[r][c] for r in range(R)) for c in range(C)]
     for r in range(R):
         for c in range(C):
-            assert out[r, c] == pytest.approx(A[r][c] * R2[c], rel=1e-13, abs=1e-13)
+            assert out[r, c] == pytest.approx(A[r][c] * A[r][c] * R2[c], rel=1e-13, abs=1e-13)
 
 
 # ---------------------------------------------------------------- plumbing

@@ -1,0 +1,189 @@
+"""GPU parity: the stitched sm_100a kernels (through the C ABI) against the fp64
+oracle, element by element, under the DESIGN.md tolerance rule.
+
+Sizes: reduced shapes that span several tiles and a ragged tail (oracle runs
+on everything), the full BASELINE.json shapes (oracle on sampled rows /
+columns), adversarial shapes and mask lengths, plus run-to-run determinism and
+the one-kernel-per-run property (Table 3's metric).
+"""
+
+import numpy as np
+import pytest
+
+from oracle import evaluate, evaluate_columns, evaluate_rows
+from tests.harness import check_close, run_gpu, spec_tol
+from workloads import gen, specs
+
+pytestmark = pytest.mark.gpu
+
+
+def _compare(spec, got, ref, tol=None):
+    tol = spec_tol(spec) if tol is None else tol
+    infos = {}
+    for name, dt in spec["outputs"]:
+        if name in ref:
+            infos[name] = check_close(got[name], ref[name], dt, tol, name=f"{spec['name']}:{name}")
+    return infos
+
+
+REDUCED = [
+    ("C1", None, None),
+    ("C2", 300, None),
+    ("C3", 3 * 256 + 7, None),
+    ("C4", 20_000 + 3, None),
+    ("C5", 3000 + 5, None),
+    ("C5int", 5000, 64),
+    ("fig5", None, None),
+    ("fig7a", None, None),
+    ("fig6a", 10_000 + 1, None),
+    ("fig6b", 8, None),
+]
+
+
+@pytest.mark.parametrize("cfg,rows,cols", REDUCED)
+def test_parity_reduced(cfg, rows, cols):
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 256
+    x = gen.generate(cfg, spec)
+    ref = evaluate(spec, x)
+    got = run_gpu(spec, x)
+    _compare(spec, got, ref)
+    if cfg == "C5int":  # small-integer data: every fp32 partial is exact -> bitwise
+        np.testing.assert_array_equal(got["db"], ref["db"])
+        np.testing.assert_array_equal(got["dz"], ref["dz"])
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C4", "C5", "fig7a"])
+@pytest.mark.parametrize("cols", [1, 3, 36, 37, 127, 129, 1023, 1025])
+def test_parity_ragged_cols(cfg, cols):
+    rows = {"C1": 149, "C2": 147, "C3": 297, "C4": 4099, "C5": 297, "fig7a": 149}[cfg]
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 64
+    x = gen.generate(cfg, spec)
+    _compare(spec, run_gpu(spec, x), evaluate(spec, x))
+
+
+@pytest.mark.parametrize("rows", [1, 2, 147, 149, 296, 297])
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C4", "C5"])
+def test_parity_ragged_rows(cfg, rows):
+    spec = specs.get(cfg, rows=rows)
+    x = gen.generate(cfg, spec)
+    _compare(spec, run_gpu(spec, x), evaluate(spec, x))
+
+
+@pytest.mark.parametrize("lengths", [[0, 1, 37, 511], [512, 512, 1, 0], [37, 200, 511, 512]])
+def test_parity_mask_lengths(lengths):
+    spec = specs.get("C3", rows=4 * 96, cols=512)
+    spec["mask"]["rows_per_segment"] = 96
+    x = gen.generate("C3", spec)
+    x["L"] = np.array(lengths, dtype=np.int32)
+    ref = evaluate(spec, x)
+    got = run_gpu(spec, x)
+    _compare(spec, got, ref)
+    for s, L in enumerate(lengths):
+        blk = got["p"][s * 96:(s + 1) * 96]
+        assert (blk[:, L:] == 0).all()           # masked tail written as exact zeros
+        if L > 0:
+            np.testing.assert_allclose(blk[:, :L].sum(axis=1), 1.0, atol=L * 4e-3)
+
+
+def test_full_c1_c2():
+    for cfg in ("C1", "C2"):
+        spec = specs.get(cfg)
+        x = gen.generate(cfg, spec)
+        _compare(spec, run_gpu(spec, x), evaluate(spec, x))
+
+
+def test_full_c3_sampled_rows():
+    spec = specs.get("C3")
+    x = gen.generate("C3", spec)
+    got = run_gpu(spec, x)
+    rng = np.random.default_rng(0)
+    rows = np.unique(np.concatenate([rng.integers(0, spec["rows"], 1500),
+                                     [0, 8191, 8192, spec["rows"] - 1]]))
+    ref = evaluate_rows(spec, x, rows)
+    check_close(got["p"][rows], ref["p"], "BF16", 2e-3, "C3 full sampled")
+    # properties at any size: masked tail zero, valid prefix sums to 1
+    L = x["L"]
+    for s in (0, 1, 63):
+        blk = got["p"][s * 8192:(s + 1) * 8192]
+        assert (blk[:, L[s]:] == 0).all()
+        np.testing.assert_allclose(blk[:, :L[s]].sum(axis=1), 1.0, atol=L[s] * 4e-3)
+
+
+def test_full_c4():
+    spec = specs.get("C4")
+    x = gen.generate("C4", spec)
+    got = run_gpu(spec, x)
+    rng = np.random.default_rng(1)
+    rows = np.unique(np.concatenate([rng.integers(0, spec["rows"], 20000), [0, spec["rows"] - 1]]))
+    ref = evaluate_rows(spec, x, rows)
+    check_close(got["o"][rows], ref["o"], "F32", 1e-5, "C4 full sampled")
+    np.testing.assert_allclose(got["o"].mean(axis=1), 0.0, atol=2e-6)
+
+
+@pytest.mark.slow
+def test_full_c5_sampled():
+    spec = specs.get("C5")
+    x = gen.generate("C5", spec)
+    got = run_gpu(spec, x)
+    rng = np.random.default_rng(2)
+    cols = np.unique(np.concatenate([rng.integers(0, 1024, 24), [0, 1023]]))
+    refc = evaluate_columns(spec, x, cols)
+    check_close(got["db"][cols], refc["db"], "F32", 2e-3, "C5 db")
+    check_close(got["b_new"][cols], refc["b_new"], "F32", 2e-3, "C5 b_new")
+    # fp32-quality report for db (reading R4): informational bound 1e-5 relative to RMS
+    s = np.sqrt(np.mean(refc["db"] ** 2))
+    assert np.max(np.abs(got["db"][cols] - refc["db"])) <= 1e-4 * s
+    rows = np.unique(rng.integers(0, spec["rows"], 3000))
+    sub = dict(spec, outputs=[("dz", "BF16")], ops=[o for o in spec["ops"] if o[0] in ("g", "dz")])
+    refr = evaluate_rows(sub, x, rows)
+    check_close(got["dz"][rows], refr["dz"], "BF16", 2e-3, "C5 dz")
+    # b_new is one fp32 rounding of b - 2^-7 db of the GPU's own db (reading R10)
+    b = x["b"].astype(np.float32)
+    exp = (b - np.float32(0.0078125) * got["db"].astype(np.float32)).astype(np.float32)
+    np.testing.assert_array_equal(got["b_new"].astype(np.float32), exp)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C4", "C5"])
+def test_determinism_bitwise(cfg):
+    import torch
+    spec = specs.get(cfg, rows=5000 if cfg != "C3" else 2048)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 256
+    x = gen.generate(cfg, spec)
+    a, plan = run_gpu(spec, x, return_plan=True)
+    b = run_gpu(spec, x, plan=plan)
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k
+    torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C4", "C5", "fig7a"])
+def test_one_kernel_no_memset_per_run(cfg):
+    """Kernel count per subgraph = 1 and no memset/memcpy (Table 3's metric)."""
+    import torch
+    from torch.profiler import ProfilerActivity, profile
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from tests.harness import device_inputs
+    spec = specs.get(cfg, rows=4096 if cfg != "C1" else None)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 512
+    x = gen.generate(cfg, spec)
+    plan = A.Plan(A.Graph.from_spec(spec), spec["rows"], spec["cols"], device=0)
+    assert plan.kernel_count() == 1
+    assert plan.describe()["memsets_per_run"] == 0
+    ins, outs = device_inputs(spec, x), plan.alloc_outputs()
+    ws = plan.alloc_workspace()
+    plan.run(ins, outs, ws=ws)
+    torch.cuda.synchronize()
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        plan.run(ins, outs, ws=ws)
+        torch.cuda.synchronize()
+    names = [e.name for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA]
+    kern = [n for n in names if n.startswith("astitch_")]
+    other = [n for n in names if not n.startswith("astitch_")]
+    assert len(kern) == 1, names
+    assert not any("memset" in n.lower() or "memcpy" in n.lower() for n in other), names

@@ -1,0 +1,140 @@
+"""Planner golden tests (host only): op classes, dominant candidates, groups,
+schemes (Table 1 / Sec. 4.3), the thread-mapping selector (Sec. 3.3)
+and the generated kernels (NVRTC sm_100a compile, no GPU needed)."""
+
+import pytest
+
+import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+from workloads import specs
+
+
+def describe(cfg, rows=None, cols=None, flags=A.FLAG_NO_COMPILE, **kw):
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    g = A.Graph.from_spec(spec)
+    p = A.Plan(g, spec["rows"], spec["cols"], device=-1, flags=flags, **kw)
+    d = p.describe()
+    ops = {name: d["ops"][vid] for name, vid in g.names.items()}
+    return d, ops, p
+
+
+def test_c1_softmax_regional_one_group():
+    d, ops, _ = describe("C1")
+    assert ops["m"]["class"] == "reduce_row" and ops["m"]["scheme"] == "regional"
+    assert ops["s"]["scheme"] == "regional"
+    assert ops["e"]["class"] == "heavy_ew" and ops["e"]["scheme"] == "local"
+    assert ops["y"]["scheme"] == "independent" and ops["y"]["candidate"]
+    assert len(d["groups"]) == 1
+    assert ops["m"]["dominant"] and ops["s"]["sub_dominant"] and ops["y"]["sub_dominant"]
+    assert d["mapping"]["template"] == "row_team"
+
+
+def test_c2_layernorm_heavy_rowvec_candidate():
+    d, ops, _ = describe("C2")
+    # rsqrt on the per-row variance is heavy EW followed by a broadcast (Fig. 5 pattern)
+    assert ops["rstd"]["class"] == "heavy_ew" and ops["rstd"]["candidate"]
+    assert ops["rstd"]["scheme"] == "regional"
+    assert ops["hs"]["scheme"] == "regional" and ops["vs"]["scheme"] == "regional"
+    assert ops["o"]["class"] == "heavy_ew"
+    assert len(d["groups"]) == 1
+    m = d["mapping"]
+    assert m["template"] == "row_team" and m["team"] == 32 and m["chunks_per_lane"] == 3 and m["vec_elems"] == 8
+    assert m["lane_util"] == 1.0
+
+
+def test_c3_mask_row_team():
+    d, ops, _ = describe("C3")
+    assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 32
+    assert ops["m"]["scheme"] == "regional" and ops["z"]["scheme"] == "regional"
+
+
+def test_c4_many_tiny_rows_packed():
+    d, _, _ = describe("C4")
+    m = d["mapping"]
+    assert m["template"] == "packed_tile"
+    assert m["team"] == 1 and m["chunks_per_lane"] == 9
+    assert m["lds128_conflict_ways"] == 1          # 144-byte rows: conflict-free LDS.128
+    assert m["smem_bytes"] > 0 and m["stages"] >= 3
+    # ablation NO_TMA falls back to a row team
+    d2, _, _ = describe("C4", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_TMA)
+    assert d2["mapping"]["template"] == "row_team"
+
+
+def test_c5_global_scheme_and_barrier():
+    d, ops, _ = describe("C5")
+    assert d["mapping"]["template"] == "global_sweep"
+    assert ops["db"]["class"] == "reduce_col" and ops["db"]["scheme"] == "global" and ops["db"]["dominant"]
+    assert ops["b_new"]["post_barrier"] and not ops["dz"]["post_barrier"]
+    assert ops["g"]["class"] == "heavy_ew" and ops["g"]["scheme"] == "local"
+    assert ops["dz"]["scheme"] == "local"            # consumed by the reduce before the barrier
+    assert d["global_fulls"] == [] and not d["needs_sweep2"]
+    assert d["workspace"]["total"] > 0
+    assert d["mapping"]["grid"] <= d["mapping"]["blocks_per_sm"] * 148
+
+
+def test_fig5_heavy_producer_once_per_row():
+    d, ops, p = describe("fig5")
+    assert ops["pw"]["candidate"] and ops["pw"]["scheme"] == "regional"
+    src = p.source(0)
+    # power is computed on the row scalar (once per row), not per element
+    assert "const float s" in src and "(s" in src
+
+
+def test_fig7a_schemes_match_paper():
+    """regional for reduce.1, global for power.1 and reduce.2,
+    independent for multiply.1, local for the others; final dominants reduce.1
+    and reduce.2, sub-dominants power.1 and multiply.1."""
+    d, ops, _ = describe("fig7a")
+    assert ops["reduce1"]["scheme"] == "regional"
+    assert ops["power1"]["scheme"] == "global"
+    assert ops["reduce2"]["scheme"] == "global"
+    assert ops["multiply1"]["scheme"] == "independent"
+    for n in ("divide1", "add1", "broadcast1", "broadcast2"):
+        assert ops[n]["scheme"] == "local", n
+    assert ops["reduce1"]["dominant"] and ops["reduce2"]["dominant"]
+    assert ops["power1"]["sub_dominant"] and ops["multiply1"]["sub_dominant"]
+    assert len(d["groups"]) == 2
+    assert d["needs_sweep2"] and d["kernel_count"] == 1
+
+
+def test_fig6_selector_branches():
+    d, _, _ = describe("fig6a")              # <750000,32>: pack many rows per block
+    m = d["mapping"]
+    assert m["template"] == "row_team" and m["team"] < 32 and m["rows_per_block"] > 32
+    assert m["grid"] <= m["blocks_per_sm"] * 148
+    d, _, _ = describe("fig6b")              # <64,30000>: the paper's split rule holds
+    assert "split rule holds" in d["mapping"]["reason"]
+    d, _, _ = describe("fig6b", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_SPLIT)
+    assert "split rule" not in d["mapping"]["reason"]
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C4"])
+def test_mapping_independent_of_rows(cfg):
+    """Reading R13: a row's reduction tree depends only on C, so shards are
+    bitwise equal to the unsharded run."""
+    a, _, _ = describe(cfg)
+    b, _, _ = describe(cfg, rows=8192 + 17)
+    for k in ("template", "team", "chunks_per_lane", "vec_elems"):
+        assert a["mapping"][k] == b["mapping"][k], k
+
+
+def test_no_pack_ablation():
+    d, _, _ = describe("fig6a", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_PACK)
+    assert d["mapping"]["team"] == 32
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C4", "C5", "fig5", "fig7a", "fig6a", "fig6b"])
+def test_generated_kernels_compile_for_sm100a(cfg):
+    """NVRTC compiles every generated kernel for sm_100a on the host (no GPU)."""
+    d, _, p = describe(cfg, flags=0)
+    cub = p.cubin(0)
+    assert len(cub) > 1000 and cub[:4] == b"\x7fELF"
+    k = d["kernels"][0]
+    assert k["spill_bytes"] == 0, k
+    assert k["name"].startswith("astitch_")
+
+
+def test_sharded_plan_has_epilogue_kernels():
+    d, _, _ = describe("C5", rows=131072, flags=0, shard_rank=1, shard_world=8)
+    assert d["kernel_count"] == 1 and d["shard_kernels"] == 2
+    d, _, _ = describe("fig7a", flags=0, shard_rank=0, shard_world=2)
+    assert d["shard_kernels"] == 3

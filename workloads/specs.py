@@ -231,7 +231,9 @@ FIG7A_MIXED = {
         ("power1", "binary", "POW", "add1", "two"),
         ("reduce2", "reduce", "SUM", "COL", "power1"),
         ("broadcast2", "broadcast", "COL", "reduce2"),
-        ("multiply1", "binary", "MUL", "add1", "broadcast2"),
+        # multiply.1 consumes power.1 across the barrier, which is what makes
+        # power.1 "global" in P:L198 (its value is buffered in HBM)
+        ("multiply1", "binary", "MUL", "power1", "broadcast2"),
     ],
     "outputs": [("multiply1", "F32")],
 }
