@@ -222,6 +222,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--flags", type=int, default=0)
+    ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -301,6 +302,22 @@ def main():
     copy_gbs = 2 * half * 10 / (ce0.elapsed_time(ce1) * 1e-3) / 1e9
     del src, dst
 
+    # K steps captured once into a CUDA graph (removes host launch overhead,
+    # which otherwise dominates the us-scale configs); eager if capture fails
+    graph = None
+    if not args.eager:
+        try:
+            graph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph):
+                for i in range(args.steps):
+                    step(i)
+            graph.replay()
+            torch.cuda.synchronize()
+        except Exception as e:  # pragma: no cover
+            print(f"[bench] graph capture failed ({e}); timing eagerly", file=sys.stderr)
+            graph = None
+            torch.cuda.synchronize()
+
     # ---- timed region
     if world > 1:
         dist.barrier()
@@ -308,8 +325,11 @@ def main():
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(dev) as clk:
         e0.record(stream)
-        for i in range(args.steps):
-            step(i)
+        if graph is not None:
+            graph.replay()
+        else:
+            for i in range(args.steps):
+                step(i)
         e1.record(stream)
         torch.cuda.synchronize()
     if world > 1:
@@ -406,6 +426,7 @@ def main():
                        "parallelism": f"dp{world} contiguous row shards" + (", 1 ncclAllReduce of fp32 column partials" if world > 1 and desc["shard_kernels"] else ""),
                        "l2": ("inputs > L2 (%.2f GB per rank vs %d MB L2)" % (nbytes / 1e9, l2 // 2**20)) if nsets == 1
                        else f"{nsets} rotating input sets >= 4x L2",
+                       "timing": "cuda_graph_replay" if graph is not None else "eager",
                        "template": desc["mapping"]["template"], "grid": desc["kernels"][0]["grid"],
                        "threads": desc["mapping"]["threads"], "regs": desc["kernels"][0]["regs"]},
             "us_per_subgraph": round(ms_step * 1e3, 3),

@@ -423,6 +423,9 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 }  // namespace as
 
 // ------------------------------------------------------------------ measurement kernels
+// Only compiled into the measurement module (and the AOT build check), not
+// into the generated stitched kernels.
+#if defined(ASTITCH_BENCH_KERNELS) || !defined(ASTITCH_JIT)
 // Barrier-only kernel (Table 6 micro-benchmark on B200).
 extern "C" __global__ void astitch_barrier_bench(u32* bar, int iters) {
   for (int i = 0; i < iters; ++i) as::grid_barrier(bar);
@@ -441,3 +444,4 @@ extern "C" __global__ void __launch_bounds__(256) astitch_copy_bench(const as::R
   }
   for (; i < n16; i += stride) as::stg(dst + i, as::ldg(src + i));
 }
+#endif  // ASTITCH_BENCH_KERNELS

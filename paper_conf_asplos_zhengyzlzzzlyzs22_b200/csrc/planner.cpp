@@ -403,20 +403,36 @@ void select_mapping(Plan& p) {
     // Horizontal packing of many tiny rows: when a row is too
     // short for a power-of-two team to tile it (e.g. 9 x 16-byte chunks),
     // stage row tiles in smem with TMA bulk copies and give each thread a row.
-    bool packed_ok = !no_tma && !no_pack && !has_mask && row16 && !has_colvec_in &&
-                     row_bytes_max <= 512 && m.lane_util < 0.95 && chunks <= 32 &&
-                     p.global_fulls.empty() && R >= 4096;
+    bool tile_common = !no_tma && row16 && p.global_fulls.empty() && R >= 4096;
+    bool packed_ok = tile_common && !no_pack && !has_mask && !has_colvec_in && row_bytes_max <= 512 &&
+                     m.lane_util < 0.95 && chunks <= 32;
+    int in_row_bytes = 0;
+    for (int id : g.inputs)
+      if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live)
+        in_row_bytes += static_cast<int>(C) * dtype_size(g.nodes[id].dtype);
+    // Team tiles: rows of up to a warp's worth of chunks staged by TMA bulk
+    // copies (deep async pipeline: bytes in flight no longer tied to registers)
+    bool team_tile_ok = tile_common && !packed_ok && m.team <= 32 && m.team >= 1 &&
+                        in_row_bytes > 0 && in_row_bytes * (256 / m.team) <= 48 * 1024;
     // Task splitting (rule P:L270): rows < blocks-per-wave and row > 1024.
     bool split_rule = !no_split && R < blocks_per_wave_1024 && C > 1024;
-    if (packed_ok) {
+    if (packed_ok || team_tile_ok) {
       m.tmpl = Template::PackedTile;
-      m.team = 1;
-      m.chunks_per_lane = chunks;
-      m.lane_util = 1.0;
-      m.threads = 128;
-      m.tile_rows = 128;
+      if (packed_ok) {
+        m.team = 1;
+        m.chunks_per_lane = chunks;
+        m.lane_util = 1.0;
+        m.threads = 128;
+        m.tile_rows = 128;
+      } else {
+        m.threads = 256;
+        int teams = m.threads / m.team;
+        int tr = 1;
+        while (tr * 2 * in_row_bytes <= 24 * 1024) tr *= 2;
+        m.tile_rows = std::max(teams, (tr / teams) * teams);
+      }
       m.stages = 4;  // prefetch distance 2 tiles + 2 tiles draining (bulk stores)
-      m.rows_per_block = m.tile_rows;
+      m.rows_per_block = m.threads / m.team;
       // stage bytes: input tiles + output tiles that cannot be written in
       // place over an input tile of the same element size (mirrors codegen)
       int in_bytes = 0, out_bytes = 0;
@@ -438,9 +454,15 @@ void select_mapping(Plan& p) {
         m.stages--;
         m.smem_bytes = m.stages * m.tile_rows * (in_bytes + out_bytes) + 64 * m.stages;
       }
-      m.bank_conflict_ways = lds128_conflict_ways(static_cast<int>(C) * es_min);
-      why << "row of " << chunks << " x " << (E * es_min)
-          << "B chunks does not tile a power-of-two team -> TMA-staged packed tiles, thread per row; ";
+      if (packed_ok) {
+        m.bank_conflict_ways = lds128_conflict_ways(static_cast<int>(C) * es_min);
+        why << "row of " << chunks << " x " << (E * es_min)
+            << "B chunks does not tile a power-of-two team -> TMA-staged packed tiles, thread per row; ";
+      } else {
+        why << "TMA bulk-staged tiles of " << m.tile_rows << " rows (" << m.stages
+            << "-stage mbarrier pipeline), team of " << m.team << " lanes x " << m.chunks_per_lane
+            << " chunks per row from smem" << (has_mask ? ", valid-prefix copies per row" : "") << "; ";
+      }
     } else {
       m.tmpl = Template::RowTeam;
       if (split_rule) {

@@ -57,10 +57,29 @@ const char* role_suffix(int role) {
 // Build (generate + compile + load) one kernel of the plan.  Applies the
 // assume-relax-apply loop: if ptxas spills under the assumed
 // register bound, relax the target blocks per SM and recompile.
+// Register use and spills come from the loaded function's attributes when a
+// device is present (authoritative), else from the ptxas -v log.
+static astitch_status compile_and_inspect(Plan& p, Kernel& k, bool load) {
+  std::string err;
+  if (k.module) drv_unload(k);
+  k.regs = -1;
+  k.spill_bytes = -1;
+  if (!nvrtc_compile(k.source, k.name, k.cubin, k.log, err)) return fail(ASTITCH_ERR_CUDA, err);
+  parse_ptxas(k);
+  if (load) {
+    int log_spill = k.spill_bytes;
+    k.spill_bytes = -1;
+    if (!drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
+    k.spill_bytes = std::max(log_spill, k.spill_bytes);
+  }
+  return ASTITCH_OK;
+}
+
 astitch_status build_kernel(Plan& p, int role, Kernel& k) {
   const bool compile = (p.desc.flags & ASTITCH_FLAG_NO_COMPILE) == 0;
+  const bool load = compile && p.device >= 0;
   const bool may_relax = (role == ROLE_MAIN);  // later kernels share the main kernel's layout
-  for (int attempt = 0; attempt < 3; ++attempt) {
+  for (int attempt = 0; attempt < 4; ++attempt) {
     std::string base = std::string("astitch_") + template_name(p.map.tmpl) + role_suffix(role);
     k.name = base;
     k.source = generate_kernel(p, role, base);
@@ -76,22 +95,25 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     k.smem = (role == ROLE_SHARD_FINAL) ? 0 : p.map.smem_bytes;
     k.cooperative = (p.map.tmpl == Template::GlobalSweep) && (role == ROLE_MAIN || role == ROLE_SHARD_MAIN);
     if (!compile) return ASTITCH_OK;
-    std::string err;
-    if (!nvrtc_compile(k.source, k.name, k.cubin, k.log, err)) return fail(ASTITCH_ERR_CUDA, err);
-    parse_ptxas(k);
+    astitch_status st = compile_and_inspect(p, k, load);
+    if (st != ASTITCH_OK) return st;
     if (k.spill_bytes > 0 && p.map.blocks_per_sm > 1 && may_relax) {
       // relax: compile once without the occupancy bound to learn the natural
       // register demand, then apply the largest occupancy that fits it.
       if (attempt == 0) {
         Plan probe = p;
         probe.map.blocks_per_sm = 1;
-        std::string src = generate_kernel(probe, role, base);
         Kernel kp;
         kp.name = base;
-        std::string e2;
-        if (!nvrtc_compile(src, base, kp.cubin, kp.log, e2)) return fail(ASTITCH_ERR_CUDA, e2);
-        parse_ptxas(kp);
-        int regs = std::max(32, (kp.regs + 7) & ~7);
+        kp.source = generate_kernel(probe, role, base);
+        kp.threads = k.threads;
+        kp.smem = k.smem;
+        st = compile_and_inspect(p, kp, load);
+        if (kp.module) drv_unload(kp);
+        if (st != ASTITCH_OK) return st;
+        // first guess from the unrounded natural demand; ptxas can usually
+        // trim a few registers to meet the bound, else the next attempt relaxes
+        int regs = std::max(32, kp.regs);
         int bps = std::max(1, std::min(p.map.blocks_per_sm - 1, 65536 / (regs * p.map.threads)));
         p.map.blocks_per_sm = bps;
       } else {
@@ -158,7 +180,7 @@ astitch_status astitch_plan(astitch_graph_t gr, const astitch_plan_desc* desc, a
     if (p.device >= 0 && (p.desc.flags & ASTITCH_FLAG_NO_COMPILE) == 0) {
       auto load = [&](Kernel& k) -> astitch_status {
         std::string err;
-        if (!drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
+        if (!k.module && !drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
         if (k.cooperative) {
           int64_t max_grid = static_cast<int64_t>(k.occupancy) * p.sm_count;
           if (max_grid < 1)
@@ -385,7 +407,7 @@ astitch_status bench_module(int device, BenchModule*& out) {
   if (!b.ok) {
     std::string err, log;
     std::vector<char> cubin;
-    std::string src = "#include \"astitch_device.cuh\"\n";
+    std::string src = "#define ASTITCH_BENCH_KERNELS 1\n#include \"astitch_device.cuh\"\n";
     if (!nvrtc_compile(src, "astitch_bench", cubin, log, err)) return fail(ASTITCH_ERR_CUDA, err);
     Plan tmp;
     tmp.device = device;

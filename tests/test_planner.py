@@ -37,14 +37,20 @@ def test_c2_layernorm_heavy_rowvec_candidate():
     assert ops["o"]["class"] == "heavy_ew"
     assert len(d["groups"]) == 1
     m = d["mapping"]
-    assert m["template"] == "row_team" and m["team"] == 32 and m["chunks_per_lane"] == 3 and m["vec_elems"] == 8
+    assert m["template"] == "packed_tile" and m["team"] == 32 and m["chunks_per_lane"] == 3 and m["vec_elems"] == 8
     assert m["lane_util"] == 1.0
-
-
-def test_c3_mask_row_team():
-    d, ops, _ = describe("C3")
+    d, _, _ = describe("C2", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_TMA)
     assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 32
+
+
+def test_c3_mask_team_tiles():
+    d, ops, _ = describe("C3")
+    m = d["mapping"]
+    assert m["template"] == "packed_tile" and m["team"] == 32 and m["tile_rows"] % m["rows_per_block"] == 0
+    assert "valid-prefix" in m["reason"]
     assert ops["m"]["scheme"] == "regional" and ops["z"]["scheme"] == "regional"
+    d, _, _ = describe("C3", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_TMA)
+    assert d["mapping"]["template"] == "row_team"
 
 
 def test_c4_many_tiny_rows_packed():
@@ -99,7 +105,7 @@ def test_fig7a_schemes_match_paper():
 def test_fig6_selector_branches():
     d, _, _ = describe("fig6a")              # <750000,32>: pack many rows per block
     m = d["mapping"]
-    assert m["template"] == "row_team" and m["team"] < 32 and m["rows_per_block"] > 32
+    assert m["team"] < 32 and m["rows_per_block"] > 32
     assert m["grid"] <= m["blocks_per_sm"] * 148
     d, _, _ = describe("fig6b")              # <64,30000>: the paper's split rule holds
     assert "split rule holds" in d["mapping"]["reason"]
