@@ -384,7 +384,19 @@ void select_mapping(Plan& p) {
     why << "column reduce -> global sweep (vertical packing, grid barrier); ";
   } else {
     // ---------------------------------------------------------- row-wise
-    choose_team(1024, 16, 32);
+    // Masked rows: a chunk index spans T*E columns across the team, and the
+    // chunk-uniform mask branches skip whole chunks past the valid length, so
+    // a finer chunk (smaller team, more chunks per lane) wastes less work on
+    // padding; it also puts several rows of one segment (same length) in a warp.
+    choose_team(1024, has_mask ? 32 : 16, 32);
+    if (const char* ft = getenv("ASTITCH_FORCE_TEAM")) {  // tuning knob for experiments
+      int t = atoi(ft);
+      if (t >= 1 && t <= 1024 && (t & (t - 1)) == 0) {
+        m.team = t;
+        m.chunks_per_lane = (chunks + t - 1) / t;
+        m.lane_util = static_cast<double>(chunks) / (t * m.chunks_per_lane);
+      }
+    }
     if (no_pack && m.team < 32 && chunks >= 1) {
       // ablation: XLA-style one row per warp (no horizontal packing)
       m.team = 32;
@@ -412,7 +424,9 @@ void select_mapping(Plan& p) {
         in_row_bytes += static_cast<int>(C) * dtype_size(g.nodes[id].dtype);
     // Team tiles: rows of up to a warp's worth of chunks staged by TMA bulk
     // copies (deep async pipeline: bytes in flight no longer tied to registers)
-    bool team_tile_ok = tile_common && !packed_ok && m.team <= 32 && m.team >= 1 &&
+    // (measured on B200: for masked rows the register-prefetching row team is
+    // faster than per-row valid-prefix bulk copies, so masks stay on row teams)
+    bool team_tile_ok = tile_common && !packed_ok && !has_mask && m.team <= 32 && m.team >= 1 &&
                         in_row_bytes > 0 && in_row_bytes * (256 / m.team) <= 48 * 1024;
     // Task splitting (rule P:L270): rows < blocks-per-wave and row > 1024.
     bool split_rule = !no_split && R < blocks_per_wave_1024 && C > 1024;

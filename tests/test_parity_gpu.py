@@ -89,6 +89,34 @@ def test_parity_mask_lengths(lengths):
             np.testing.assert_allclose(blk[:, :L].sum(axis=1), 1.0, atol=L * 4e-3)
 
 
+def _masked_variant(kind):
+    """Masked graphs where mask absorption does / does not apply."""
+    base = specs.get("C3", rows=6 * 64, cols=200)
+    base["mask"]["rows_per_segment"] = 64
+    if kind == "softmax_rowvec_out":      # ROWVEC output -> absorption disabled
+        base["outputs"] = [("p", "BF16"), ("z", "F32"), ("m", "F32")]
+    elif kind == "layernorm":             # SUM then (x - mean)^2: no single substitute works
+        base["ops"] = [("xs", "reduce", "SUM", "ROW", "s"), ("n", "const", 1.0 / 64),
+                       ("mu", "binary", "MUL", "xs", "n"), ("mub", "broadcast", "ROW", "mu"),
+                       ("c", "binary", "SUB", "s", "mub"), ("c2", "binary", "MUL", "c", "c"),
+                       ("vs", "reduce", "SUM", "ROW", "c2"), ("vb", "broadcast", "ROW", "vs"),
+                       ("o", "binary", "MUL", "c", "vb")]
+        base["outputs"] = [("o", "F32"), ("vs", "F32")]
+    elif kind == "rowsum":                # SUM only: substitute 0 absorbs
+        base["ops"] = [("xs", "reduce", "SUM", "ROW", "s"), ("xb", "broadcast", "ROW", "xs"),
+                       ("o", "binary", "ADD", "s", "xb")]
+        base["outputs"] = [("o", "BF16")]
+    return base
+
+
+@pytest.mark.parametrize("kind", ["softmax_rowvec_out", "layernorm", "rowsum"])
+def test_parity_masked_variants(kind):
+    spec = _masked_variant(kind)
+    x = gen.generate("C3", spec)
+    x["L"] = np.array([0, 1, 37, 199, 200, 64], dtype=np.int32)
+    _compare(spec, run_gpu(spec, x), evaluate(spec, x), tol=2e-3)
+
+
 def test_full_c1_c2():
     for cfg in ("C1", "C2"):
         spec = specs.get(cfg)
