@@ -278,6 +278,60 @@ __device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * erfcf(-0.
 
 __device__ __forceinline__ float fpow(float a, float b) { return powf(a, b); }
 
+// ------------------------------------------------------------------ local: paired fp32 math
+// sm_100 executes two fp32 add/mul/fma per instruction (FADD2 / FMUL2 /
+// FFMA2 on an aligned register pair).  Element-wise chains are emitted on
+// element pairs so the issue slots per element halve; MUFU ops stay scalar.
+struct f2 { float x, y; };
+__device__ __forceinline__ u64 pk2(f2 a) { u64 r; asm("mov.b64 %0, {%1,%2};" : "=l"(r) : "f"(a.x), "f"(a.y)); return r; }
+__device__ __forceinline__ f2 upk2(u64 r) { f2 d; asm("mov.b64 {%0,%1}, %2;" : "=f"(d.x), "=f"(d.y) : "l"(r)); return d; }
+__device__ __forceinline__ f2 bc2(float s) { return f2{s, s}; }
+__device__ __forceinline__ f2 add2(f2 a, f2 b) { u64 r; asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(pk2(a)), "l"(pk2(b))); return upk2(r); }
+__device__ __forceinline__ f2 sub2(f2 a, f2 b) { u64 r; asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(pk2(a)), "l"(pk2(b))); return upk2(r); }
+__device__ __forceinline__ f2 mul2(f2 a, f2 b) { u64 r; asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(pk2(a)), "l"(pk2(b))); return upk2(r); }
+__device__ __forceinline__ f2 fma2(f2 a, f2 b, f2 c) {
+  u64 r; asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(pk2(a)), "l"(pk2(b)), "l"(pk2(c))); return upk2(r);
+}
+__device__ __forceinline__ f2 abs2(f2 a) { return f2{fabsf(a.x), fabsf(a.y)}; }
+__device__ __forceinline__ f2 neg2(f2 a) { return f2{-a.x, -a.y}; }
+__device__ __forceinline__ f2 max2(f2 a, f2 b) { return f2{fmaxf(a.x, b.x), fmaxf(a.y, b.y)}; }
+__device__ __forceinline__ f2 min2(f2 a, f2 b) { return f2{fminf(a.x, b.x), fminf(a.y, b.y)}; }
+__device__ __forceinline__ f2 ex2_2(f2 a) { return f2{ex2(a.x), ex2(a.y)}; }
+__device__ __forceinline__ f2 rcp_2(f2 a) { return f2{rcp(a.x), rcp(a.y)}; }
+__device__ __forceinline__ f2 fexp2(f2 a) { return ex2_2(mul2(a, bc2(1.4426950408889634f))); }
+__device__ __forceinline__ f2 fdiv2(f2 a, f2 b) { return mul2(a, rcp_2(b)); }
+__device__ __forceinline__ f2 rsq2(f2 a) { return f2{rsq(a.x), rsq(a.y)}; }
+__device__ __forceinline__ f2 sqrt2_(f2 a) { return f2{sqrt_(a.x), sqrt_(a.y)}; }
+__device__ __forceinline__ f2 flog2_(f2 a) { return f2{flog(a.x), flog(a.y)}; }
+__device__ __forceinline__ f2 ftanh2(f2 a) { return f2{ftanh(a.x), ftanh(a.y)}; }
+__device__ __forceinline__ f2 ferf2(f2 a) { return f2{ferf(a.x), ferf(a.y)}; }
+__device__ __forceinline__ f2 gelu_erf2(f2 a) { return f2{gelu_erf(a.x), gelu_erf(a.y)}; }
+__device__ __forceinline__ f2 fpow2(f2 a, f2 b) { return f2{fpow(a.x, b.x), fpow(a.y, b.y)}; }
+__device__ __forceinline__ f2 fsigmoid2(f2 a) {
+  f2 e = ex2_2(mul2(a, bc2(-1.4426950408889634f)));
+  return rcp_2(add2(e, bc2(1.0f)));
+}
+// gelu_tanh = x * sigmoid(2u), u = x * (c + c k x^2)
+__device__ __forceinline__ f2 gelu_tanh2(f2 x) {
+  f2 x2 = mul2(x, x);
+  f2 u = mul2(x, fma2(bc2(AS_GELU_C * AS_GELU_K), x2, bc2(AS_GELU_C)));
+  f2 e = ex2_2(mul2(u, bc2(-2.8853900817779268f)));
+  return mul2(x, rcp_2(add2(e, bc2(1.0f))));
+}
+// gelu_tanh' = sigmoid(2u) + (x e r^2) * 2c(1 + 3k x^2),  e = exp(-2|u|), r = 1/(1+e)
+// (same cancellation-free form as gelu_tanh_grad, reassociated for FFMA2)
+__device__ __forceinline__ f2 gelu_tanh_grad2(f2 x) {
+  f2 x2 = mul2(x, x);
+  f2 u = mul2(x, fma2(bc2(AS_GELU_C * AS_GELU_K), x2, bc2(AS_GELU_C)));
+  f2 e = ex2_2(mul2(abs2(u), bc2(-2.8853900817779268f)));
+  f2 r = rcp_2(add2(e, bc2(1.0f)));
+  f2 er = mul2(e, r);
+  f2 sig = f2{u.x >= 0.f ? r.x : er.x, u.y >= 0.f ? r.y : er.y};
+  f2 du2 = fma2(bc2(6.0f * AS_GELU_C * AS_GELU_K), x2, bc2(2.0f * AS_GELU_C));
+  return fma2(mul2(mul2(x, er), r), du2, sig);
+}
+__device__ __forceinline__ f2 gelu_tanh_grad_2(f2 x) { return gelu_tanh_grad2(x); }
+
 // ------------------------------------------------------------------ regional: team reductions
 template <int T> __device__ __forceinline__ float team_sum(float v) {
 #pragma unroll

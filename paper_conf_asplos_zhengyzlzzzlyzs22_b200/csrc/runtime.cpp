@@ -79,7 +79,10 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
   const bool compile = (p.desc.flags & ASTITCH_FLAG_NO_COMPILE) == 0;
   const bool load = compile && p.device >= 0;
   const bool may_relax = (role == ROLE_MAIN);  // later kernels share the main kernel's layout
-  for (int attempt = 0; attempt < 4; ++attempt) {
+  // assume-relax-apply as a bisection on blocks per SM: the largest occupancy
+  // whose register bound (65536 / (bps * threads)) compiles without spills
+  int good = 0, bad = 0;  // best spill-free / smallest spilling bps seen
+  for (int attempt = 0; attempt < 6; ++attempt) {
     std::string base = std::string("astitch_") + template_name(p.map.tmpl) + role_suffix(role);
     k.name = base;
     k.source = generate_kernel(p, role, base);
@@ -97,33 +100,17 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     if (!compile) return ASTITCH_OK;
     astitch_status st = compile_and_inspect(p, k, load);
     if (st != ASTITCH_OK) return st;
-    if (k.spill_bytes > 0 && p.map.blocks_per_sm > 1 && may_relax) {
-      // relax: compile once without the occupancy bound to learn the natural
-      // register demand, then apply the largest occupancy that fits it.
-      if (attempt == 0) {
-        Plan probe = p;
-        probe.map.blocks_per_sm = 1;
-        Kernel kp;
-        kp.name = base;
-        kp.source = generate_kernel(probe, role, base);
-        kp.threads = k.threads;
-        kp.smem = k.smem;
-        st = compile_and_inspect(p, kp, load);
-        if (kp.module) drv_unload(kp);
-        if (st != ASTITCH_OK) return st;
-        // first guess from the unrounded natural demand; ptxas can usually
-        // trim a few registers to meet the bound, else the next attempt relaxes
-        int regs = std::max(32, kp.regs);
-        int bps = std::max(1, std::min(p.map.blocks_per_sm - 1, 65536 / (regs * p.map.threads)));
-        p.map.blocks_per_sm = bps;
-      } else {
-        p.map.blocks_per_sm = std::max(1, p.map.blocks_per_sm - 1);
-      }
-      p.map.reg_cap = std::min(255, (65536 / (p.map.blocks_per_sm * p.map.threads)) & ~7);
-      retune_grid(p);
-      continue;
-    }
-    return ASTITCH_OK;
+    if (!may_relax) return ASTITCH_OK;
+    const int cur = p.map.blocks_per_sm;
+    if (k.spill_bytes > 0 && cur > 1) bad = cur;
+    else good = cur;
+    if (good == cur && (bad == 0 || bad - good <= 1)) return ASTITCH_OK;  // best found
+    int next = good > 0 ? (good + bad) / 2 : std::max(1, bad / 2);
+    if (next == cur || next < 1) return ASTITCH_OK;
+    if (good > 0 && next <= good) next = good;  // re-emit the best spill-free version
+    p.map.blocks_per_sm = next;
+    p.map.reg_cap = std::min(255, (65536 / (p.map.blocks_per_sm * p.map.threads)) & ~7);
+    retune_grid(p);
   }
   return ASTITCH_OK;
 }
