@@ -102,6 +102,13 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     if (st != ASTITCH_OK) return st;
     if (!may_relax) return ASTITCH_OK;
     const int cur = p.map.blocks_per_sm;
+    if (k.spill_bytes > 0 && cur == 1 && p.map.row_unroll > 1) {
+      // even one block per SM spills: fewer rows in flight per team
+      p.map.row_unroll /= 2;
+      good = bad = 0;
+      retune_grid(p);
+      continue;
+    }
     if (k.spill_bytes > 0 && cur > 1) bad = cur;
     else good = cur;
     if (good == cur && (bad == 0 || bad - good <= 1)) return ASTITCH_OK;  // best found

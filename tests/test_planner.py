@@ -43,14 +43,17 @@ def test_c2_layernorm_heavy_rowvec_candidate():
     assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 32
 
 
-def test_c3_mask_team_tiles():
-    d, ops, _ = describe("C3")
+def test_c3_mask_row_team_absorbed():
+    d, ops, p = describe("C3")
     m = d["mapping"]
-    assert m["template"] == "packed_tile" and m["team"] == 32 and m["tile_rows"] % m["rows_per_block"] == 0
-    assert "valid-prefix" in m["reason"]
+    # masked rows: finer chunks (T=16 x 4 chunks of 8 bf16) for chunk-uniform skipping
+    assert m["template"] == "row_team" and m["team"] == 16 and m["chunks_per_lane"] == 4
     assert ops["m"]["scheme"] == "regional" and ops["z"]["scheme"] == "regional"
-    d, _, _ = describe("C3", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_TMA)
-    assert d["mapping"]["template"] == "row_team"
+    src = p.source(0)
+    # mask absorption: invalid logits take -inf, reductions carry no selects
+    assert "= (-AS_INF);" in src
+    assert "r_ = r_ * 0x1p-3f;" in src          # max(0.125 x) = 0.125 max(x) hoist
+    assert "as::ex2_2(as::fma2(" in src         # exp(kx - m) fused to ex2(fma)
 
 
 def test_c4_many_tiny_rows_packed():
