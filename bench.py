@@ -39,6 +39,11 @@ WORKLOAD_NAMES = {
     "C4": "DIEN row standardise fp32 [2,000,000,36]",
     "C5": "bias-GELU backward + bias-grad column reduce + in-kernel SGD step, bf16 [1,048,576,1024]",
 }
+def spec_name(cfg):
+    from workloads import specs
+    return specs.ALL[cfg]["name"]
+
+
 METRIC = "stitched-subgraph achieved HBM GB/s (% of 8 TB/s) and us/subgraph"
 
 
@@ -185,7 +190,7 @@ def run_reference(args, rank, world):
     from workloads import specs
     cfg = args.config
     spec_full = specs.get(cfg)
-    sample_rows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 200_000, "C5": 16384}[cfg]
+    sample_rows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 200_000, "C5": 16384}.get(cfg, 4096)
     spec = specs.get(cfg, rows=min(sample_rows, spec_full["rows"]))
     if spec.get("mask"):
         spec["mask"]["rows_per_segment"] = min(spec["mask"]["rows_per_segment"], spec["rows"])
@@ -204,7 +209,7 @@ def run_reference(args, rank, world):
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic",
-        "config": {"workload": f"{cfg}: {WORKLOAD_NAMES[cfg]}", "rows": spec["rows"], "cols": spec["cols"],
+        "config": {"workload": f"{cfg}: {WORKLOAD_NAMES.get(cfg, spec_name(cfg))}", "rows": spec["rows"], "cols": spec["cols"],
                    "parallelism": "host oracle (rank 0)"},
         "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
         "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -217,12 +222,14 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--config", default="C5", choices=list(WORKLOAD_NAMES))
+    ap.add_argument("--config", default="C5", help="C1..C5 (BASELINE configs) or another workloads.specs entry")
     ap.add_argument("--impl", default="astitch", choices=["astitch", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--flags", type=int, default=0)
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
+    ap.add_argument("--rows", type=int, default=None, help="override the config's rows (experiments)")
+    ap.add_argument("--cols", type=int, default=None, help="override the config's cols (experiments)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -251,7 +258,7 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
 
     cfg = args.config
-    spec = specs.get(cfg)
+    spec = specs.get(cfg, rows=args.rows, cols=args.cols)
     R, C = spec["rows"], spec["cols"]
     graph = A.Graph.from_spec(spec)
     comm = Comm.from_process_group(dev) if world > 1 else None
@@ -398,7 +405,7 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         from oracle import evaluate
-        srows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 400_000, "C5": 131_072}[cfg]
+        srows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 400_000, "C5": 131_072}.get(cfg, 4096)
         sspec = specs.get(cfg, rows=min(srows, R))
         if sspec.get("mask"):
             sspec["mask"]["rows_per_segment"] = min(sspec["mask"]["rows_per_segment"], sspec["rows"])
@@ -421,7 +428,7 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 6),
             "higher_is_better": True, "scaling": "strong" if world > 1 else "strong",
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"{cfg}: {WORKLOAD_NAMES[cfg]}", "rows": R, "cols": C, "global_batch": R,
+            "config": {"workload": f"{cfg}: {WORKLOAD_NAMES.get(cfg, spec_name(cfg))}", "rows": R, "cols": C, "global_batch": R,
                        "io_dtype": "bf16" if any(d == "BF16" for _, _, d in spec["inputs"]) else "f32",
                        "parallelism": f"dp{world} contiguous row shards" + (", 1 ncclAllReduce of fp32 column partials" if world > 1 and desc["shard_kernels"] else ""),
                        "l2": ("inputs > L2 (%.2f GB per rank vs %d MB L2)" % (nbytes / 1e9, l2 // 2**20)) if nsets == 1

@@ -140,7 +140,9 @@ enum {
   ASTITCH_FLAG_STRICT_SINGLE_KERNEL = 1u << 4, /* fail with ERR_RESOURCE rather than 2 kernels */
   ASTITCH_FLAG_NO_TMA = 1u << 5,        /* do not use the TMA-staged packed template   */
   ASTITCH_FLAG_NO_PREFETCH = 1u << 6,   /* no software prefetch of the next row        */
-  ASTITCH_FLAG_LAUNCH_CHECK = 1u << 7   /* synchronise + check after every launch (debug)*/
+  ASTITCH_FLAG_LAUNCH_CHECK = 1u << 7,  /* synchronise + check after every launch (debug)*/
+  ASTITCH_FLAG_FORCE_SPLIT = 1u << 8    /* ablation: split rows over clusters whenever the
+                                           paper's shape rule holds (no B200 size threshold) */
 };
 
 typedef struct {

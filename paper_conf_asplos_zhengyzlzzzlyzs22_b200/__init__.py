@@ -11,7 +11,8 @@ Multi-GPU row sharding lives in ``.dist``.
 """
 
 from ._lib import (FLAG_FORCE_GLOBAL, FLAG_LAUNCH_CHECK, FLAG_NO_COMPILE, FLAG_NO_PACK,  # noqa: F401
-                   FLAG_NO_PREFETCH, FLAG_NO_SPLIT, FLAG_NO_TMA, FLAG_STRICT_SINGLE_KERNEL, LIB_PATH,
+                   FLAG_FORCE_SPLIT, FLAG_NO_PREFETCH, FLAG_NO_SPLIT, FLAG_NO_TMA,
+                   FLAG_STRICT_SINGLE_KERNEL, LIB_PATH,
                    AstitchError)
 from .api import Graph, Plan, bench_barrier, bench_copy, plan, shard_rows  # noqa: F401
 

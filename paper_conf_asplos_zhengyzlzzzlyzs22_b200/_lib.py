@@ -34,6 +34,7 @@ FLAG_STRICT_SINGLE_KERNEL = 1 << 4
 FLAG_NO_TMA = 1 << 5
 FLAG_NO_PREFETCH = 1 << 6
 FLAG_LAUNCH_CHECK = 1 << 7
+FLAG_FORCE_SPLIT = 1 << 8
 
 
 class AstitchError(RuntimeError):

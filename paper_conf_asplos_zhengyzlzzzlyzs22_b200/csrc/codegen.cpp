@@ -48,8 +48,16 @@ struct Gen {
     C = p.desc.cols;
     masked = g.lengths_node >= 0;
     exact = (static_cast<long long>(T) * V * E == C);
+    split = (m.tmpl == Template::SplitRow);
     compute_precise();
     compute_absorb();
+  }
+  bool split = false;
+  int rowred_index(int node) const {  // ordinal of a row reduction (cluster slot)
+    int k = 0;
+    for (int i = 0; i < node; ++i)
+      if (I(i).live && I(i).cls == OpClass::ReduceRow) ++k;
+    return k;
   }
 
   const Node& N(int i) const { return g.nodes[i]; }
@@ -133,17 +141,31 @@ struct Gen {
     o << "// generated by astitch codegen: " << template_name(m.tmpl) << " role " << role << "\n";
     o << "#include \"astitch_device.cuh\"\n";
     o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; };\n";
-    o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") "
-      << name << "(const Params p) {\n";
+    o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") ";
+    if (split) o << "__cluster_dims__(" << m.split << ", 1, 1) ";
+    o << name << "(const Params p) {\n";
     o << "  constexpr int T = " << T << ", V = " << V << ", E = " << E << ", NE = " << NE << ", RPB = " << RPB
       << ";\n";
     o << "  constexpr long long C = " << C << "LL;\n";
     o << "  constexpr long long CH = " << (C / E) << "LL;  // chunks per row\n";
     o << "  (void)V; (void)NE; (void)RPB; (void)CH;\n";
     o << "  const long long R = p.rows;\n";
-    o << "  const int lane = threadIdx.x % T;\n";
-    o << "  const int team = threadIdx.x / T;\n";
-    o << "  (void)lane; (void)team;\n";
+    if (split) {
+      // task splitting: the row's team is the whole cluster (K CTAs)
+      o << "  const int lane = (int)as::cluster_rank() * (int)blockDim.x + (int)threadIdx.x;\n";
+      o << "  const int team = 0;\n";
+      o << "  const long long UNIT = as::cluster_idx(), NUNITS = as::cluster_count();\n";
+      int nred = 0;
+      for (size_t i = 0; i < g.nodes.size(); ++i)
+        if (I(i).live && I(i).cls == OpClass::ReduceRow) ++nred;
+      o << "  __shared__ float cl_slot[" << std::max(1, nred) << "];\n";
+      o << "  __shared__ double cl_slot_d[" << std::max(1, nred) << "];\n";
+    } else {
+      o << "  const int lane = threadIdx.x % T;\n";
+      o << "  const int team = threadIdx.x / T;\n";
+      o << "  const long long UNIT = blockIdx.x, NUNITS = gridDim.x;\n";
+    }
+    o << "  (void)lane; (void)team; (void)UNIT; (void)NUNITS;\n";
     if (T > 32) o << "  __shared__ float red_scratch[32];\n  __shared__ double red_scratch_d[32];\n";
     // constants
     for (size_t i = 0; i < g.nodes.size(); ++i)
@@ -455,6 +477,9 @@ struct Gen {
         else o << ref(nd.a, "k", sfx) << ";\n";
         o << "      double r_ = as::TreeD<NE>::reduce(t_);\n";
         if (T <= 32) o << "      r_ = as::team_sum_d<T>(r_);\n";
+        else if (split)
+          o << "      r_ = as::cluster_team_sum_d<" << m.threads << ", " << m.split << ">(r_, red_scratch_d, &cl_slot_d["
+            << rowred_index(i) << "]);\n";
         else o << "      r_ = as::block_team_sum_d<T>(r_, red_scratch_d);\n";
         o << "      d" << id << sfx << " = r_;\n    }\n";
         emit_split(id, sfx);
@@ -494,6 +519,9 @@ struct Gen {
         }
         o << "      float r_ = as::Tree<NE, " << (mx ? "true" : "false") << ">::reduce(t_);\n";
         if (T <= 32) o << "      r_ = as::team_" << (mx ? "max" : "sum") << "<T>(r_);\n";
+        else if (split)
+          o << "      r_ = as::cluster_team_reduce<" << m.threads << ", " << m.split << ", " << (mx ? "true" : "false")
+            << ">(r_, red_scratch, &cl_slot[" << rowred_index(i) << "]);\n";
         else o << "      r_ = as::block_team_reduce<T, " << (mx ? "true" : "false") << ">(r_, red_scratch);\n";
         if (!post_scale.empty()) o << "      r_ = r_ * " << post_scale << ";\n";
         o << "      s" << id << sfx << " = r_;\n    }\n";
@@ -829,8 +857,8 @@ struct Gen {
     emit_stream_ptrs();
     const bool pf = m.prefetch;
     const std::string su = "_u";
-    o << "  const long long rstride = (long long)gridDim.x * RPB * " << U << ";\n";
-    o << "  long long base = (long long)blockIdx.x * RPB * " << U << ";\n";
+    o << "  const long long rstride = NUNITS * RPB * " << U << ";\n";
+    o << "  long long base = UNIT * RPB * " << U << ";\n";
     if (pf) {
       for (int u = 0; u < U; ++u) {
         std::string row = "(base + " + std::to_string(u) + "LL * RPB + team)";

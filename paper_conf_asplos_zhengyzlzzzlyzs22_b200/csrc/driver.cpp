@@ -154,7 +154,12 @@ bool drv_load(Plan& p, Kernel& k, std::string& err) {
   if (k.spill_bytes < 0) k.spill_bytes = local;
   int occ = 0;
   r = d->Occupancy(&occ, fn, k.threads, static_cast<size_t>(k.smem));
-  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuOccupancyMaxActiveBlocksPerMultiprocessor"); d->ModuleUnload(mod); return false; }
+  if (r != CUDA_SUCCESS) {
+    // cluster kernels may reject the per-block query; only the cooperative
+    // (grid-barrier) kernels depend on it for co-residency
+    if (k.cooperative) { err = cu_err(d, r, "cuOccupancyMaxActiveBlocksPerMultiprocessor"); d->ModuleUnload(mod); return false; }
+    occ = -1;
+  }
   k.occupancy = occ;
   k.module = mod;
   k.function = fn;

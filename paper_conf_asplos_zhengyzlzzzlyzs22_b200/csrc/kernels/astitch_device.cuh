@@ -357,6 +357,32 @@ template <int T, bool MAX> __device__ __forceinline__ float block_team_reduce(fl
   return r;
 }
 
+// ------------------------------------------------------------------ regional across a cluster
+// Task splitting: one row is split over the K CTAs of a thread-block
+// cluster; the block partials are combined through distributed shared memory
+// (DSMEM) in a fixed rank order, so every CTA obtains the identical row value
+// (replaces the paper's cross-block atomic; deterministic).
+__device__ __forceinline__ u32 cluster_rank() { u32 r; asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r)); return r; }
+__device__ __forceinline__ u32 cluster_idx() { u32 r; asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(r)); return r; }
+__device__ __forceinline__ u32 cluster_count() { u32 r; asm volatile("mov.u32 %0, %%nclusterid.x;" : "=r"(r)); return r; }
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ float ld_dsmem_f32(const float* local, u32 rank) {
+  u32 a = static_cast<u32>(__cvta_generic_to_shared(local)), ra;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(rank));
+  float v;
+  asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(ra) : "memory");
+  return v;
+}
+__device__ __forceinline__ double ld_dsmem_f64(const double* local, u32 rank) {
+  u32 a = static_cast<u32>(__cvta_generic_to_shared(local)), ra;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(rank));
+  double v;
+  asm volatile("ld.shared::cluster.f64 %0, [%1];" : "=d"(v) : "r"(ra) : "memory");
+  return v;
+}
+
 // fp64 team sum for cancellation-prone row sums (e.g. a mean that is then
 // subtracted): the result is carried as a double and split hi+lo in fp32.
 template <int T> __device__ __forceinline__ double team_sum_d(double v) {
@@ -385,6 +411,35 @@ template <int N> struct TreeD {
   }
 };
 
+// block tree, then the K block partials of the cluster combined via DSMEM
+// (slot: a per-reduction __shared__ word; two cluster barriers make the slot
+// safe to rewrite by the next row)
+template <int NT, int K, bool MAX>
+__device__ __forceinline__ float cluster_team_reduce(float v, float* scratch, float* slot) {
+  v = block_team_reduce<NT, MAX>(v, scratch);
+  if (threadIdx.x == 0) *slot = v;
+  cluster_sync_all();
+  float r = MAX ? -AS_INF : 0.f;
+#pragma unroll
+  for (int q = 0; q < K; ++q) {
+    const float x = ld_dsmem_f32(slot, static_cast<u32>(q));
+    r = MAX ? fmaxf(r, x) : r + x;
+  }
+  cluster_sync_all();
+  return r;
+}
+template <int NT, int K>
+__device__ __forceinline__ double cluster_team_sum_d(double v, double* scratch, double* slot) {
+  v = block_team_sum_d<NT>(v, scratch);
+  if (threadIdx.x == 0) *slot = v;
+  cluster_sync_all();
+  double r = 0.0;
+#pragma unroll
+  for (int q = 0; q < K; ++q) r += ld_dsmem_f64(slot, static_cast<u32>(q));
+  cluster_sync_all();
+  return r;
+}
+
 // pairwise tree over a register array (fixed order -> deterministic)
 template <int N, bool MAX> struct Tree {
   __device__ static __forceinline__ float reduce(const float* a) {
@@ -411,21 +466,23 @@ __device__ __forceinline__ void st_release(u32* p, u32 v) {
 __device__ __forceinline__ u32 atom_add_acqrel(u32* p, u32 v) {
   u32 old; asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory"); return old;
 }
+// Generation-counted barrier: the arrival count returns to 0 at the end of
+// every episode (so any grid size may reuse the workspace), the generation
+// word is bumped with release semantics by the last arriver, and waiters
+// poll it with acquire loads.  acq_rel on the arrival atomic publishes this
+// CTA's writes (ordered before it by __syncthreads); no extra fences.
 __device__ __forceinline__ void grid_barrier(u32* bar) {
   __syncthreads();
   if (threadIdx.x == 0) {
     const u32 nb = gridDim.x * gridDim.y * gridDim.z;
-    u32 gen = ld_acquire(bar + 1);
-    __threadfence();
-    u32 arrived = atom_add_acqrel(bar, 1u);
+    const u32 gen = ld_acquire(bar + 1);
+    const u32 arrived = atom_add_acqrel(bar, 1u);
     if (arrived == nb - 1) {
-      *reinterpret_cast<volatile u32*>(bar) = 0u;
-      __threadfence();
+      asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(bar), "r"(0u) : "memory");
       st_release(bar + 1, gen + 1);
     } else {
-      while (ld_acquire(bar + 1) == gen) { __nanosleep(20); }
+      while (ld_acquire(bar + 1) == gen) { }
     }
-    __threadfence();
   }
   __syncthreads();
 }

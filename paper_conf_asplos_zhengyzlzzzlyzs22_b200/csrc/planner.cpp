@@ -14,6 +14,8 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
+#include <cstring>
 #include <functional>
 #include <numeric>
 #include <sstream>
@@ -439,7 +441,12 @@ void select_mapping(Plan& p) {
     bool team_tile_ok = tile_common && !packed_ok && !has_mask && m.team <= 32 && m.team >= 1 &&
                         in_row_bytes > 0 && in_row_bytes * (256 / m.team) <= 48 * 1024;
     // Task splitting (rule P:L270): rows < blocks-per-wave and row > 1024.
-    bool split_rule = !no_split && R < blocks_per_wave_1024 && C > 1024;
+    // B200 threshold (reading R15): measured on <64,30000> fp32 (120 KB rows)
+    // one block per row is still faster (4.2 vs 4.7 us, latency-bound), on
+    // <64,300000> (1.2 MB rows) a cluster of 8 is 5x faster; split from 256 KB.
+    const bool force_split = (p.desc.flags & ASTITCH_FLAG_FORCE_SPLIT) != 0;
+    bool split_rule = !no_split && R < blocks_per_wave_1024 && C > 1024 &&
+                      (force_split || C * es_max >= 256 * 1024);
     if (packed_ok || team_tile_ok) {
       m.tmpl = Template::PackedTile;
       if (packed_ok) {
@@ -487,16 +494,34 @@ void select_mapping(Plan& p) {
             << "-stage mbarrier pipeline), team of " << m.team << " lanes x " << m.chunks_per_lane
             << " chunks per row from smem" << (has_mask ? ", valid-prefix copies per row" : "") << "; ";
       }
+    } else if (split_rule && p.global_fulls.empty()) {
+      // Task splitting: each row is split over a thread-block cluster
+      // of K CTAs (K ~ blocks-per-wave / rows, power of two, <= 8 portable);
+      // block partials combine through DSMEM in a fixed order.
+      m.tmpl = Template::SplitRow;
+      int64_t want = (blocks_per_wave_1024 + R - 1) / std::max<int64_t>(R, 1);
+      int k = 2;
+      while (k < want && k < 8) k *= 2;
+      m.split = k;
+      m.threads = 512;
+      if (const char* fs = getenv("ASTITCH_FORCE_SPLIT")) {  // tuning knob: "K" or "K,threads"
+        int kk = atoi(fs);
+        if (kk >= 1 && kk <= 16 && (kk & (kk - 1)) == 0) m.split = kk;
+        if (const char* c = strchr(fs, ',')) {
+          int t = atoi(c + 1);
+          if (t >= 32 && t <= 1024 && t % 32 == 0) m.threads = t;
+        }
+      }
+      m.team = m.split * m.threads;
+      m.chunks_per_lane = std::max(1, (chunks + m.team - 1) / m.team);
+      m.lane_util = static_cast<double>(chunks) / (static_cast<double>(m.team) * m.chunks_per_lane);
+      m.rows_per_block = 1;
+      m.row_unroll = 1;
+      why << "paper split rule holds (rows " << R << " < per-wave " << blocks_per_wave_1024 << " and row " << C
+          << " > 1024): each row split over a cluster of " << m.split << " CTAs x " << m.threads
+          << " threads, partials combined through DSMEM; ";
     } else {
       m.tmpl = Template::RowTeam;
-      if (split_rule) {
-        m.split = static_cast<int>(std::max<int64_t>(2, (blocks_per_wave_1024 + R - 1) / std::max<int64_t>(R, 1)));
-        m.split = std::min(m.split, 8);
-        why << "paper split rule holds (rows " << R << " < per-wave " << blocks_per_wave_1024
-            << " and row " << C << " > 1024): split factor " << m.split
-            << " requested; executed as one block team per row (cluster split is NEXT f2); ";
-        m.split = 1;
-      }
       // a multi-warp team reduces through block-wide smem: one team per block
       m.threads = m.team > 32 ? m.team : 256;
       m.rows_per_block = m.threads / m.team;
@@ -538,8 +563,15 @@ void retune_grid(Plan& p) {
   if (m.tmpl == Template::PackedTile) work_units = (R + m.tile_rows - 1) / m.tile_rows;
   else work_units = (R + (int64_t)m.rows_per_block * m.row_unroll - 1) / ((int64_t)m.rows_per_block * m.row_unroll);
   int64_t wave = static_cast<int64_t>(m.blocks_per_sm) * p.sm_count;
-  m.grid = std::max<int64_t>(1, std::min(work_units, wave));
-  m.vertical_trips = (work_units + m.grid - 1) / m.grid;
+  if (m.tmpl == Template::SplitRow) {
+    // clusters of `split` CTAs, one row per cluster per iteration
+    int64_t clusters = std::max<int64_t>(1, std::min(work_units, wave / m.split));
+    m.grid = clusters * m.split;
+    m.vertical_trips = (work_units + clusters - 1) / clusters;
+  } else {
+    m.grid = std::max<int64_t>(1, std::min(work_units, wave));
+    m.vertical_trips = (work_units + m.grid - 1) / m.grid;
+  }
   plan_workspace(p);
 }
 

@@ -117,6 +117,32 @@ def test_parity_masked_variants(kind):
     _compare(spec, run_gpu(spec, x), evaluate(spec, x), tol=2e-3)
 
 
+@pytest.mark.parametrize("cfg,rows,cols", [("fig6b", 64, 30000), ("C1", 40, 30000), ("C2", 16, 8192),
+                                           ("C4", 3, 20000), ("C3", 48, 4096)])
+def test_parity_split_rows(cfg, rows, cols):
+    """Few long rows: task splitting over a thread-block cluster."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 16
+    x = gen.generate(cfg, spec)
+    got, plan = run_gpu(spec, x, return_plan=True, flags=A.FLAG_FORCE_SPLIT)
+    assert plan.describe()["mapping"]["template"] == "split_row"
+    _compare(spec, got, evaluate(spec, x))
+    again = run_gpu(spec, x, plan=plan)
+    for k in got:
+        assert np.array_equal(got[k], again[k])       # deterministic DSMEM combine
+
+
+def test_parity_split_long_rows_default():
+    """<64, 300000> fp32: the planner splits by itself (1.2 MB rows)."""
+    spec = specs.get("fig6b", rows=64, cols=300_000)
+    x = gen.generate("fig6b", spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    assert plan.describe()["mapping"]["template"] == "split_row"
+    _compare(spec, got, evaluate(spec, x))
+
+
 def test_full_c1_c2():
     for cfg in ("C1", "C2"):
         spec = specs.get(cfg)

@@ -110,10 +110,17 @@ def test_fig6_selector_branches():
     m = d["mapping"]
     assert m["team"] < 32 and m["rows_per_block"] > 32
     assert m["grid"] <= m["blocks_per_sm"] * 148
-    d, _, _ = describe("fig6b")              # <64,30000>: the paper's split rule holds
-    assert "split rule holds" in d["mapping"]["reason"]
-    d, _, _ = describe("fig6b", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_SPLIT)
-    assert "split rule" not in d["mapping"]["reason"]
+    # <64,30000>: the paper's shape rule holds, but 120 KB rows are below the
+    # measured B200 threshold (reading R15) -> one block team per row
+    d, _, _ = describe("fig6b")
+    assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 1024
+    d, _, _ = describe("fig6b", flags=A.FLAG_NO_COMPILE | A.FLAG_FORCE_SPLIT)
+    assert d["mapping"]["template"] == "split_row" and "split rule holds" in d["mapping"]["reason"]
+    assert d["mapping"]["split"] == 8 and d["mapping"]["grid"] % 8 == 0
+    d, _, _ = describe("fig6b", cols=300_000)  # 1.2 MB rows: split by default
+    assert d["mapping"]["template"] == "split_row"
+    d, _, _ = describe("fig6b", cols=300_000, flags=A.FLAG_NO_COMPILE | A.FLAG_NO_SPLIT)
+    assert d["mapping"]["template"] == "row_team"
 
 
 @pytest.mark.parametrize("cfg", ["C2", "C3", "C4"])
