@@ -213,6 +213,18 @@ astitch_status astitch_comm_create(int32_t world, int32_t rank, const uint8_t id
 astitch_status astitch_comm_destroy(astitch_comm_t c);
 astitch_status astitch_run_sharded(astitch_plan_t p, astitch_comm_t c, const void* const* inputs,
                                    void* const* outputs, void* ws, void* stream);
+/* The two halves of astitch_run_sharded around the collective, for callers
+ * that combine the partials themselves (another collective library, or a
+ * single-GPU "virtual shards" check):
+ *   stage 0: stitched kernel over the shard's rows; leaves the rank-local fp32
+ *            column totals at ws + offset (ncolred x cols floats, see below);
+ *   stage 1: column consumers (+ the FULL sweep after the barrier) reading the
+ *            combined totals from the same place.
+ * astitch_plan_colpart reports the byte offset in ws and the float count.
+ * Plans without a column reduction: stage 0 = astitch_run, stage 1 = no-op. */
+astitch_status astitch_run_shard_stage(astitch_plan_t p, int32_t stage, const void* const* inputs,
+                                       void* const* outputs, void* ws, void* stream);
+astitch_status astitch_plan_colpart(astitch_plan_t p, size_t* byte_offset, size_t* count);
 /* Contiguous row partition: rows_k = floor(R/g) (+1 for the first R mod g ranks). */
 astitch_status astitch_shard_rows(int64_t rows, int32_t world, int32_t rank, int64_t* row_begin,
                                   int64_t* row_count);

@@ -89,6 +89,8 @@ _sig = {
     "astitch_comm_create": (ct.c_int, [ct.c_int32, ct.c_int32, ct.c_char_p, ct.c_int32, ct.POINTER(_vp)]),
     "astitch_comm_destroy": (ct.c_int, [_vp]),
     "astitch_run_sharded": (ct.c_int, [_vp, _vp, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
+    "astitch_run_shard_stage": (ct.c_int, [_vp, ct.c_int32, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
+    "astitch_plan_colpart": (ct.c_int, [_vp, ct.POINTER(ct.c_size_t), ct.POINTER(ct.c_size_t)]),
     "astitch_shard_rows": (ct.c_int, [ct.c_int64, ct.c_int32, ct.c_int32, ct.POINTER(ct.c_int64),
                                       ct.POINTER(ct.c_int64)]),
     "astitch_bench_barrier": (ct.c_int, [ct.c_int32, ct.c_int32, ct.c_int32, ct.c_int32, _vp, _vp]),

@@ -163,4 +163,31 @@ astitch_status astitch_run_sharded(astitch_plan_t h, astitch_comm_t c, const voi
   return ASTITCH_OK;
 }
 
+astitch_status astitch_plan_colpart(astitch_plan_t h, size_t* byte_offset, size_t* count) {
+  if (!h || !byte_offset || !count) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  const Plan& p = *h->p;
+  const size_t C = static_cast<size_t>(p.desc.cols);
+  *byte_offset = p.ws.colvals + p.post_colvecs.size() * C * 4;
+  *count = p.colreds.size() * C;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_run_shard_stage(astitch_plan_t h, int32_t stage, const void* const* inputs,
+                                       void* const* outputs, void* ws, void* stream) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  if (stage != 0 && stage != 1) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "stage must be 0 or 1");
+  const Plan& p = *h->p;
+  if (p.colreds.empty() || p.desc.shard_world <= 1)
+    return stage == 0 ? astitch_run(h, inputs, outputs, ws, stream) : ASTITCH_OK;
+  if (p.shard_kernels.empty() || !p.shard_kernels[0].function)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "plan has no loaded sharded kernels");
+  astitch_status s = check_io(p, inputs, outputs, ws);
+  if (s != ASTITCH_OK) return s;
+  KernelParams kp = make_params(p, inputs, outputs, ws);
+  if (stage == 0) return launch(p, p.shard_kernels[0], kp, stream);
+  for (size_t i = 1; i < p.shard_kernels.size(); ++i)
+    if ((s = launch(p, p.shard_kernels[i], kp, stream)) != ASTITCH_OK) return s;
+  return ASTITCH_OK;
+}
+
 }  // extern "C"

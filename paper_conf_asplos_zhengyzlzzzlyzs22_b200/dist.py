@@ -75,6 +75,21 @@ class ShardedPlan:
                                       ct.c_void_p(ws.data_ptr() if ws is not None else 0),
                                       ct.c_void_p(_stream_ptr(stream))), "astitch_run_sharded")
 
+    def run_stage(self, stage: int, inputs, outputs, ws, stream=None) -> None:
+        """astitch_run_shard_stage: 0 = stitched kernel leaving rank-local column
+        totals in ws; 1 = column consumers reading the combined totals."""
+        ins = ptr_array([t.data_ptr() for t in inputs])
+        outs = ptr_array([t.data_ptr() for t in outputs])
+        check(lib.astitch_run_shard_stage(self.plan.handle, int(stage), ins, outs,
+                                          ct.c_void_p(ws.data_ptr() if ws is not None else 0),
+                                          ct.c_void_p(_stream_ptr(stream))), "astitch_run_shard_stage")
+
+    def colpart(self):
+        """(byte offset in the workspace, float count) of the column totals."""
+        off, n = ct.c_size_t(), ct.c_size_t()
+        check(lib.astitch_plan_colpart(self.plan.handle, ct.byref(off), ct.byref(n)), "astitch_plan_colpart")
+        return off.value, n.value
+
     def kernels_per_run(self) -> int:
         d = self.plan.describe()
         if self.world > 1 and d["shard_kernels"] > 0:
