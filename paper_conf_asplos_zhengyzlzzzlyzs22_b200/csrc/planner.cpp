@@ -403,7 +403,7 @@ void select_mapping(Plan& p) {
     choose_team(1024, has_mask ? 32 : 16, 32);
     if (const char* ft = getenv("ASTITCH_FORCE_TEAM")) {  // tuning knob for experiments
       int t = atoi(ft);
-      if (t >= 1 && t <= 1024 && (t & (t - 1)) == 0) {
+      if (t >= 1 && t <= 1024 && ((t & (t - 1)) == 0 || t % 32 == 0)) {
         m.team = t;
         m.chunks_per_lane = (chunks + t - 1) / t;
         m.lane_util = static_cast<double>(chunks) / (t * m.chunks_per_lane);
@@ -438,7 +438,13 @@ void select_mapping(Plan& p) {
     // copies (deep async pipeline: bytes in flight no longer tied to registers)
     // (measured on B200: for masked rows the register-prefetching row team is
     // faster than per-row valid-prefix bulk copies, so masks stay on row teams)
-    bool team_tile_ok = tile_common && !packed_ok && !has_mask && m.team <= 32 && m.team >= 1 &&
+    // Measured on B200 (C2: 8.7 vs 8.0 us, C3: 3.8 vs 4.6 TB/s) the register
+    // row team beats TMA-staged team tiles whenever a power-of-two team tiles
+    // the row, so team tiles are opt-in (ASTITCH_TEAM_TILES=1); the T=1
+    // packed tiles (rows a team cannot tile, C4) stay the default.
+    const char* tt_env = getenv("ASTITCH_TEAM_TILES");
+    bool team_tile_ok = tile_common && tt_env && atoi(tt_env) == 1 && !packed_ok && !has_mask &&
+                        m.team <= 32 && m.team >= 1 &&
                         in_row_bytes > 0 && in_row_bytes * (256 / m.team) <= 48 * 1024;
     // Task splitting (rule P:L270): rows < blocks-per-wave and row > 1024.
     // B200 threshold (reading R15): measured on <64,30000> fp32 (120 KB rows)

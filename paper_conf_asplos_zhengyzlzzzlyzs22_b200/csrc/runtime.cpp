@@ -82,7 +82,7 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
   // assume-relax-apply as a bisection on blocks per SM: the largest occupancy
   // whose register bound (65536 / (bps * threads)) compiles without spills
   int good = 0, bad = 0;  // best spill-free / smallest spilling bps seen
-  for (int attempt = 0; attempt < 6; ++attempt) {
+  for (int attempt = 0; attempt < 10; ++attempt) {
     std::string base = std::string("astitch_") + template_name(p.map.tmpl) + role_suffix(role);
     k.name = base;
     k.source = generate_kernel(p, role, base);

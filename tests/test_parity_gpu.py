@@ -37,6 +37,7 @@ REDUCED = [
     ("fig7a", None, None),
     ("fig6a", 10_000 + 1, None),
     ("fig6b", 8, None),
+    ("remote", None, None),
 ]
 
 
@@ -203,6 +204,17 @@ def test_virtual_shards(cfg, rows, cols, world):
             if name in ("dz",) or not any(o[1] == "reduce" and o[3] == "COL" for o in spec["ops"]):
                 assert np.array_equal(got, full[name]), name       # row outputs bitwise = unsharded
             check_close(got, ref[name], dt, spec_tol(spec), f"{cfg}:{name} sharded")
+
+
+@pytest.mark.parametrize("cfg,rows", [("C2", 4500), ("remote", 5000), ("C1", 9000)])
+def test_team_tiles_optin(cfg, rows, monkeypatch):
+    """TMA-staged team tiles (opt-in template) stay correct."""
+    monkeypatch.setenv("ASTITCH_TEAM_TILES", "1")
+    spec = specs.get(cfg, rows=rows)
+    x = gen.generate(cfg, spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    assert plan.describe()["mapping"]["template"] == "packed_tile"
+    _compare(spec, got, evaluate(spec, x))
 
 
 def test_full_c1_c2():

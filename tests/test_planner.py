@@ -37,10 +37,8 @@ def test_c2_layernorm_heavy_rowvec_candidate():
     assert ops["o"]["class"] == "heavy_ew"
     assert len(d["groups"]) == 1
     m = d["mapping"]
-    assert m["template"] == "packed_tile" and m["team"] == 32 and m["chunks_per_lane"] == 3 and m["vec_elems"] == 8
+    assert m["template"] == "row_team" and m["team"] == 32 and m["chunks_per_lane"] == 3 and m["vec_elems"] == 8
     assert m["lane_util"] == 1.0
-    d, _, _ = describe("C2", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_TMA)
-    assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 32
 
 
 def test_c3_mask_row_team_absorbed():
@@ -131,6 +129,15 @@ def test_mapping_independent_of_rows(cfg):
     b, _, _ = describe(cfg, rows=8192 + 17)
     for k in ("template", "team", "chunks_per_lane", "vec_elems"):
         assert a["mapping"][k] == b["mapping"][k], k
+
+
+def test_remote_stitching_one_kernel():
+    """Two independent subgraphs in one stitch op (remote stitching):
+    separate groups, one kernel, outputs of both are independent."""
+    d, ops, p = describe("remote")
+    assert len(d["groups"]) == 2
+    assert ops["m"]["group"] != ops["ys"]["group"]
+    assert d["kernel_count"] == 1 and d["mapping"]["template"] in ("row_team", "packed_tile")
 
 
 def test_no_pack_ablation():

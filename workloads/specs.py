@@ -259,6 +259,29 @@ FIG6B_FEW_LONG_ROWS = {
     "outputs": [("s", "F32")],
 }
 
+# Remote stitching: two subgraphs with no data dependency merged into
+# one stitch op (the "independent" scheme between them), one kernel.
+REMOTE_TWO_SUBGRAPHS = {
+    "name": "remote_softmax_and_rowsum",
+    "rows": 3000,
+    "cols": 256,
+    "inputs": [("x", "FULL", "BF16"), ("y", "FULL", "F32")],
+    "mask": None,
+    "ops": [
+        ("m", "reduce", "RMAX", "ROW", "x"),
+        ("mb", "broadcast", "ROW", "m"),
+        ("xm", "binary", "SUB", "x", "mb"),
+        ("e", "unary", "EXP", "xm"),
+        ("s", "reduce", "SUM", "ROW", "e"),
+        ("sb", "broadcast", "ROW", "s"),
+        ("p", "binary", "DIV", "e", "sb"),
+        ("ys", "reduce", "SUM", "ROW", "y"),
+        ("ya", "unary", "ABS", "y"),
+        ("yn", "reduce", "RMAX", "ROW", "ya"),
+    ],
+    "outputs": [("p", "BF16"), ("ys", "F32"), ("yn", "F32")],
+}
+
 CONFIGS = {
     "C1": C1_SOFTMAX,
     "C2": C2_BERT_LN_GELU,
@@ -273,6 +296,7 @@ EXTRA = {
     "fig7a": FIG7A_MIXED,
     "fig6a": FIG6A_MANY_SHORT_ROWS,
     "fig6b": FIG6B_FEW_LONG_ROWS,
+    "remote": REMOTE_TWO_SUBGRAPHS,
 }
 
 ALL = {**CONFIGS, **EXTRA}
