@@ -149,7 +149,7 @@ struct Gen {
     o << "  constexpr long long C = " << C << "LL;\n";
     o << "  constexpr long long CH = " << (C / E) << "LL;  // chunks per row\n";
     o << "  (void)V; (void)NE; (void)RPB; (void)CH;\n";
-    o << "  const long long R = p.rows;\n";
+    o << "  const " << rowt() << " R = (" << rowt() << ")p.rows;\n";
     if (split) {
       // task splitting: the row's team is the whole cluster (K CTAs)
       o << "  const int lane = (int)as::cluster_rank() * (int)blockDim.x + (int)threadIdx.x;\n";
@@ -298,7 +298,9 @@ struct Gen {
       o << "      if (" << cond << ") r" << s << sfx << "[j] = "
         << (st.ws_buf ? "as::ldg_cg(" : "as::ldg(") << "gs" << s << " + (" << row
         << ") * CH + (j * T + lane));\n";
-      o << "      else r" << s << sfx << "[j] = " << raw_t(st) << "{};\n";
+      // chunks that are not loaded need no defined bits when the mask is
+      // absorbed: the unpack step overwrites every invalid element with S
+      if (!(absorb && !st.ws_buf)) o << "      else r" << s << sfx << "[j] = " << raw_t(st) << "{};\n";
       o << "    }\n";
     }
   }
@@ -314,9 +316,11 @@ struct Gen {
         << "[j], " << dst << " + j * E);\n";
       if (absorb && masked && !st.ws_buf && !lim.empty()) {
         // mask absorption: invalid elements take the substitute value
+        // d_ = elements of this lane's chunk that are valid (may be <= 0)
         o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n      if (!((j + 1) * T * E <= " << lim
-          << ")) {\n#pragma unroll\n        for (int e = 0; e < E; ++e) if (" << col_expr("j", "e") << " >= " << lim
-          << ") " << dst << "[j * E + e] = " << fconst(absorb_sub) << ";\n      }\n    }\n";
+          << ")) {\n        const int d_ = " << lim << " - (j * T + lane) * E;\n#pragma unroll\n"
+          << "        for (int e = 0; e < E; ++e) if (e >= d_) " << dst << "[j * E + e] = " << fconst(absorb_sub)
+          << ";\n      }\n    }\n";
       }
     }
   }
@@ -852,18 +856,83 @@ struct Gen {
 
   // ------------------------------------------------------------ row sweep
   // Block-uniform loop over row groups; each team owns rows base + team.
+  // Row indices fit 32 bits for every plan below 2^30 rows (cheaper compares
+  // and increments than 64-bit); addresses are still formed in 64 bits.
+  std::string rowt() const { return p.desc.rows < (1LL << 30) ? "int" : "long long"; }
+
+  // one ping-pong half of the software-pipelined row loop: loads of the rows
+  // one stride ahead go to buffer `nx` while the rows of `base` are computed
+  // from buffer `cu` (no register copies between the halves)
+  void emit_pingpong_half(bool post, const std::string& cu, const std::string& nx) {
+    const std::string su = "_u";
+    const std::string rt = rowt();
+    for (int u = 0; u < U; ++u) {
+      o << "    const " << rt << " row" << u << " = base + " << u << " * RPB + team;\n";
+      o << "    const bool act" << u << " = row" << u << " < R;\n";
+      o << "    const int lim" << u << " = "
+        << (masked ? "act" + std::to_string(u) + " ? " + lim_expr("row" + std::to_string(u)) + " : 0" : "(int)C")
+        << ";\n    (void)lim" << u << ";\n";
+    }
+    for (int u = 0; u < U; ++u) {
+      o << "    {\n      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
+      o << "      const bool pact = nrow < R;\n";
+      o << "      const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
+      o << "      (void)plim;\n";
+      emit_loads("nrow", "pact", "plim", su + std::to_string(u) + nx, false);
+      o << "    }\n";
+    }
+    for (int u = 0; u < U; ++u) {
+      std::string s = su + std::to_string(u) + cu;
+      std::string row = "row" + std::to_string(u), act = "act" + std::to_string(u), lim = "lim" + std::to_string(u);
+      o << "    {\n";
+      emit_unpack(s, lim);
+      emit_colvecs(true);
+      emit_rowvec_inputs(post, s, row, act);
+      emit_body(post, s, row, act, lim);
+      emit_stores(post, s, row, act, lim);
+      o << "    }\n";
+    }
+  }
+
   void emit_sweep(bool post) {
     collect_streams(post);
     emit_stream_ptrs();
     const bool pf = m.prefetch;
     const std::string su = "_u";
-    o << "  const long long rstride = NUNITS * RPB * " << U << ";\n";
-    o << "  long long base = UNIT * RPB * " << U << ";\n";
+    const std::string rt = rowt();
+    o << "  const " << rt << " rstride = (" << rt << ")(NUNITS * RPB * " << U << ");\n";
+    o << "  " << rt << " base = (" << rt << ")(UNIT * RPB * " << U << ");\n";
+    // The ping-pong form removes the per-row register copies but raised the
+    // register count on B200 (C3: 120 vs 80 regs, 153 vs 146 us), so the copy
+    // form is the default; ASTITCH_PINGPONG=1 selects the other for experiments.
+    const char* pp_env = getenv("ASTITCH_PINGPONG");
+    if (pf && pp_env && atoi(pp_env) == 1) {
+      // ping-pong buffers a / b
+      for (int u = 0; u < U; ++u)
+        for (const char* bf : {"a", "b"})
+          for (size_t q = 0; q < streams.size(); ++q)
+            o << "  " << raw_t(streams[q]) << " r" << q << su << u << bf << "[V];\n";
+      for (int u = 0; u < U; ++u) {
+        o << "  {\n    const " << rt << " nrow = base + " << u << " * RPB + team;\n";
+        o << "    const bool pact = nrow < R;\n";
+        o << "    const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
+        o << "    (void)plim;\n";
+        emit_loads("nrow", "pact", "plim", su + std::to_string(u) + "a", false);
+        o << "  }\n";
+      }
+      o << "  while (base < R) {\n";
+      o << "   {\n";
+      emit_pingpong_half(post, "a", "b");
+      o << "   }\n    base += rstride;\n    if (base >= R) break;\n";
+      o << "   {\n";
+      emit_pingpong_half(post, "b", "a");
+      o << "   }\n    base += rstride;\n  }\n";
+      return;
+    }
     if (pf) {
       for (int u = 0; u < U; ++u) {
-        std::string row = "(base + " + std::to_string(u) + "LL * RPB + team)";
-        std::string s = su + std::to_string(u) + "n";
-        o << "  const long long prow" << u << " = " << row << ";\n";
+        std::string row = "(base + " + std::to_string(u) + " * RPB + team)";
+        o << "  const " << rt << " prow" << u << " = " << row << ";\n";
       }
       for (int u = 0; u < U; ++u) {
         std::string s = su + std::to_string(u) + "n";
@@ -878,7 +947,7 @@ struct Gen {
     o << "  for (; base < R; base += rstride) {\n";
     for (int u = 0; u < U; ++u) {
       std::string s = su + std::to_string(u);
-      o << "    const long long row" << u << " = base + " << u << "LL * RPB + team;\n";
+      o << "    const " << rt << " row" << u << " = base + " << u << " * RPB + team;\n";
       o << "    const bool act" << u << " = row" << u << " < R;\n";
       o << "    const int lim" << u << " = " << (masked ? "act" + std::to_string(u) + " ? " + lim_expr("row" + std::to_string(u)) + " : 0" : "(int)C") << ";\n";
       o << "    (void)lim" << u << ";\n";
@@ -894,7 +963,7 @@ struct Gen {
       for (int u = 0; u < U; ++u) {
         std::string s = su + std::to_string(u) + "n";
         o << "    {\n";
-        o << "      const long long nrow = base + rstride + " << u << "LL * RPB + team;\n";
+        o << "      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
         o << "      const bool pact = nrow < R;\n";
         o << "      const int plim =" << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
         o << "      (void)plim;\n";

@@ -469,6 +469,12 @@ void select_mapping(Plan& p) {
         m.tile_rows = std::max(teams, (tr / teams) * teams);
       }
       m.stages = 4;  // prefetch distance 2 tiles + 2 tiles draining (bulk stores)
+      if (const char* fs = getenv("ASTITCH_TILE")) {  // tuning knob: "stages,tile_rows,threads"
+        int s = 0, tr = 0, th = 0;
+        if (sscanf(fs, "%d,%d,%d", &s, &tr, &th) >= 1 && s >= 3 && s <= 8) m.stages = s;
+        if (th >= 32 && th <= 1024 && th % 32 == 0 && th % m.team == 0) m.threads = th;
+        if (tr >= 1 && tr % (m.threads / m.team) == 0) m.tile_rows = tr;
+      }
       m.rows_per_block = m.threads / m.team;
       // stage bytes: input tiles + output tiles that cannot be written in
       // place over an input tile of the same element size (mirrors codegen)
