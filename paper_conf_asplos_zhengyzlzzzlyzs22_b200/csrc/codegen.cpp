@@ -139,6 +139,9 @@ struct Gen {
   void header(const std::string& name, bool cooperative_sync) {
     (void)cooperative_sync;
     o << "// generated by astitch codegen: " << template_name(m.tmpl) << " role " << role << "\n";
+    if (const char* q = getenv("ASTITCH_ST_HINT"))  // experiments: output store cache qualifier
+      if (std::string(q) == ".cs" || std::string(q) == ".wt" || std::string(q) == ".cg")
+        o << "#define AS_STQ \"" << q << "\"\n";
     o << "#include \"astitch_device.cuh\"\n";
     o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; };\n";
     o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") ";

@@ -116,8 +116,13 @@ __device__ __forceinline__ void stg(Raw<4>* p, const Raw<4>& r) {
 __device__ __forceinline__ void stg(Raw<8>* p, const Raw<8>& r) {
   asm volatile("st.global.v2.b32 [%0], {%1,%2};" ::"l"(p), "r"(r.x), "r"(r.y) : "memory");
 }
+// store cache qualifier for the streaming outputs (empty = default policy;
+// e.g. ".cs" evict-first), selectable at JIT time for experiments
+#ifndef AS_STQ
+#define AS_STQ ""
+#endif
 __device__ __forceinline__ void stg(Raw<16>* p, const Raw<16>& r) {
-  asm volatile("st.global.v4.b32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w)
+  asm volatile("st.global" AS_STQ ".v4.b32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w)
                : "memory");
 }
 __device__ __forceinline__ void stg(Raw<32>* p, const Raw<32>& r) {
