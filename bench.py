@@ -225,6 +225,8 @@ def main():
     ap.add_argument("--config", default="C5", help="C1..C5 (BASELINE configs) or another workloads.specs entry")
     ap.add_argument("--impl", default="astitch", choices=["astitch", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-chunks", type=int, default=16,
+                    help="row chunks of the pipelined host path (H2D / kernel / D2H overlap); 1 = serial")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--flags", type=int, default=0)
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
@@ -380,7 +382,7 @@ def main():
     if world > 1:
         e2e_run = None
     for _ in range(2):
-        plan.run_host(host_in, host_out, dev_in[0], dev_out[0], ws=ws) if world == 1 else \
+        plan.run_host(host_in, host_out, dev_in[0], dev_out[0], ws=ws, chunks=args.e2e_chunks) if world == 1 else \
             _sharded_host(sp, host_in, host_out, dev_in[0], dev_out[0], ws)
     torch.cuda.synchronize()
     if world > 1:
@@ -389,7 +391,7 @@ def main():
     h0.record(stream)
     for _ in range(args.e2e_steps):
         if world == 1:
-            plan.run_host(host_in, host_out, dev_in[0], dev_out[0], ws=ws)
+            plan.run_host(host_in, host_out, dev_in[0], dev_out[0], ws=ws, chunks=args.e2e_chunks)
         else:
             _sharded_host(sp, host_in, host_out, dev_in[0], dev_out[0], ws)
     h1.record(stream)
@@ -447,7 +449,10 @@ def main():
                          "kernel_us": round(kern_ms * 1e3, 3),
                          "algorithmic_bytes_per_launch": int(nbytes)},
             "e2e": {"value": round(e2e_gbs, 3), "unit": "GB/s", "h2d_bytes_per_step": int(h2d),
-                    "d2h_bytes_per_step": int(d2h), "ms_per_step": round(e2e_ms, 3)},
+                    "d2h_bytes_per_step": int(d2h), "ms_per_step": round(e2e_ms, 3),
+                    "api": "astitch_run_host_pipelined" if (world == 1 and args.e2e_chunks > 1) else
+                           ("astitch_run_host" if world == 1 else "torch H2D/D2H + astitch_run_sharded"),
+                    "chunks": args.e2e_chunks if world == 1 else 1},
             "gpu_launches": int(args.steps * sp.kernels_per_run()),
             "clocks": clocks,
             "cpu_baseline": cpu,

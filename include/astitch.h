@@ -141,8 +141,9 @@ enum {
   ASTITCH_FLAG_NO_TMA = 1u << 5,        /* do not use the TMA-staged packed template   */
   ASTITCH_FLAG_NO_PREFETCH = 1u << 6,   /* no software prefetch of the next row        */
   ASTITCH_FLAG_LAUNCH_CHECK = 1u << 7,  /* synchronise + check after every launch (debug)*/
-  ASTITCH_FLAG_FORCE_SPLIT = 1u << 8    /* ablation: split rows over clusters whenever the
+  ASTITCH_FLAG_FORCE_SPLIT = 1u << 8,   /* ablation: split rows over clusters whenever the
                                            paper's shape rule holds (no B200 size threshold) */
+  ASTITCH_FLAG_NO_PDL = 1u << 9         /* launch without programmatic dependent launch   */
 };
 
 typedef struct {
@@ -200,6 +201,19 @@ astitch_status astitch_run(astitch_plan_t p, const void* const* inputs, void* co
 astitch_status astitch_run_host(astitch_plan_t p, const void* const* host_inputs,
                                 void* const* host_outputs, const void* const* dev_inputs,
                                 void* const* dev_outputs, void* ws, void* stream);
+/* Same result as astitch_run_host, pipelined over `chunks` row chunks (rows are
+ * the independent units): chunk i+1 is copied in while chunk i is computed and
+ * chunk i-1 copied out, on three internal streams forked from and joined back
+ * into `stream` (PCIe is full duplex).  A column reduction accumulates its
+ * totals across chunks and its consumers run once after the last chunk.
+ * Host buffers must be pinned.  Falls back to astitch_run_host for plans that
+ * cannot be chunked (FULL values buffered across a grid barrier, cluster-split
+ * rows, sharded plans, chunks < 2).  The first call on a global plan compiles
+ * its chunk kernels.  Not safe to call concurrently on one plan. */
+astitch_status astitch_run_host_pipelined(astitch_plan_t p, const void* const* host_inputs,
+                                          void* const* host_outputs, const void* const* dev_inputs,
+                                          void* const* dev_outputs, void* ws, void* stream,
+                                          int32_t chunks);
 
 /* ---------------------------------------------------------------- multi-GPU
  * Row-sharded execution (BASELINE north_star (4)): each process owns a

@@ -35,6 +35,7 @@ FLAG_NO_TMA = 1 << 5
 FLAG_NO_PREFETCH = 1 << 6
 FLAG_LAUNCH_CHECK = 1 << 7
 FLAG_FORCE_SPLIT = 1 << 8
+FLAG_NO_PDL = 1 << 9
 
 
 class AstitchError(RuntimeError):
@@ -85,6 +86,8 @@ _sig = {
     "astitch_run": (ct.c_int, [_vp, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
     "astitch_run_host": (ct.c_int, [_vp, ct.POINTER(_vp), ct.POINTER(_vp), ct.POINTER(_vp),
                                     ct.POINTER(_vp), _vp, _vp]),
+    "astitch_run_host_pipelined": (ct.c_int, [_vp, ct.POINTER(_vp), ct.POINTER(_vp), ct.POINTER(_vp),
+                                              ct.POINTER(_vp), _vp, _vp, ct.c_int32]),
     "astitch_comm_unique_id": (ct.c_int, [ct.c_char_p]),
     "astitch_comm_create": (ct.c_int, [ct.c_int32, ct.c_int32, ct.c_char_p, ct.c_int32, ct.POINTER(_vp)]),
     "astitch_comm_destroy": (ct.c_int, [_vp]),

@@ -234,8 +234,10 @@ class Plan:
         check(lib.astitch_run(self._h, ins, outs, ct.c_void_p(ws.data_ptr() if ws is not None else 0),
                               ct.c_void_p(_stream_ptr(stream))), "astitch_run")
 
-    def run_host(self, host_inputs, host_outputs, dev_inputs, dev_outputs, ws=None, stream=None) -> None:
-        """astitch_run_host: H2D inputs, stitched kernel, D2H outputs (all async on `stream`)."""
+    def run_host(self, host_inputs, host_outputs, dev_inputs, dev_outputs, ws=None, stream=None,
+                 chunks: int = 1) -> None:
+        """astitch_run_host (chunks == 1) / astitch_run_host_pipelined (chunks > 1):
+        H2D inputs, stitched kernel(s), D2H outputs, asynchronous on `stream`."""
         if ws is None and self.workspace_bytes() > 0:
             if self._ws_cache is None:
                 self._ws_cache = self.alloc_workspace(stream)
@@ -244,8 +246,13 @@ class Plan:
         ho = ptr_array([t.data_ptr() for t in host_outputs])
         di = ptr_array([t.data_ptr() for t in dev_inputs])
         do = ptr_array([t.data_ptr() for t in dev_outputs])
-        check(lib.astitch_run_host(self._h, hi, ho, di, do, ct.c_void_p(ws.data_ptr() if ws is not None else 0),
-                                   ct.c_void_p(_stream_ptr(stream))), "astitch_run_host")
+        w = ct.c_void_p(ws.data_ptr() if ws is not None else 0)
+        s = ct.c_void_p(_stream_ptr(stream))
+        if chunks > 1:
+            check(lib.astitch_run_host_pipelined(self._h, hi, ho, di, do, w, s, int(chunks)),
+                  "astitch_run_host_pipelined")
+        else:
+            check(lib.astitch_run_host(self._h, hi, ho, di, do, w, s), "astitch_run_host")
 
 
 def plan(graph: Graph, rows: int, cols: int, device: int = 0, flags: int = 0, **kw) -> Plan:

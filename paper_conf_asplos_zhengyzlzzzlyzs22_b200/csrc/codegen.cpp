@@ -143,10 +143,15 @@ struct Gen {
       if (std::string(q) == ".cs" || std::string(q) == ".wt" || std::string(q) == ".cg")
         o << "#define AS_STQ \"" << q << "\"\n";
     o << "#include \"astitch_device.cuh\"\n";
-    o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; };\n";
+    o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; };\n";
     o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") ";
     if (split) o << "__cluster_dims__(" << m.split << ", 1, 1) ";
     o << name << "(const Params p) {\n";
+    // Programmatic dependent launch: wait for the preceding grid's memory
+    // (no-op when launched without the attribute), then let the next stitched
+    // kernel in the stream be scheduled while this one runs.
+    o << "  asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n";
+    o << "  asm volatile(\"griddepcontrol.launch_dependents;\");\n";
     o << "  constexpr int T = " << T << ", V = " << V << ", E = " << E << ", NE = " << NE << ", RPB = " << RPB
       << ";\n";
     o << "  constexpr long long C = " << C << "LL;\n";
@@ -854,7 +859,8 @@ struct Gen {
     if (!masked) return "C";
     // 32-bit valid bound; the segment index is an unsigned division by the
     // compile-time rows-per-segment (a shift when it is a power of two)
-    return "min(max(__ldg(Lp + (unsigned long long)(" + row + ") / (unsigned long long)RPS), 0), (int)C)";
+    // p.row_offset: global row of local row 0 (chunked host pipelines)
+    return "min(max(__ldg(Lp + (unsigned long long)((" + row + ") + p.row_offset) / (unsigned long long)RPS), 0), (int)C)";
   }
 
   // ------------------------------------------------------------ row sweep
@@ -1065,7 +1071,14 @@ struct Gen {
     }
     o << "      if (own && pi == 0) {\n";
     if (!final_chain) {
-      for (int q = 0; q < ncr; ++q) o << "        colpart[" << q << "LL * C + col] = t" << p.colreds[q] << ";\n";
+      // p.flags & 1: accumulate onto the totals of earlier row chunks
+      for (int q = 0; q < ncr; ++q) {
+        bool mx = N(p.colreds[q]).sub == ASTITCH_RMAX;
+        std::string slot = "colpart[" + std::to_string(q) + "LL * C + col]";
+        std::string t = "t" + std::to_string(p.colreds[q]);
+        o << "        " << slot << " = (p.flags & 1) ? "
+          << (mx ? "fmaxf(" + slot + ", " + t + ")" : "(" + slot + " + " + t + ")") << " : " << t << ";\n";
+      }
     } else {
       emit_colvec_chain("t");
     }
@@ -1296,7 +1309,7 @@ struct Gen {
       // small epilogue: one thread per column, consumers of the all-reduced
       // column totals (sharded global stage)
       o << "#include \"astitch_device.cuh\"\n";
-      o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; };\n";
+      o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; };\n";
       o << "extern \"C\" __global__ void __launch_bounds__(256) " << name << "(const Params p) {\n";
       o << "  constexpr long long C = " << C << "LL;\n";
       for (size_t i = 0; i < g.nodes.size(); ++i)

@@ -32,6 +32,12 @@ struct Driver {
   CUresult (*MemcpyAsync)(CUdeviceptr, CUdeviceptr, size_t, CUstream);
   CUresult (*StreamSynchronize)(CUstream);
   CUresult (*GetErrorString)(CUresult, const char**);
+  CUresult (*StreamCreate)(CUstream*, unsigned int);
+  CUresult (*StreamDestroy)(CUstream);
+  CUresult (*EventCreate)(CUevent*, unsigned int);
+  CUresult (*EventDestroy)(CUevent);
+  CUresult (*EventRecord)(CUevent, CUstream);
+  CUresult (*StreamWaitEvent)(CUstream, CUevent, unsigned int);
 };
 
 namespace {
@@ -87,6 +93,12 @@ Driver* driver(std::string& err) {
   SYM(MemcpyAsync, "cuMemcpyAsync");
   SYM(StreamSynchronize, "cuStreamSynchronize");
   SYM(GetErrorString, "cuGetErrorString");
+  SYM(StreamCreate, "cuStreamCreate");
+  SYM(StreamDestroy, "cuStreamDestroy_v2");
+  SYM(EventCreate, "cuEventCreate");
+  SYM(EventDestroy, "cuEventDestroy_v2");
+  SYM(EventRecord, "cuEventRecord");
+  SYM(StreamWaitEvent, "cuStreamWaitEvent");
 #undef SYM
   CUresult r = d.Init(0);
   if (r != CUDA_SUCCESS) {
@@ -199,6 +211,13 @@ bool drv_launch_args(const Kernel& k, void** args, void* stream, std::string& er
     attr[0].value.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+  } else if (k.pdl) {
+    // the kernel starts with griddepcontrol.wait, so it may be scheduled
+    // before its predecessor in the stream completes (hides launch latency)
+    attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+    attr[0].value.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
   }
   CUresult r = d->LaunchKernelEx(&cfg, static_cast<CUfunction>(k.function), args, nullptr);
   if (r != CUDA_SUCCESS) { err = cu_err(d, r, ("cuLaunchKernelEx(" + k.name + ")").c_str()); return false; }
@@ -221,6 +240,54 @@ bool drv_memcpy_async(void* dst, const void* src, size_t bytes, int kind, void* 
                               static_cast<CUstream>(stream));
   if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuMemcpyAsync"); return false; }
   return true;
+}
+
+bool drv_stream_create(void** s, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUstream st;
+  CUresult r = d->StreamCreate(&st, CU_STREAM_NON_BLOCKING);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuStreamCreate"); return false; }
+  *s = st;
+  return true;
+}
+
+bool drv_event_create(void** e, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUevent ev;
+  CUresult r = d->EventCreate(&ev, CU_EVENT_DISABLE_TIMING);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuEventCreate"); return false; }
+  *e = ev;
+  return true;
+}
+
+bool drv_event_record(void* e, void* s, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUresult r = d->EventRecord(static_cast<CUevent>(e), static_cast<CUstream>(s));
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuEventRecord"); return false; }
+  return true;
+}
+
+bool drv_stream_wait(void* s, void* e, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUresult r = d->StreamWaitEvent(static_cast<CUstream>(s), static_cast<CUevent>(e), 0);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuStreamWaitEvent"); return false; }
+  return true;
+}
+
+void drv_stream_destroy(void* s) {
+  std::string err;
+  Driver* d = driver(err);
+  if (d && s) d->StreamDestroy(static_cast<CUstream>(s));
+}
+
+void drv_event_destroy(void* e) {
+  std::string err;
+  Driver* d = driver(err);
+  if (d && e) d->EventDestroy(static_cast<CUevent>(e));
 }
 
 bool drv_sync(void* stream, std::string& err) {

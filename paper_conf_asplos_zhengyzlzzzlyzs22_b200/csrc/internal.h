@@ -119,6 +119,7 @@ struct Kernel {
   int64_t grid = 1;
   int smem = 0;
   bool cooperative = false;
+  bool pdl = false;          // programmatic dependent launch attribute
   int regs = -1;
   int spill_bytes = -1;
   int occupancy = -1;        // blocks per SM from the occupancy API
@@ -147,6 +148,12 @@ struct Plan {
   bool needs_sweep2 = false;
   std::vector<Kernel> kernels;   // kernels launched by astitch_run, in order
   std::vector<Kernel> shard_kernels; // kernels of the sharded path (after the allreduce)
+  // chunked host pipeline (astitch_run_host_pipelined): copy-in / compute /
+  // copy-out streams, per-chunk events, and for global plans the row-chunk
+  // kernels (shard-main with accumulation + column epilogue), built lazily
+  std::vector<Kernel> chunk_kernels;
+  void* pipe_streams[3] = {nullptr, nullptr, nullptr};
+  std::vector<void*> pipe_events;
   WsLayout ws;
   uint64_t compulsory_bytes = 0;
   int device = -1;
@@ -182,6 +189,12 @@ bool drv_memcpy_async(void* dst, const void* src, size_t bytes, int kind, void* 
                       std::string& err);
 bool drv_device_info(int device, int& sm_count, int& max_smem_optin, std::string& err);
 bool drv_sync(void* stream, std::string& err);
+bool drv_stream_create(void** s, std::string& err);
+bool drv_event_create(void** e, std::string& err);
+bool drv_event_record(void* e, void* s, std::string& err);
+bool drv_stream_wait(void* s, void* e, std::string& err);
+void drv_stream_destroy(void* s);
+void drv_event_destroy(void* e);
 
 // kernel parameter block (mirrors the struct emitted by codegen)
 constexpr int kMaxIO = 16;
@@ -190,7 +203,8 @@ struct KernelParams {
   void* out[kMaxIO];
   void* ws;
   long long rows;
-  long long row_offset;   // global row index of row 0 (sharded plans; mask segments)
+  long long row_offset;   // global row index of row 0 (chunked runs; mask segments)
+  int flags;              // bit 0: accumulate column totals onto earlier chunks
 };
 
 }  // namespace astitch

@@ -97,6 +97,7 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     k.grid = (role == ROLE_SHARD_FINAL) ? std::max<int64_t>(1, (p.desc.cols + 255) / 256) : p.map.grid;
     k.smem = (role == ROLE_SHARD_FINAL) ? 0 : p.map.smem_bytes;
     k.cooperative = (p.map.tmpl == Template::GlobalSweep) && (role == ROLE_MAIN || role == ROLE_SHARD_MAIN);
+    k.pdl = !k.cooperative && role != ROLE_SHARD_FINAL && (p.desc.flags & ASTITCH_FLAG_NO_PDL) == 0;
     if (!compile) return ASTITCH_OK;
     astitch_status st = compile_and_inspect(p, k, load);
     if (st != ASTITCH_OK) return st;
@@ -205,6 +206,9 @@ astitch_status astitch_plan_destroy(astitch_plan_t h) {
   if (!h) return ASTITCH_OK;
   for (auto& k : h->p->kernels) drv_unload(k);
   for (auto& k : h->p->shard_kernels) drv_unload(k);
+  for (auto& k : h->p->chunk_kernels) drv_unload(k);
+  for (void* s : h->p->pipe_streams) drv_stream_destroy(s);
+  for (void* e : h->p->pipe_events) drv_event_destroy(e);
   delete h;
   return ASTITCH_OK;
 }
@@ -381,6 +385,115 @@ astitch_status astitch_run_host(astitch_plan_t h, const void* const* host_inputs
       return fail(ASTITCH_ERR_CUDA, err);
   }
   return ASTITCH_OK;
+}
+
+astitch_status astitch_run_host_pipelined(astitch_plan_t h, const void* const* host_inputs,
+                                          void* const* host_outputs, const void* const* dev_inputs,
+                                          void* const* dev_outputs, void* ws, void* stream, int32_t chunks) {
+  if (!h || !host_inputs || !host_outputs || !dev_inputs || !dev_outputs)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  Plan& p = *h->p;
+  const int64_t R = p.desc.rows;
+  const bool global = p.map.tmpl == Template::GlobalSweep;
+  // rows are the independent units: chunk them; a column reduction accumulates
+  // its totals across chunks and its consumers run once at the end
+  if (chunks <= 1 || R < static_cast<int64_t>(chunks) * 64 || (global && p.needs_sweep2) ||
+      p.desc.shard_world > 1 || p.map.tmpl == Template::SplitRow || p.device < 0)
+    return astitch_run_host(h, host_inputs, host_outputs, dev_inputs, dev_outputs, ws, stream);
+  if (chunks > 64) chunks = 64;
+  astitch_status s = check_io(p, dev_inputs, dev_outputs, ws);
+  if (s != ASTITCH_OK) return s;
+  std::string err;
+  if (global && p.chunk_kernels.empty()) {
+    p.chunk_kernels.resize(2);
+    if ((s = build_kernel(p, ROLE_SHARD_MAIN, p.chunk_kernels[0])) != ASTITCH_OK) return s;
+    if ((s = build_kernel(p, ROLE_SHARD_FINAL, p.chunk_kernels[1])) != ASTITCH_OK) return s;
+    for (Kernel& k : p.chunk_kernels) {
+      if (!k.module && !drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
+      if (k.cooperative) k.grid = std::min<int64_t>(k.grid, static_cast<int64_t>(k.occupancy) * p.sm_count);
+    }
+  }
+  for (int i = 0; i < 3; ++i)
+    if (!p.pipe_streams[i] && !drv_stream_create(&p.pipe_streams[i], err)) return fail(ASTITCH_ERR_CUDA, err);
+  while (p.pipe_events.size() < static_cast<size_t>(2 * chunks + 3)) {
+    void* e = nullptr;
+    if (!drv_event_create(&e, err)) return fail(ASTITCH_ERR_CUDA, err);
+    p.pipe_events.push_back(e);
+  }
+  void* s_in = p.pipe_streams[0];
+  void* s_comp = p.pipe_streams[1];
+  void* s_out = p.pipe_streams[2];
+  auto& ev = p.pipe_events;
+  auto ck = [&](bool ok) { return ok ? ASTITCH_OK : fail(ASTITCH_ERR_CUDA, err); };
+  // fork from the caller's stream
+  if ((s = ck(drv_event_record(ev[0], stream, err))) != ASTITCH_OK) return s;
+  for (void* st : {s_in, s_comp, s_out})
+    if ((s = ck(drv_stream_wait(st, ev[0], err))) != ASTITCH_OK) return s;
+  const size_t C = static_cast<size_t>(p.desc.cols);
+  auto row_scaled = [&](astitch_kind k, int64_t rows, astitch_dtype dt) -> size_t {
+    if (k == ASTITCH_FULL) return static_cast<size_t>(rows) * C * dtype_size(dt);
+    if (k == ASTITCH_ROWVEC) return static_cast<size_t>(rows) * dtype_size(dt);
+    return 0;
+  };
+  for (int c = 0; c < chunks; ++c) {
+    const int64_t b = (R * c) / chunks, n = (R * (c + 1)) / chunks - b;
+    // copy-in of the chunk's rows (vectors and lengths once, with chunk 0)
+    for (size_t i = 0; i < p.g.inputs.size(); ++i) {
+      const Node& nd = p.g.nodes[p.g.inputs[i]];
+      size_t off = row_scaled(nd.kind, b, nd.dtype), nb = row_scaled(nd.kind, n, nd.dtype);
+      if (nd.kind != ASTITCH_FULL && nd.kind != ASTITCH_ROWVEC) {
+        if (c != 0) continue;
+        off = 0;
+        nb = io_bytes(p, p.g.inputs[i], nd.dtype);
+      }
+      if (!host_inputs[i]) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "host input NULL");
+      if (!drv_memcpy_async(static_cast<char*>(const_cast<void*>(dev_inputs[i])) + off,
+                            static_cast<const char*>(host_inputs[i]) + off, nb, 1, s_in, err))
+        return fail(ASTITCH_ERR_CUDA, err);
+    }
+    if ((s = ck(drv_event_record(ev[1 + 2 * c], s_in, err))) != ASTITCH_OK) return s;
+    if ((s = ck(drv_stream_wait(s_comp, ev[1 + 2 * c], err))) != ASTITCH_OK) return s;
+    // the stitched kernel on the chunk's rows
+    KernelParams kp = make_params(p, dev_inputs, dev_outputs, ws);
+    for (size_t i = 0; i < p.g.inputs.size(); ++i) {
+      const Node& nd = p.g.nodes[p.g.inputs[i]];
+      kp.in[i] = static_cast<const char*>(dev_inputs[i]) + row_scaled(nd.kind, b, nd.dtype);
+    }
+    for (size_t i = 0; i < p.g.outputs.size(); ++i)
+      kp.out[i] = static_cast<char*>(dev_outputs[i]) +
+                  row_scaled(p.g.nodes[p.g.outputs[i]].kind, b, p.g.output_dtypes[i]);
+    kp.rows = n;
+    kp.row_offset = b;
+    kp.flags = (global && c > 0) ? 1 : 0;
+    if ((s = launch(p, global ? p.chunk_kernels[0] : p.kernels[0], kp, s_comp)) != ASTITCH_OK) return s;
+    if ((s = ck(drv_event_record(ev[2 + 2 * c], s_comp, err))) != ASTITCH_OK) return s;
+    if ((s = ck(drv_stream_wait(s_out, ev[2 + 2 * c], err))) != ASTITCH_OK) return s;
+    // copy-out of the chunk's row outputs
+    for (size_t i = 0; i < p.g.outputs.size(); ++i) {
+      const astitch_kind k = p.g.nodes[p.g.outputs[i]].kind;
+      if (k != ASTITCH_FULL && k != ASTITCH_ROWVEC) continue;
+      size_t off = row_scaled(k, b, p.g.output_dtypes[i]), nb = row_scaled(k, n, p.g.output_dtypes[i]);
+      if (!host_outputs[i]) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "host output NULL");
+      if (!drv_memcpy_async(static_cast<char*>(host_outputs[i]) + off, static_cast<char*>(dev_outputs[i]) + off, nb,
+                            2, s_out, err))
+        return fail(ASTITCH_ERR_CUDA, err);
+    }
+  }
+  if (global) {  // column consumers once every chunk has accumulated
+    KernelParams kp = make_params(p, dev_inputs, dev_outputs, ws);
+    if ((s = launch(p, p.chunk_kernels[1], kp, s_comp)) != ASTITCH_OK) return s;
+    if ((s = ck(drv_event_record(ev[2 * chunks + 1], s_comp, err))) != ASTITCH_OK) return s;
+    if ((s = ck(drv_stream_wait(s_out, ev[2 * chunks + 1], err))) != ASTITCH_OK) return s;
+    for (size_t i = 0; i < p.g.outputs.size(); ++i) {
+      if (p.g.nodes[p.g.outputs[i]].kind != ASTITCH_COLVEC) continue;
+      if (!drv_memcpy_async(host_outputs[i], dev_outputs[i], io_bytes(p, p.g.outputs[i], p.g.output_dtypes[i]), 2,
+                            s_out, err))
+        return fail(ASTITCH_ERR_CUDA, err);
+    }
+  }
+  // join back into the caller's stream
+  if ((s = ck(drv_event_record(ev[2 * chunks + 2], s_out, err))) != ASTITCH_OK) return s;
+  return ck(drv_stream_wait(stream, ev[2 * chunks + 2], err));
 }
 
 }  // extern "C"
