@@ -32,8 +32,11 @@ NaN (numpy semantics); R14 a fully-masked reduction yields its identity.
 Evaluation order: the rows are processed in chunks (memory only).  Column
 reductions accumulate fp64 chunk partials in chunk order; ops that consume a
 column reduction (directly or through ``broadcast COL``) are evaluated in a
-second pass once every chunk has been reduced.  This is the definition,
-split over rows; it has no blocking across columns and no fusion.
+later pass over the rows once every chunk has been reduced — one pass per
+level of dependent column reductions (e.g. BatchNorm: mean, then variance of
+the centred values), recomputing the lower-level values in each pass.  This
+is the definition, split over rows; it has no blocking across columns and no
+fusion.
 """
 
 from __future__ import annotations
@@ -153,22 +156,30 @@ def _kinds(spec):
     return kind
 
 
-def _after_colreduce(spec):
-    """Values that depend (transitively) on a column reduction."""
-    post = set()
+def _operands(op):
+    typ = op[1]
+    if typ == "unary":
+        return [op[3]]
+    if typ == "binary":
+        return [op[3], op[4]]
+    if typ == "reduce":
+        return [op[4]]
+    if typ == "broadcast":
+        return [op[3]]
+    return []
+
+
+def _levels(spec):
+    """Number of column reductions on each value's dependency path: a column
+    reduction is complete only after every row has been visited, so its
+    consumers belong to the next pass over the rows."""
+    level = {n: 0 for n, _, _ in spec["inputs"]}
     for op in spec["ops"]:
-        name, typ = op[0], op[1]
-        if typ == "reduce" and op[3] == "COL":
-            post.add(name)
-        elif typ in ("unary", "broadcast") and op[-1] in post:
-            post.add(name)
-        elif typ == "binary" and (op[3] in post or op[4] in post):
-            post.add(name)
-        elif typ == "reduce" and op[4] in post:
-            if op[3] == "COL":
-                raise NotImplementedError("a column reduction downstream of another one")
-            post.add(name)
-    return post
+        lv = max([level[a] for a in _operands(op)] or [0])
+        if op[1] == "reduce" and op[3] == "COL":
+            lv += 1
+        level[op[0]] = lv
+    return level
 
 
 # ----------------------------------------------------------------------------
@@ -184,7 +195,7 @@ def evaluate(spec: dict, inputs: dict, row_chunk: int = 16384) -> dict:
     """
     R, C = int(spec["rows"]), int(spec["cols"])
     kind = _kinds(spec)
-    post = _after_colreduce(spec)
+    level = _levels(spec)
     out_names = [n for n, _ in spec["outputs"]]
     mask = spec.get("mask")
 
@@ -208,19 +219,18 @@ def evaluate(spec: dict, inputs: dict, row_chunk: int = 16384) -> dict:
         seg = np.arange(r0, r1) // rps
         return np.arange(C)[None, :] < lengths[seg][:, None]
 
-    def eval_ops(env, valid, second_pass):
-        """Evaluate the ops in order on one row chunk.  First pass: only the
-        ops that do not depend on a column reduction.  Second pass: the rest."""
+    def eval_ops(env, valid, lvl):
+        """Evaluate, in spec order on one row chunk, every op of level <= lvl.
+        Column reductions of level-lvl operands produce chunk partials (combined
+        by the caller); completed column reductions come from `glob`."""
         for op in spec["ops"]:
             name, typ = op[0], op[1]
-            if typ == "const":
-                continue
-            if name in env and not (second_pass and name in post):
+            if typ == "const" or name in env:
                 continue
             is_colred = typ == "reduce" and op[3] == "COL"
-            if not second_pass and name in post and not is_colred:
-                continue
-            if second_pass and is_colred:
+            if is_colred and level[op[4]] != lvl:
+                continue  # complete (in glob) or not yet reachable
+            if not is_colred and level[name] > lvl:
                 continue
             if kind[name] == "COLVEC" and name in glob:
                 env[name] = glob[name]
@@ -293,59 +303,43 @@ def evaluate(spec: dict, inputs: dict, row_chunk: int = 16384) -> dict:
             elif k == "COLVEC":
                 outs[n][:] = env[n]
 
+    D = max(level.values()) if level else 0
     with np.errstate(all="ignore"):
-        # pass 1: everything not downstream of a column reduction
-        for r0 in range(0, R, row_chunk):
-            r1 = min(R, r0 + row_chunk)
-            valid = valid_for(r0, r1)
-            env = chunk_env(r0, r1)
-            eval_ops(env, valid, second_pass=False)
-            for op in colred:
-                p = env.get("__colpart__" + op[0])
-                if p is None:
-                    continue
-                if op[2] == "SUM":
-                    colacc[op[0]] = colacc[op[0]] + p
-                else:
-                    colacc[op[0]] = np.maximum(colacc[op[0]], p)
-            store(env, r0, r1, valid, [n for n in out_names if n not in post])
-
-        if colred:
-            # the column reductions are complete: evaluate their COLVEC consumers
-            for k_, v in colacc.items():
-                glob[k_] = v
-            cenv = dict(glob)
-            cenv["__nrows__"] = 0
-            for op in spec["ops"]:
-                name, typ = op[0], op[1]
-                if name not in post or kind[name] != "COLVEC" or name in glob:
-                    continue
-                if typ == "unary":
-                    glob[name] = UNARY[op[2]](cenv[op[3]])
-                elif typ == "binary":
-                    glob[name] = BINARY[op[2]](cenv[op[3]], cenv[op[4]])
-                cenv[name] = glob[name]
-            for n in out_names:
-                if kind[n] == "COLVEC":
-                    outs[n][:] = glob[n]
-                elif kind[n] == "SCALAR":
-                    outs[n] = np.float64(glob[n])
-
-            # pass 2: FULL / ROWVEC values downstream of a column reduction
-            need2 = [n for n in out_names if n in post and kind[n] in ("FULL", "ROWVEC")]
-            if need2:
+        # one pass over the rows per level of dependent column reductions
+        for lvl in range(D + 1):
+            red_here = [op for op in colred if level[op[4]] == lvl]
+            rows_out = [n for n in out_names if level[n] == lvl and kind[n] in ("FULL", "ROWVEC")]
+            if lvl == 0 or red_here or rows_out:
                 for r0 in range(0, R, row_chunk):
                     r1 = min(R, r0 + row_chunk)
                     valid = valid_for(r0, r1)
                     env = chunk_env(r0, r1)
-                    eval_ops(env, valid, second_pass=False)
-                    env.update({k_: glob[k_] for k_ in glob})
-                    eval_ops(env, valid, second_pass=True)
-                    store(env, r0, r1, valid, need2)
-        else:
-            for n in out_names:
-                if kind[n] == "COLVEC" and n in glob:
-                    outs[n][:] = glob[n]
+                    eval_ops(env, valid, lvl)
+                    for op in red_here:
+                        p = env["__colpart__" + op[0]]
+                        if op[2] == "SUM":
+                            colacc[op[0]] = colacc[op[0]] + p
+                        else:
+                            colacc[op[0]] = np.maximum(colacc[op[0]], p)
+                    store(env, r0, r1, valid, [n for n in out_names if level[n] == lvl])
+            # these column reductions are complete: their COLVEC consumers
+            for op in red_here:
+                glob[op[0]] = colacc[op[0]]
+            for op in spec["ops"]:
+                name, typ = op[0], op[1]
+                if kind[name] != "COLVEC" or name in glob or level[name] > lvl + 1:
+                    continue
+                if typ == "reduce":
+                    continue  # a later level's column reduction
+                if typ == "unary":
+                    glob[name] = UNARY[op[2]](glob[op[3]])
+                elif typ == "binary":
+                    glob[name] = BINARY[op[2]](glob[op[3]], glob[op[4]])
+        for n in out_names:
+            if kind[n] == "COLVEC" and n in glob:
+                outs[n][:] = glob[n]
+            elif kind[n] == "SCALAR":
+                outs[n] = np.float64(glob[n])
     return outs
 
 

@@ -286,6 +286,42 @@ def test_fig7a_bruteforce():
             assert out[r, c] == pytest.approx(A[r][c] * A[r][c] * R2[c], rel=1e-13, abs=1e-13)
 
 
+# ---------------------------------------------------------------- dependent column reductions
+
+def test_batchnorm_two_levels_invariants():
+    """Training BatchNorm: mean, then variance of the centred values (two
+    dependent column reductions).  Per channel the normalised output has mean 0
+    and variance v/(v+eps) (closed form); mean/var match numpy's routines."""
+    spec = specs.get("bn", rows=3000, cols=24)
+    x = gen.generate("bn", spec)
+    x["gamma"] = np.ones(24, np.float32)
+    x["beta"] = np.zeros(24, np.float32)
+    for chunk in (7, 512, 100000):
+        out = evaluate(spec, x, row_chunk=chunk)
+        X = x["x"].astype(np.float64)
+        np.testing.assert_allclose(out["mean"], X.mean(axis=0), rtol=1e-13, atol=1e-15)
+        v = X.var(axis=0)
+        np.testing.assert_allclose(out["var"], v, rtol=1e-12)
+        np.testing.assert_allclose(out["y"].mean(axis=0), 0.0, atol=1e-13)
+        np.testing.assert_allclose(out["y"].var(axis=0), v / (v + 1e-5), rtol=1e-11)
+
+
+def test_batchnorm_bruteforce_tiny():
+    spec = specs.get("bn", rows=5, cols=2)
+    x = gen.generate("bn", spec)
+    out = evaluate(spec, x, row_chunk=2)
+    X = x["x"].astype(np.float64)
+    g, b = x["gamma"].astype(np.float64), x["beta"].astype(np.float64)
+    for c in range(2):
+        m = sum(X[r, c] for r in range(5)) / 5
+        var = sum((X[r, c] - m) ** 2 for r in range(5)) / 5
+        assert out["mean"][c] == pytest.approx(m, rel=1e-14)
+        assert out["var"][c] == pytest.approx(var, rel=1e-13)
+        for r in range(5):
+            assert out["y"][r, c] == pytest.approx((X[r, c] - m) / math.sqrt(var + 1e-5) * g[c] + b[c],
+                                                   rel=1e-12, abs=1e-13)
+
+
 # ---------------------------------------------------------------- plumbing
 
 def test_bf16_widening_golden():

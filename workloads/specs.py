@@ -259,6 +259,38 @@ FIG6B_FEW_LONG_ROWS = {
     "outputs": [("s", "F32")],
 }
 
+# Training BatchNorm forward (the BN of CRNN-style convnets, Table 2):
+# two DEPENDENT column reductions (mean, then variance of the centred values),
+# i.e. two grid barriers in one stitched kernel.  rows = N*H*W, cols = channels.
+# The const named "nrows" follows the row count (see resized()).
+BN_TRAIN_FWD = {
+    "name": "batchnorm_train_forward_f32",
+    "rows": 32 * 28 * 28,
+    "cols": 128,
+    "inputs": [("x", "FULL", "F32"), ("gamma", "COLVEC", "F32"), ("beta", "COLVEC", "F32")],
+    "mask": None,
+    "ops": [
+        ("s1", "reduce", "SUM", "COL", "x"),
+        ("nrows", "const", float(32 * 28 * 28)),
+        ("mean", "binary", "DIV", "s1", "nrows"),
+        ("meanb", "broadcast", "COL", "mean"),
+        ("xc", "binary", "SUB", "x", "meanb"),
+        ("xc2", "binary", "MUL", "xc", "xc"),
+        ("s2", "reduce", "SUM", "COL", "xc2"),
+        ("var", "binary", "DIV", "s2", "nrows"),
+        ("eps", "const", 1e-5),
+        ("ve", "binary", "ADD", "var", "eps"),
+        ("rstd", "unary", "RSQRT", "ve"),
+        ("rstdb", "broadcast", "COL", "rstd"),
+        ("xhat", "binary", "MUL", "xc", "rstdb"),
+        ("gb", "broadcast", "COL", "gamma"),
+        ("yg", "binary", "MUL", "xhat", "gb"),
+        ("bb", "broadcast", "COL", "beta"),
+        ("y", "binary", "ADD", "yg", "bb"),
+    ],
+    "outputs": [("y", "F32"), ("mean", "F32"), ("var", "F32")],
+}
+
 # Remote stitching: two subgraphs with no data dependency merged into
 # one stitch op (the "independent" scheme between them), one kernel.
 REMOTE_TWO_SUBGRAPHS = {
@@ -297,6 +329,7 @@ EXTRA = {
     "fig6a": FIG6A_MANY_SHORT_ROWS,
     "fig6b": FIG6B_FEW_LONG_ROWS,
     "remote": REMOTE_TWO_SUBGRAPHS,
+    "bn": BN_TRAIN_FWD,
 }
 
 ALL = {**CONFIGS, **EXTRA}
@@ -309,10 +342,13 @@ def get(name: str, rows: int | None = None, cols: int | None = None) -> dict:
 
 def resized(spec: dict, rows: int | None = None, cols: int | None = None) -> dict:
     """Copy of ``spec`` at another shape.  A const op named ``ncols`` (the mean
-    divisor of the LayerNorm-style specs) follows the new column count."""
+    divisor of the LayerNorm-style specs) follows the new column count, one
+    named ``nrows`` (BatchNorm) the new row count."""
     s = copy.deepcopy(spec)
     if rows is not None:
         s["rows"] = int(rows)
+        s["ops"] = [(o[0], "const", float(rows)) if (o[1] == "const" and o[0] == "nrows") else o
+                    for o in s["ops"]]
     if cols is not None:
         s["cols"] = int(cols)
         s["ops"] = [(o[0], "const", float(cols)) if (o[1] == "const" and o[0] == "ncols") else o
