@@ -221,10 +221,20 @@ struct Gen {
     }
   }
 
-  // post-barrier COLVEC values needed by sweep 2 (finalised values from ws)
+  // ---- barrier levels ----------------------------------------------------
+  // Sweep `cur_level` computes every FULL/ROWVEC op whose level equals it; a
+  // column reduction accumulates in the sweep of its operand's level.
+  int cur_level = 0;
+  int phase_of(int u) const {
+    if (I(u).cls == OpClass::ReduceCol) return I(N(u).a).level;
+    return I(u).level;
+  }
+
+  // COLVEC values finalised after earlier barriers (loaded from ws)
   void emit_post_colvec_loads() {
     for (size_t q = 0; q < p.post_colvecs.size(); ++q) {
       int i = p.post_colvecs[q];
+      if (I(i).level > cur_level) continue;  // not computed yet
       o << "  float cp" << i << "[NE];\n";
       o << "  { const float* cv = (const float*)((char*)p.ws + " << p.ws.colvals << "LL) + " << q << "LL * C;\n";
       o << "#pragma unroll\n  for (int j = 0; j < V; ++j)\n#pragma unroll\n  for (int e = 0; e < E; ++e) {\n";
@@ -244,35 +254,24 @@ struct Gen {
   };
   std::vector<Stream> streams;
 
-  bool node_used_in_phase(int i, bool post) const {
-    for (int u : I(i).consumers) {
-      if (!I(u).live) continue;
-      // a column reduction accumulates its operand before the barrier
-      bool u_post = I(u).post && I(u).cls != OpClass::ReduceCol;
-      if (u_post == post) return true;
-    }
+  // does any consumer of node i run in the current sweep?
+  bool node_used_in_phase(int i, bool /*post*/) const {
+    for (int u : I(i).consumers)
+      if (I(u).live && phase_of(u) == cur_level) return true;
     return false;
   }
 
-  void collect_streams(bool post) {
+  void collect_streams(bool /*post*/) {
     streams.clear();
-    if (!post) {
-      for (int id : g.inputs) {
-        const Node& nd = N(id);
-        if (nd.kind == ASTITCH_FULL && I(id).live && node_used_in_phase(id, false))
-          streams.push_back({id, false, nd.dtype, 0});
-      }
-    } else {
-      for (int id : g.inputs) {
-        const Node& nd = N(id);
-        if (nd.kind == ASTITCH_FULL && I(id).live && node_used_in_phase(id, true))
-          streams.push_back({id, false, nd.dtype, 0});
-      }
-      for (size_t q = 0; q < p.global_fulls.size(); ++q) {
-        int id = p.global_fulls[q];
-        if (N(id).kind == ASTITCH_FULL)
-          streams.push_back({id, true, ASTITCH_F32, static_cast<long long>(p.ws.globals + gbuf_offset(q))});
-      }
+    for (int id : g.inputs) {
+      const Node& nd = N(id);
+      if (nd.kind == ASTITCH_FULL && I(id).live && node_used_in_phase(id, false))
+        streams.push_back({id, false, nd.dtype, 0});  // re-read from HBM in later sweeps
+    }
+    for (size_t q = 0; q < p.global_fulls.size(); ++q) {
+      int id = p.global_fulls[q];
+      if (N(id).kind == ASTITCH_FULL && I(id).level < cur_level && node_used_in_phase(id, false))
+        streams.push_back({id, true, ASTITCH_F32, static_cast<long long>(p.ws.globals + gbuf_offset(q))});
     }
   }
   size_t gbuf_offset(size_t q) const {
@@ -452,15 +451,12 @@ struct Gen {
       const NodeInfo& in = I(i);
       if (!in.live || nd.type == NodeType::Input || nd.type == NodeType::Const) continue;
       if (nd.type == NodeType::Bcast) continue;  // folded into operand references
-      // a column reduction accumulates in the pre-barrier sweep
-      const bool node_post = in.post && in.cls != OpClass::ReduceCol;
-      if (node_post != post) {
-        // pre-phase values re-materialised in sweep 2 come from global buffers;
-        // column reductions are handled by the accumulators below
-        continue;
-      }
-      if (post && nd.kind == ASTITCH_COLVEC) continue;  // finalised after the barrier
-      if (!post && nd.kind == ASTITCH_COLVEC && nd.type != NodeType::Reduce) continue;  // hoisted
+      (void)post;
+      // only the ops of this sweep's level; a column reduction accumulates in
+      // the sweep of its operand (earlier levels come from HBM buffers)
+      if (phase_of(i) != cur_level) continue;
+      // COLVEC values: level 0 hoisted per lane, later ones finalised per column
+      if (nd.kind == ASTITCH_COLVEC && !(nd.type == NodeType::Reduce && nd.axis == ASTITCH_AXIS_COL)) continue;
       std::string id = std::to_string(i);
       if (nd.type == NodeType::Reduce && nd.axis == ASTITCH_AXIS_COL) {
         bool mx = nd.sub == ASTITCH_RMAX;
@@ -792,10 +788,10 @@ struct Gen {
       o << "    const float s" << id << sfx << " = (" << act << ") ? as::ld_scalar<" << dt_code(nd.dtype)
         << ">(p.in[" << nd.input_index << "], " << row << ") : 0.f;\n";
     }
-    if (post) {  // pre ROWVEC values consumed after the barrier: global row buffers
+    if (cur_level > 0) {  // earlier-level ROWVEC values: global row buffers
       for (size_t q = 0; q < p.global_fulls.size(); ++q) {
         int id = p.global_fulls[q];
-        if (N(id).kind != ASTITCH_ROWVEC) continue;
+        if (N(id).kind != ASTITCH_ROWVEC || I(id).level >= cur_level || !node_used_in_phase(id, true)) continue;
         o << "    const float s" << id << sfx << " = (" << act << ") ? as::ld_cg((const float*)((const char*)p.ws + "
           << (p.ws.globals + gbuf_offset(q)) << "LL) + " << row << ") : 0.f;\n";
       }
@@ -809,7 +805,7 @@ struct Gen {
     for (size_t k = 0; k < g.outputs.size(); ++k) {
       int id = g.outputs[k];
       const Node& nd = N(id);
-      if (I(id).post != post) continue;
+      if (I(id).level != cur_level) continue;
       astitch_dtype dt = g.output_dtypes[k];
       if (nd.kind == ASTITCH_FULL) {
         std::string rt = "as::Raw<" + std::to_string(nb(dt)) + ">";
@@ -834,9 +830,11 @@ struct Gen {
       }
     }
     (void)check;
-    if (!post) {
+    (void)post;
+    {  // values of this level read by later sweeps: buffered in HBM (global scheme)
       for (size_t q = 0; q < p.global_fulls.size(); ++q) {
         int id = p.global_fulls[q];
+        if (I(id).level != cur_level) continue;
         long long off = static_cast<long long>(p.ws.globals + gbuf_offset(q));
         if (N(id).kind == ASTITCH_FULL) {
           std::string rt = "as::Raw<" + std::to_string(E * 4) + ">";
@@ -1002,6 +1000,7 @@ struct Gen {
   // ------------------------------------------------------------ global pieces
   void emit_colred_acc_decl() {
     for (int id : p.colreds) {
+      if (phase_of(id) != cur_level) continue;
       bool mx = N(id).sub == ASTITCH_RMAX;
       o << "  float acc" << id << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) acc" << id
         << "[k] = " << (mx ? "-AS_INF" : "0.f") << ";\n";
@@ -1015,6 +1014,7 @@ struct Gen {
     if (RPB == 1) {
       for (int q = 0; q < ncr; ++q) {
         int id = p.colreds[q];
+        if (phase_of(id) != cur_level) continue;
         o << "#pragma unroll\n    for (int k = 0; k < NE; ++k) {\n      const long long col = "
           << col_expr("(k / E)", "(k % E)") << ";\n";
         o << "      if (col < C) part[((long long)blockIdx.x * " << ncr << " + " << q << ") * C + col] = acc" << id
@@ -1025,6 +1025,7 @@ struct Gen {
       o << "    const long long CC = (long long)T * V * E;\n";
       for (int q = 0; q < ncr; ++q) {
         int id = p.colreds[q];
+        if (phase_of(id) != cur_level) continue;
         bool mx = N(id).sub == ASTITCH_RMAX;
         o << "    __syncthreads();\n";
         o << "#pragma unroll\n    for (int k = 0; k < NE; ++k) cp_smem[team * CC + " << col_expr("(k / E)", "(k % E)")
@@ -1058,6 +1059,7 @@ struct Gen {
     o << "      const bool own = (wi < (int)(blockDim.x / P)) && col < c1;\n";
     for (int q = 0; q < ncr; ++q) {
       int id = p.colreds[q];
+      if (phase_of(id) != cur_level) continue;
       bool mx = N(id).sub == ASTITCH_RMAX;
       std::string ident = mx ? "-AS_INF" : "0.f";
       o << "      float t" << id << " = " << ident << ";\n";
@@ -1085,14 +1087,26 @@ struct Gen {
     o << "      }\n    }\n  }\n";
   }
 
-  // COLVEC chain for one column `col` given totals t<id> of the column reductions
+  // COLVEC chain for one column `col` given totals t<id> of the column
+  // reductions finalised at this barrier (level cur_level + 1); values of
+  // earlier barriers are read back from the workspace, level-0 ones recomputed
+  int post_index(int id) const {
+    for (size_t q = 0; q < p.post_colvecs.size(); ++q)
+      if (p.post_colvecs[q] == id) return static_cast<int>(q);
+    return -1;
+  }
   void emit_colvec_chain(const std::string& tpref) {
+    const int lv = cur_level + 1;
     for (size_t ii = 0; ii < g.nodes.size(); ++ii) {
       int i = static_cast<int>(ii);
       const Node& nd = N(i);
       if (!I(i).live || nd.kind != ASTITCH_COLVEC) continue;
+      if (I(i).level > lv) continue;
       std::string id = std::to_string(i);
-      if (nd.type == NodeType::Reduce) {
+      if (I(i).level >= 1 && I(i).level < lv) {
+        o << "        const float x" << id << " = as::ld_cg((const float*)((const char*)p.ws + " << p.ws.colvals
+          << "LL) + " << post_index(i) << "LL * C + col);\n";
+      } else if (nd.type == NodeType::Reduce) {
         o << "        const float x" << id << " = " << tpref << id << ";\n";
       } else if (nd.type == NodeType::Input) {
         o << "        const float x" << id << " = as::ld_scalar<" << dt_code(nd.dtype) << ">(p.in[" << nd.input_index
@@ -1105,11 +1119,12 @@ struct Gen {
     }
     for (size_t k = 0; k < g.outputs.size(); ++k) {
       int id = g.outputs[k];
-      if (N(id).kind != ASTITCH_COLVEC) continue;
+      if (N(id).kind != ASTITCH_COLVEC || I(id).level != lv) continue;
       o << "        as::st_scalar<" << dt_code(g.output_dtypes[k]) << ">(p.out[" << k << "], col, x" << id << ");\n";
     }
     for (size_t q = 0; q < p.post_colvecs.size(); ++q) {
       int id = p.post_colvecs[q];
+      if (I(id).level != lv) continue;
       o << "        ((float*)((char*)p.ws + " << p.ws.colvals << "LL))[" << q << "LL * C + col] = x" << id << ";\n";
     }
   }
@@ -1328,7 +1343,8 @@ struct Gen {
     if (m.tmpl == Template::GlobalSweep) {
       o << "  unsigned int* bar = (unsigned int*)((char*)p.ws + " << p.ws.barrier << "LL);\n  (void)bar;\n";
     }
-    if (role == ROLE_SHARD_SWEEP2) {
+    if (role == ROLE_SHARD_SWEEP2) {  // sharded plans have one barrier level
+      cur_level = 1;
       emit_colvecs(false);
       emit_post_colvec_loads();
       emit_sweep(true);
@@ -1337,23 +1353,43 @@ struct Gen {
     }
     emit_colvecs(false);
     emit_pre_colvec_outputs();
-    if (m.tmpl == Template::GlobalSweep) emit_colred_acc_decl();
-    emit_sweep(false);
-    if (m.tmpl == Template::GlobalSweep) {
-      emit_block_partials();
-      o << "  as::grid_barrier(bar);\n";
-      if (role == ROLE_SHARD_MAIN) {
-        emit_column_finalize(false);
-      } else {
-        emit_column_finalize(true);
-        if (p.needs_sweep2) {
-          o << "  as::grid_barrier(bar);\n";
-          o << "  {\n";
-          emit_post_colvec_loads();
-          emit_sweep(true);
-          o << "  }\n";
+    if (m.tmpl != Template::GlobalSweep) {
+      cur_level = 0;
+      emit_sweep(false);
+      o << "}\n";
+      return o.str();
+    }
+    // global stitching: sweep level 0 -> [partials -> barrier -> finalise
+    // level 1 -> barrier -> sweep level 1 -> ...]: one grid barrier pair per
+    // level of dependent column reductions
+    const int D = p.max_level;
+    for (int lv = 0; lv <= D; ++lv) {
+      cur_level = lv;
+      bool colred_here = false, sweep_here = (lv == 0);
+      for (int id : p.colreds)
+        if (phase_of(id) == lv) colred_here = true;
+      for (size_t i = 0; i < g.nodes.size(); ++i) {
+        const Node& nd = N(i);
+        if (!I(i).live || I(i).level != lv || lv == 0) continue;
+        if (nd.kind == ASTITCH_FULL || nd.kind == ASTITCH_ROWVEC) sweep_here = true;
+      }
+      if (!sweep_here && !colred_here) continue;
+      o << "  {  // ---- level " << lv << "\n";
+      if (lv > 0) emit_post_colvec_loads();
+      if (colred_here) emit_colred_acc_decl();
+      emit_sweep(lv > 0);
+      if (colred_here) {
+        emit_block_partials();
+        o << "  as::grid_barrier(bar);\n";
+        if (role == ROLE_SHARD_MAIN) {
+          emit_column_finalize(false);
+        } else {
+          emit_column_finalize(true);
+          if (lv < D) o << "  as::grid_barrier(bar);\n";
         }
       }
+      o << "  }\n";
+      if (role == ROLE_SHARD_MAIN) break;
     }
     o << "}\n";
     return o.str();

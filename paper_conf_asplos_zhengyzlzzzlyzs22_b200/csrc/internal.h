@@ -68,6 +68,7 @@ struct NodeInfo {
   OpClass cls = OpClass::Input;
   bool live = false;           // reaches an output
   bool post = false;           // depends on a column reduction (after the grid barrier)
+  int level = 0;               // number of column reductions (grid barriers) on its path
   bool candidate = false;      // dominant candidate (Step 1)
   bool dominant = false;       // final dominant
   bool sub_dominant = false;
@@ -145,7 +146,8 @@ struct Plan {
   std::vector<int> colreds;      // column reduce node ids (in order)
   std::vector<int> post_colvecs; // COLVEC values computed after the barrier (incl. colreds)
   std::vector<int> global_fulls; // FULL values buffered in HBM across the barrier
-  bool needs_sweep2 = false;
+  bool needs_sweep2 = false;     // FULL / ROWVEC work after the (first) grid barrier
+  int max_level = 0;             // grid barriers needed by dependent column reductions
   std::vector<Kernel> kernels;   // kernels launched by astitch_run, in order
   std::vector<Kernel> shard_kernels; // kernels of the sharded path (after the allreduce)
   // chunked host pipeline (astitch_run_host_pipelined): copy-in / compute /

@@ -124,22 +124,28 @@ void analyse(Plan& p) {
     info[i].cls = c;
   }
 
-  // values downstream of a column reduction run after the grid barrier
+  // Barrier levels: a value's level is the number of column reductions on
+  // its dependency path (each needs a grid barrier before it is usable);
+  // values downstream of a column reduction run after the grid barrier.
+  // A column reduction accumulates during the sweep of its operand's level.
   p.colreds.clear();
+  p.max_level = 0;
   for (int i = 0; i < n; ++i) {
     const Node& nd = g.nodes[i];
     if (!info[i].live) continue;
-    bool post = false;
-    if (nd.a >= 0 && info[nd.a].post) post = true;
-    if (nd.b >= 0 && info[nd.b].post) post = true;
+    int lv = 0;
+    if (nd.a >= 0) lv = std::max(lv, info[nd.a].level);
+    if (nd.b >= 0) lv = std::max(lv, info[nd.b].level);
     if (info[i].cls == OpClass::ReduceCol) {
-      if (post) throw Error{ASTITCH_ERR_UNSUPPORTED,
-                            "a column reduction downstream of another column reduction"};
-      post = true;
+      lv += 1;
       p.colreds.push_back(i);
     }
-    info[i].post = post;
+    info[i].level = lv;
+    info[i].post = lv > 0;
+    p.max_level = std::max(p.max_level, lv);
   }
+  if (p.max_level > 4)
+    throw Error{ASTITCH_ERR_UNSUPPORTED, "more than 4 dependent column reductions (grid barriers)"};
 
   // a2 step 1: dominant candidates = reduces, heavy EW followed by a broadcast,
   // and the outputs of the stitch op.
@@ -157,10 +163,10 @@ void analyse(Plan& p) {
     // Reading R17: a value read after the grid barrier (by anything but the
     // column reduce that accumulates it) has a one-to-many dependency across
     // groups too, so it is a candidate (power.1 of Fig. 7(a)).
-    if (!info[i].post && c != OpClass::Input && c != OpClass::Const &&
+    if (c != OpClass::Input && c != OpClass::Const &&
         (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC)) {
       for (int u : info[i].consumers)
-        if (info[u].live && info[u].post && info[u].cls != OpClass::ReduceCol) cand = true;
+        if (info[u].live && info[u].level > info[i].level && info[u].cls != OpClass::ReduceCol) cand = true;
     }
     info[i].candidate = cand;
   }
@@ -176,7 +182,7 @@ void analyse(Plan& p) {
     for (int src : {nd.a, nd.b}) {
       if (src < 0 || info[src].cls == OpClass::Const) continue;
       if (info[i].cls == OpClass::ReduceCol) continue;
-      if (!info[src].post && info[i].post) continue;
+      if (info[src].level < info[i].level) continue;
       dsu.unite(src, i);
     }
   }
@@ -238,12 +244,20 @@ void analyse(Plan& p) {
               ? Scheme::Regional : Scheme::Local;
     // a pre-barrier FULL / ROWVEC value read after the barrier (by anything
     // but the column reduction that accumulates it before the barrier)
-    auto used_after_barrier = [&](int v) {
-      for (int u : info[v].consumers)
-        if (info[u].live && info[u].post && info[u].cls != OpClass::ReduceCol) return true;
+    // (broadcasts are folded into their consumers: look through them)
+    std::function<bool(int, int)> later_use = [&](int v, int lvl) {
+      for (int u : info[v].consumers) {
+        if (!info[u].live) continue;
+        if (g.nodes[u].type == NodeType::Bcast) {
+          if (later_use(u, lvl)) return true;
+        } else if (info[u].level > lvl && info[u].cls != OpClass::ReduceCol) {
+          return true;
+        }
+      }
       return false;
     };
-    if (c != OpClass::Const && c != OpClass::Input && !info[i].post &&
+    auto used_after_barrier = [&](int v) { return later_use(v, info[v].level); };
+    if (c != OpClass::Const && c != OpClass::Input && g.nodes[i].type != NodeType::Bcast &&
         (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC) && used_after_barrier(i)) {
       s = Scheme::Global;
       info[i].global_full = true;

@@ -153,6 +153,9 @@ astitch_status astitch_plan(astitch_graph_t gr, const astitch_plan_desc* desc, a
       if (desc->sm_count <= 0) p.sm_count = sms;
     }
     analyse(p);
+    if (p.desc.shard_world > 1 && p.max_level > 1)
+      return fail(ASTITCH_ERR_UNSUPPORTED,
+                  "row-sharded plans support one level of column reductions (one allreduce)");
     select_mapping(p);
     plan_workspace(p);
     p.compulsory_bytes = compulsory_bytes(p);

@@ -38,6 +38,9 @@ REDUCED = [
     ("fig6a", 10_000 + 1, None),
     ("fig6b", 8, None),
     ("remote", None, None),
+    ("bn", None, None),
+    ("bn", 1001, 37),
+    ("bn", 20000, 512),
 ]
 
 

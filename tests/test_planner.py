@@ -140,6 +140,19 @@ def test_remote_stitching_one_kernel():
     assert d["kernel_count"] == 1 and d["mapping"]["template"] in ("row_team", "packed_tile")
 
 
+def test_batchnorm_two_barrier_levels():
+    """Dependent column reductions (BatchNorm: mean, then variance): levels
+    1 and 2, the centred values buffered in HBM (global), one kernel."""
+    d, ops, p = describe("bn")
+    assert ops["s1"]["class"] == "reduce_col" and ops["s2"]["class"] == "reduce_col"
+    assert ops["s1"]["scheme"] == "global" and ops["s2"]["scheme"] == "global"
+    assert ops["xc"]["scheme"] == "global"                 # read again after the 2nd barrier
+    assert len(d["global_fulls"]) == 1
+    assert d["kernel_count"] == 1 and d["mapping"]["template"] == "global_sweep"
+    # per level: partials -> barrier -> finalise -> barrier (publish) -> next sweep
+    assert p.source(0).count("as::grid_barrier(bar);") == 4
+
+
 def test_no_pack_ablation():
     d, _, _ = describe("fig6a", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_PACK)
     assert d["mapping"]["team"] == 32
