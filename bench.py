@@ -228,6 +228,7 @@ def main():
     ap.add_argument("--e2e-chunks", type=int, default=16,
                     help="row chunks of the pipelined host path (H2D / kernel / D2H overlap); 1 = serial")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg (ablation sweeps)")
     ap.add_argument("--flags", type=int, default=0)
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
     ap.add_argument("--rows", type=int, default=None, help="override the config's rows (experiments)")
@@ -381,7 +382,9 @@ def main():
     d2h = sum(t.numel() * t.element_size() for t in host_out)
     if world > 1:
         e2e_run = None
-    for _ in range(2):
+    if args.no_e2e:
+        args.e2e_steps = 0
+    for _ in range(2 if args.e2e_steps else 0):
         plan.run_host(host_in, host_out, dev_in[0], dev_out[0], ws=ws, chunks=args.e2e_chunks) if world == 1 else \
             _sharded_host(sp, host_in, host_out, dev_in[0], dev_out[0], ws)
     torch.cuda.synchronize()
@@ -396,12 +399,12 @@ def main():
             _sharded_host(sp, host_in, host_out, dev_in[0], dev_out[0], ws)
     h1.record(stream)
     torch.cuda.synchronize()
-    e2e_ms = h0.elapsed_time(h1) / args.e2e_steps
+    e2e_ms = h0.elapsed_time(h1) / max(args.e2e_steps, 1)
     if world > 1:
         t = torch.tensor([e2e_ms], device=f"cuda:{dev}")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
-    e2e_gbs = total_bytes / (e2e_ms * 1e-3) / 1e9
+    e2e_gbs = total_bytes / (e2e_ms * 1e-3) / 1e9 if args.e2e_steps else None
 
     # ---- oracle on the host cores: bounded sample of the same workload (rank 0, N=1)
     cpu = None
@@ -448,7 +451,7 @@ def main():
                          "peak_source": peak_src, "kernel": desc["kernels"][0]["name"],
                          "kernel_us": round(kern_ms * 1e3, 3),
                          "algorithmic_bytes_per_launch": int(nbytes)},
-            "e2e": {"value": round(e2e_gbs, 3), "unit": "GB/s", "h2d_bytes_per_step": int(h2d),
+            "e2e": None if e2e_gbs is None else {"value": round(e2e_gbs, 3), "unit": "GB/s", "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": int(d2h), "ms_per_step": round(e2e_ms, 3),
                     "api": "astitch_run_host_pipelined" if (world == 1 and args.e2e_chunks > 1) else
                            ("astitch_run_host" if world == 1 else "torch H2D/D2H + astitch_run_sharded"),

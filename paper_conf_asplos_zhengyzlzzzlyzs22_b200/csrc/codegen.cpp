@@ -421,6 +421,9 @@ struct Gen {
     for (size_t i = 0; i < g.nodes.size(); ++i)
       if (I(i).live && N(i).type == NodeType::Reduce) any_reduce = true;
     if (!any_reduce) return;
+    // values buffered in HBM across a barrier are re-read for the valid
+    // prefix only (chunks past it load as 0), which is not S: keep selects
+    if (!p.global_fulls.empty()) return;
     const double cands[3] = {-HUGE_VAL, 0.0, HUGE_VAL};
     for (double S : cands) {
       std::vector<double> vals[3];
@@ -502,7 +505,8 @@ struct Gen {
         std::string post_scale;
         {
           const Node& sn = N(src);
-          if (mx && sn.type == NodeType::Binary && sn.sub == ASTITCH_MUL && sn.kind == ASTITCH_FULL) {
+          if (mx && sn.type == NodeType::Binary && sn.sub == ASTITCH_MUL && sn.kind == ASTITCH_FULL &&
+              phase_of(src) == cur_level) {
             if (N(sn.b).type == NodeType::Const && N(sn.b).cval > 0) { post_scale = flit(N(sn.b).cval); src = sn.a; }
             else if (N(sn.a).type == NodeType::Const && N(sn.a).cval > 0) { post_scale = flit(N(sn.a).cval); src = sn.b; }
           }
@@ -710,7 +714,8 @@ struct Gen {
           std::string bs = b_row ? ("s" + std::to_string(b.a) + sfx) : ("k" + std::to_string(a.b));
           std::string nbs = "as::bc2(-(" + bs + ") * 1.4426950408889634f)";
           const Node& x = N(a.a);
-          if (x.type == NodeType::Binary && x.sub == ASTITCH_MUL && x.kind == ASTITCH_FULL) {
+          if (x.type == NodeType::Binary && x.sub == ASTITCH_MUL && x.kind == ASTITCH_FULL &&
+              phase_of(a.a) == cur_level) {
             if (N(x.b).type == NodeType::Const)
               return "as::ex2_2(as::fma2(" + ref2(x.a, sfx) + ", as::bc2(" +
                      flit(N(x.b).cval * 1.4426950408889634) + "), " + nbs + "))";
@@ -748,7 +753,8 @@ struct Gen {
           std::string bs = b_row ? ("s" + std::to_string(b.a) + sfx) : ("k" + std::to_string(a.b));
           std::string nbs = "(-(" + bs + ") * 1.4426950408889634f)";
           const Node& x = N(a.a);
-          if (x.type == NodeType::Binary && x.sub == ASTITCH_MUL && x.kind == ASTITCH_FULL) {
+          if (x.type == NodeType::Binary && x.sub == ASTITCH_MUL && x.kind == ASTITCH_FULL &&
+              phase_of(a.a) == cur_level) {
             if (N(x.b).type == NodeType::Const)
               return "as::ex2(fmaf(" + ref(x.a, "k", sfx) + ", " + flit(N(x.b).cval * 1.4426950408889634) + ", " +
                      nbs + "))";
@@ -1387,6 +1393,9 @@ struct Gen {
           emit_column_finalize(true);
           if (lv < D) o << "  as::grid_barrier(bar);\n";
         }
+      } else if (lv < D) {
+        // FORCE_GLOBAL: row-reduction results of this level are in HBM
+        o << "  as::grid_barrier(bar);\n";
       }
       o << "  }\n";
       if (role == ROLE_SHARD_MAIN) break;

@@ -128,14 +128,22 @@ void analyse(Plan& p) {
   // its dependency path (each needs a grid barrier before it is usable);
   // values downstream of a column reduction run after the grid barrier.
   // A column reduction accumulates during the sweep of its operand's level.
+  // FORCE_GLOBAL ablation (the paper's regional -> global demotion, P:L288;
+  // Table 4 mirror): a row reduction's result is stored to HBM and its
+  // consumers read it back after a grid barrier, so every consumer of a row
+  // reduction sits one barrier level above it (FULL operands are re-read from
+  // HBM or buffered there, like the values of a column-reduction level).
+  const bool force_global = (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) != 0;
   p.colreds.clear();
   p.max_level = 0;
+  auto operand_level = [&](int a) {
+    if (a < 0) return 0;
+    return info[a].level + ((force_global && info[a].cls == OpClass::ReduceRow) ? 1 : 0);
+  };
   for (int i = 0; i < n; ++i) {
     const Node& nd = g.nodes[i];
     if (!info[i].live) continue;
-    int lv = 0;
-    if (nd.a >= 0) lv = std::max(lv, info[nd.a].level);
-    if (nd.b >= 0) lv = std::max(lv, info[nd.b].level);
+    int lv = std::max(operand_level(nd.a), operand_level(nd.b));
     if (info[i].cls == OpClass::ReduceCol) {
       lv += 1;
       p.colreds.push_back(i);
@@ -232,7 +240,6 @@ void analyse(Plan& p) {
   p.global_fulls.clear();
   p.post_colvecs.clear();
   p.needs_sweep2 = false;
-  bool force_global = (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) != 0;
   for (int i = 0; i < n; ++i) {
     if (!info[i].live) continue;
     Scheme s = Scheme::Local;
@@ -273,9 +280,6 @@ void analyse(Plan& p) {
     if (info[i].post && (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC))
       p.needs_sweep2 = true;
   }
-  if (force_global)
-    throw Error{ASTITCH_ERR_UNSUPPORTED,
-                "FORCE_GLOBAL ablation (regional -> global demotion) is not implemented yet"};
 }
 
 // ------------------------------------------------------------------------ a3/a4/a6/a7
@@ -375,7 +379,7 @@ void select_mapping(Plan& p) {
   // of 1024-thread-equivalent blocks the chip runs at once = 2 per SM.
   const int64_t blocks_per_wave_1024 = 2LL * sms;
 
-  if (has_colred) {
+  if (has_colred || p.max_level > 0) {
     // ---------------------------------------------------------- global sweep
     // Column reductions (K3) need all rows: a one-wave persistent grid sweeps
     // the rows (vertical packing), each lane keeps fp32 column
@@ -403,11 +407,12 @@ void select_mapping(Plan& p) {
       if (u >= 1 && u <= 8) m.row_unroll = u;
     }
     // a6: block-level combine of the teams' column partials in smem
-    if (m.rows_per_block > 1) {
+    if (m.rows_per_block > 1 && has_colred) {
       int64_t cb = static_cast<int64_t>(m.rows_per_block) * m.team * m.chunks_per_lane * E * 4;
       if (cb <= 96 * 1024) m.smem_bytes = static_cast<int>(cb);
     }
-    why << "column reduce -> global sweep (vertical packing, grid barrier); ";
+    why << (has_colred ? "column reduce -> global sweep (vertical packing, grid barrier); "
+                       : "FORCE_GLOBAL: row reductions demoted to global (HBM + grid barrier); ");
   } else {
     // ---------------------------------------------------------- row-wise
     // Masked rows: a chunk index spans T*E columns across the team, and the

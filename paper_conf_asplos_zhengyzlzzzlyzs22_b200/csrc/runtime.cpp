@@ -153,6 +153,8 @@ astitch_status astitch_plan(astitch_graph_t gr, const astitch_plan_desc* desc, a
       if (desc->sm_count <= 0) p.sm_count = sms;
     }
     analyse(p);
+    if (p.desc.shard_world > 1 && (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL))
+      return fail(ASTITCH_ERR_UNSUPPORTED, "FORCE_GLOBAL ablation runs unsharded only");
     if (p.desc.shard_world > 1 && p.max_level > 1)
       return fail(ASTITCH_ERR_UNSUPPORTED,
                   "row-sharded plans support one level of column reductions (one allreduce)");

@@ -147,6 +147,23 @@ def test_parity_split_long_rows_default():
     _compare(spec, got, evaluate(spec, x))
 
 
+@pytest.mark.parametrize("cfg,rows,cols", [("C1", None, None), ("C2", 300, None), ("C3", 3 * 256 + 7, None),
+                                           ("C4", 20_000 + 3, None), ("fig7a", None, None), ("remote", None, None),
+                                           ("C5", 3000 + 5, None), ("bn", 1001, 37)])
+def test_parity_force_global_ablation(cfg, rows, cols):
+    """FORCE_GLOBAL ablation (regional -> global demotion): row
+    reductions go through HBM and a grid barrier; same results, one kernel."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 256
+    x = gen.generate(cfg, spec)
+    got, plan = run_gpu(spec, x, return_plan=True, flags=A.FLAG_FORCE_GLOBAL)
+    d = plan.describe()
+    assert d["mapping"]["template"] == "global_sweep" and d["kernel_count"] == 1
+    _compare(spec, got, evaluate(spec, x))
+
+
 @pytest.mark.parametrize("cfg,rows,cols,world", [("C5", 3001, 1024, 2), ("C5", 4099, 256, 8), ("fig7a", 1001, 96, 3),
                                                  ("C5int", 4096, 128, 4), ("C2", 777, 768, 4), ("C3", 4 * 512, 512, 4)])
 def test_virtual_shards(cfg, rows, cols, world):

@@ -153,6 +153,23 @@ def test_batchnorm_two_barrier_levels():
     assert p.source(0).count("as::grid_barrier(bar);") == 4
 
 
+def test_force_global_ablation_demotes_row_reductions():
+    """FORCE_GLOBAL (regional -> global demotion; the Table 4 mirror):
+    every row reduction is stored to HBM and read back after a grid barrier."""
+    d, ops, p = describe("C1", flags=A.FLAG_NO_COMPILE | A.FLAG_FORCE_GLOBAL)
+    assert ops["m"]["scheme"] == "global" and ops["s"]["scheme"] == "global"
+    assert d["mapping"]["template"] == "global_sweep" and d["kernel_count"] == 1
+    # softmax: max | exp + sum | divide -> 3 sweeps, 2 barriers; e buffered in HBM
+    assert p.source(0).count("as::grid_barrier(bar);") == 2
+    assert set(d["global_fulls"]) == {ops[n]["id"] for n in ("m", "e", "s")}
+    d2, ops2, p2 = describe("C2", flags=A.FLAG_NO_COMPILE | A.FLAG_FORCE_GLOBAL)
+    assert p2.source(0).count("as::grid_barrier(bar);") == 2   # mean | variance | normalise
+    d3, _, _ = describe("C1")
+    assert d3["mapping"]["template"] == "row_team"
+    with pytest.raises(A.AstitchError):
+        describe("C1", flags=A.FLAG_NO_COMPILE | A.FLAG_FORCE_GLOBAL, shard_rank=0, shard_world=2)
+
+
 def test_no_pack_ablation():
     d, _, _ = describe("fig6a", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_PACK)
     assert d["mapping"]["team"] == 32
