@@ -38,6 +38,7 @@ WORKLOAD_NAMES = {
     "C3": "Transformer attention masked softmax bf16 [64*16*512,512], lengths 37-512",
     "C4": "DIEN row standardise fp32 [2,000,000,36]",
     "C5": "bias-GELU backward + bias-grad column reduce + in-kernel SGD step, bf16 [1,048,576,1024]",
+    "C3v": "Transformer attention softmax bf16, packed varlen (64 batches x 16 heads x L_b rows of L_b, L_b 37-512)",
 }
 def spec_name(cfg):
     from workloads import specs
@@ -138,6 +139,14 @@ def compulsory_bytes(spec, inputs, rows=None):
     es = {"F32": 4, "BF16": 2, "F16": 2, "I32": 4}
     mask = spec.get("mask")
     valid = None
+    seg = spec.get("segments")
+    if seg is not None:  # packed varlen: every element of every row is valid (no padding)
+        valid = int(sum(r * c for r, c in zip(seg["seg_rows"], seg["seg_cols"])))
+        kinds = {"FULL": valid, "ROWVEC": R, "COLVEC": C}
+        b = sum(kinds[k] * es[dt] for _, k, dt in spec["inputs"] if k in kinds)
+        b += 16 * len(seg["seg_rows"])
+        b += sum(kinds[_out_kind(spec, n)] * es[dt] for n, dt in spec["outputs"])
+        return b
     if mask is not None:
         L = np.clip(np.asarray(inputs[mask["lengths"]], dtype=np.int64), 0, C)
         rps = mask["rows_per_segment"]
@@ -189,12 +198,31 @@ def run_reference(args, rank, world):
     from oracle import evaluate
     from workloads import specs
     cfg = args.config
-    spec_full = specs.get(cfg)
+    spec_full = _full_spec(cfg)
+    if spec_full.get("segments"):  # packed varlen: a bounded subset of whole segments
+        from workloads import gen
+        spec = gen.ragged_subset(spec_full, list(range(4)))
+        x = make_inputs(cfg, spec)
+        return _reference_line(args, world, cfg, spec, spec_full, x)
     sample_rows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 200_000, "C5": 16384}.get(cfg, 4096)
     spec = specs.get(cfg, rows=min(sample_rows, spec_full["rows"]))
     if spec.get("mask"):
         spec["mask"]["rows_per_segment"] = min(spec["mask"]["rows_per_segment"], spec["rows"])
     x = make_inputs(cfg, spec)
+    return _reference_line(args, world, cfg, spec, spec_full, x)
+
+
+def _full_spec(cfg, rows=None, cols=None):
+    """The workload spec; packed varlen specs get their seeded segment layout."""
+    from workloads import gen, specs
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("segments"):
+        spec = gen.ragged_spec(spec, gen.CONFIG_SEEDS.get(cfg, 0))
+    return spec
+
+
+def _reference_line(args, world, cfg, spec, spec_full, x):
+    from oracle import evaluate
     nbytes = compulsory_bytes(spec, x)
     for _ in range(args.warmup):
         evaluate(spec, x)
@@ -204,6 +232,9 @@ def run_reference(args, rank, world):
     dt = (time.perf_counter() - t0) / args.steps
     gbs = nbytes / dt / 1e9
     sample = f"{spec['rows']} of {spec_full['rows']} rows x {spec['cols']} cols per step"
+    if spec.get("segments"):
+        sample = (f"segments 0-{len(spec['segments']['seg_rows']) - 1} of {len(spec_full['segments']['seg_rows'])} "
+                  f"({spec['rows']} of {spec_full['rows']} packed rows) per step")
     return {
         "impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
@@ -261,18 +292,29 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
 
     cfg = args.config
-    spec = specs.get(cfg, rows=args.rows, cols=args.cols)
+    spec = _full_spec(cfg, rows=args.rows, cols=args.cols)
+    ragged = bool(spec.get("segments"))
+    if ragged and world > 1:
+        # packed varlen: shard whole segments (independent problems, no
+        # communication), contiguous ranges balanced by packed bytes
+        from workloads import gen
+        seg = spec["segments"]
+        w = np.asarray(seg["seg_rows"], dtype=np.float64) * (np.asarray(seg["seg_cols"]) + 7) // 8 * 8
+        cut = np.searchsorted(np.cumsum(w), np.sum(w) * np.arange(1, world) / world)
+        bounds = [0] + [int(c) + 1 for c in cut] + [len(w)]
+        spec = gen.ragged_subset(spec, list(range(bounds[rank], max(bounds[rank], bounds[rank + 1]))))
     R, C = spec["rows"], spec["cols"]
     graph = A.Graph.from_spec(spec)
     comm = Comm.from_process_group(dev) if world > 1 else None
-    sp = ShardedPlan(graph, R, C, world, rank, dev, comm=comm, flags=args.flags)
+    sp = ShardedPlan(graph, R, C, 1 if ragged else world, 0 if ragged else rank, dev, comm=comm, flags=args.flags)
     plan = sp.plan
     desc = plan.describe()
     r0, nr = sp.row_begin, sp.row_count
 
     # seeded inputs of this rank's row slice, resident in HBM
     t_gen = time.time()
-    x = make_inputs(cfg, spec, row_start=r0 if r0 % 8192 == 0 else 0, row_count=nr) if r0 % 8192 == 0 \
+    x = make_inputs(cfg, spec) if ragged else \
+        make_inputs(cfg, spec, row_start=r0 if r0 % 8192 == 0 else 0, row_count=nr) if r0 % 8192 == 0 \
         else {k: v[r0:r0 + nr] if getattr(v, "ndim", 0) == 2 else v
               for k, v in make_inputs(cfg, spec).items()}
     if spec.get("mask") and world > 1:  # the rank's slice of the per-segment lengths
@@ -410,13 +452,18 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         from oracle import evaluate
-        srows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 400_000, "C5": 131_072}.get(cfg, 4096)
-        sspec = specs.get(cfg, rows=min(srows, R))
-        if sspec.get("mask"):
-            sspec["mask"]["rows_per_segment"] = min(sspec["mask"]["rows_per_segment"], sspec["rows"])
-        sx = {k: (v[: sspec["rows"]] if getattr(v, "ndim", 0) == 2 else v) for k, v in x.items()}
-        if sspec.get("mask"):
-            sx[sspec["mask"]["lengths"]] = x[spec["mask"]["lengths"]][: -(-sspec["rows"] // sspec["mask"]["rows_per_segment"])]
+        if ragged:  # whole segments 0-7 (bit-identical to the full problem's)
+            from workloads import gen
+            sspec = gen.ragged_subset(spec, list(range(min(8, len(spec["segments"]["seg_rows"])))))
+            sx = make_inputs(cfg, sspec)
+        else:
+            srows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 400_000, "C5": 131_072}.get(cfg, 4096)
+            sspec = specs.get(cfg, rows=min(srows, R))
+            if sspec.get("mask"):
+                sspec["mask"]["rows_per_segment"] = min(sspec["mask"]["rows_per_segment"], sspec["rows"])
+            sx = {k: (v[: sspec["rows"]] if getattr(v, "ndim", 0) == 2 else v) for k, v in x.items()}
+            if sspec.get("mask"):
+                sx[sspec["mask"]["lengths"]] = x[spec["mask"]["lengths"]][: -(-sspec["rows"] // sspec["mask"]["rows_per_segment"])]
         reps = 3 if cfg in ("C1", "C2") else 1
         t0 = time.perf_counter()
         for _ in range(reps):

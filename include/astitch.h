@@ -61,7 +61,8 @@ typedef enum {
   ASTITCH_ROWVEC = 1,  /* [rows]   (one value per row)                   */
   ASTITCH_COLVEC = 2,  /* [cols]   (one value per column)                */
   ASTITCH_SCALAR = 3,  /* constant                                       */
-  ASTITCH_LENGTHS = 4  /* int32 valid lengths, one per row segment       */
+  ASTITCH_LENGTHS = 4, /* int32 valid lengths, one per row segment       */
+  ASTITCH_SEGMENTS = 5 /* int32 [nseg][4] packed varlen segment table    */
 } astitch_kind;
 
 /* Element-wise unary ops.  Light vs heavy follows P:L101 (heavy: exp, log,
@@ -126,6 +127,34 @@ astitch_status astitch_graph_broadcast(astitch_graph_t g, astitch_axis axis, ast
  * RMAX) and written as 0 in FULL outputs.  At most one mask per graph. */
 astitch_status astitch_graph_lengths(astitch_graph_t g, int64_t rows_per_segment,
                                      astitch_value_t* out);
+/* Packed variable-length rows ("varlen" layout: irregular shapes without
+ * padding, Sec. 3.3 Challenge II).  Adds an
+ * int32 SEGMENTS input (next in input order) of nseg entries of 4 int32
+ *     { row_start, cols, pitch, offset8 }:
+ * segment s owns global rows [row_start_s, row_start_{s+1}) (row_start_0 = 0,
+ * increasing, row_start_nseg := plan rows); each of its rows has `cols_s`
+ * elements (1 <= cols_s <= plan cols), stored in EVERY FULL tensor (input and
+ * output) at element offset 8*offset8_s + (r - row_start_s) * pitch_s, with
+ * pitch_s a multiple of 8 and >= cols_s.  FULL tensors therefore hold `elems`
+ * elements (>= the last segment's end); ROWVEC tensors stay [rows], COLVEC
+ * [cols] (column c of any segment reads entry c).  The plan's cols is the
+ * maximum row length: the thread mapping is chosen for it and shorter rows
+ * are handled like key-padding masks (chunks past cols_s are skipped), but
+ * nothing past a row is read and only whole 16-byte chunks up to cols_s are
+ * written (elements cols_s .. next 16-byte boundary are written as 0, inside
+ * the pitch).  Row-wise subgraphs only: column reductions, masks, sharding and
+ * FORCE_GLOBAL are ERR_UNSUPPORTED with segments.  The table must be valid
+ * (see astitch_segments_layout); it is read on the device and not checked. */
+astitch_status astitch_graph_segments(astitch_graph_t g, int32_t nseg, int64_t elems,
+                                      astitch_value_t* out);
+/* Host helper: the canonical segment table for nseg segments of seg_rows[s]
+ * rows x seg_cols[s] columns, packed back to back in segment order with
+ * pitch = cols rounded up to a multiple of 8 elements.  Writes table[4*nseg],
+ * *rows = total rows and *elems = total elements per FULL tensor.
+ * Errors: ERR_INVALID_ARGUMENT (NULL, nseg < 1, rows < 0, cols < 1),
+ * ERR_SHAPE (offsets beyond 2^31 x 8 elements). */
+astitch_status astitch_segments_layout(int32_t nseg, const int64_t* seg_rows, const int32_t* seg_cols,
+                                       int32_t* table, int64_t* rows, int64_t* elems);
 /* Marks value v as a stitch-op output stored with dtype (F32 / BF16 / F16).
  * FULL, ROWVEC and COLVEC values can be outputs. */
 astitch_status astitch_graph_output(astitch_graph_t g, astitch_value_t v, astitch_dtype dtype,

@@ -187,12 +187,60 @@ def _levels(spec):
 # ----------------------------------------------------------------------------
 
 
+def evaluate_ragged(spec: dict, inputs: dict) -> dict:
+    """Packed varlen layout (spec "segments", include/astitch.h
+    astitch_graph_segments): segment s is an independent dense problem of
+    rows_s x cols_s, read from the packed buffers through the segment table
+    {row_start, cols, pitch, offset/8}.  Each segment is evaluated by
+    :func:`evaluate` as the plain unmasked graph; FULL outputs are returned in
+    the packed layout (1-D, pitch padding 0), ROWVEC outputs per global row."""
+    seg = spec["segments"]
+    table = np.asarray(inputs[seg["table"]], dtype=np.int64)
+    R = int(spec["rows"])
+    elems = int(seg["elems"])
+    kind = _kinds(spec)
+    assert not any(op[1] == "reduce" and op[3] == "COL" for op in spec["ops"]), \
+        "packed varlen subgraphs are row-wise"
+    outs = {}
+    for n, _ in spec["outputs"]:
+        outs[n] = np.zeros(elems if kind[n] == "FULL" else R, dtype=np.float64)
+    sub_inputs_decl = [(n, k, d) for n, k, d in spec["inputs"] if k != "SEGMENTS"]
+    for s in range(table.shape[0]):
+        r0, cols, pitch, off = int(table[s, 0]), int(table[s, 1]), int(table[s, 2]), 8 * int(table[s, 3])
+        r1 = int(table[s + 1, 0]) if s + 1 < table.shape[0] else R
+        nr = r1 - r0
+        if nr <= 0:
+            continue
+        sub = {"name": spec["name"], "rows": nr, "cols": cols, "inputs": sub_inputs_decl, "mask": None,
+               "ops": spec["ops"], "outputs": spec["outputs"]}
+        sin = {}
+        for n, k, d in sub_inputs_decl:
+            a = inputs[n]
+            if k == "FULL":
+                sin[n] = np.asarray(a)[off: off + nr * pitch].reshape(nr, pitch)[:, :cols]
+            elif k == "ROWVEC":
+                sin[n] = np.asarray(a)[r0:r1]
+            elif k == "COLVEC":
+                sin[n] = np.asarray(a)[:cols]
+            else:
+                raise ValueError(k)
+        res = evaluate(sub, sin)
+        for n, _ in spec["outputs"]:
+            if kind[n] == "FULL":
+                outs[n][off: off + nr * pitch].reshape(nr, pitch)[:, :cols] = res[n]
+            else:
+                outs[n][r0:r1] = res[n]
+    return outs
+
+
 def evaluate(spec: dict, inputs: dict, row_chunk: int = 16384) -> dict:
     """Evaluate ``spec`` on ``inputs`` (raw stored arrays keyed by input name).
 
     Returns ``{output name: fp64 ndarray}`` with shapes FULL [R,C], ROWVEC [R],
-    COLVEC [C], SCALAR ().
+    COLVEC [C], SCALAR ().  Packed varlen specs go to :func:`evaluate_ragged`.
     """
+    if spec.get("segments"):
+        return evaluate_ragged(spec, inputs)
     R, C = int(spec["rows"]), int(spec["cols"])
     kind = _kinds(spec)
     level = _levels(spec)

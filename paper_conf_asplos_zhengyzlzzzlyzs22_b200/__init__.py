@@ -14,6 +14,6 @@ from ._lib import (FLAG_FORCE_GLOBAL, FLAG_LAUNCH_CHECK, FLAG_NO_COMPILE, FLAG_N
                    FLAG_FORCE_SPLIT, FLAG_NO_PREFETCH, FLAG_NO_SPLIT, FLAG_NO_TMA,
                    FLAG_STRICT_SINGLE_KERNEL, LIB_PATH,
                    AstitchError)
-from .api import Graph, Plan, bench_barrier, bench_copy, plan, shard_rows  # noqa: F401
+from .api import Graph, Plan, bench_barrier, bench_copy, plan, segments_layout, shard_rows  # noqa: F401
 
 __version__ = "0.1.0"

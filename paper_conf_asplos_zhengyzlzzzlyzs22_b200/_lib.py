@@ -19,7 +19,7 @@ STATUS = {
 }
 
 DTYPES = {"F32": 0, "BF16": 1, "F16": 2, "I32": 3}
-KINDS = {"FULL": 0, "ROWVEC": 1, "COLVEC": 2, "SCALAR": 3, "LENGTHS": 4}
+KINDS = {"FULL": 0, "ROWVEC": 1, "COLVEC": 2, "SCALAR": 3, "LENGTHS": 4, "SEGMENTS": 5}
 UNOPS = {n: i for i, n in enumerate(["NEG", "ABS", "EXP", "LOG", "TANH", "ERF", "SQRT", "RSQRT", "RCP",
                                      "SIGMOID", "GELU_TANH", "GELU_ERF", "GELU_TANH_GRAD"])}
 BINOPS = {n: i for i, n in enumerate(["ADD", "SUB", "MUL", "DIV", "MAX", "MIN", "POW"])}
@@ -72,6 +72,9 @@ _sig = {
     "astitch_graph_reduce": (ct.c_int, [_vp, ct.c_int, ct.c_int, ct.c_int32, _i32p]),
     "astitch_graph_broadcast": (ct.c_int, [_vp, ct.c_int, ct.c_int32, _i32p]),
     "astitch_graph_lengths": (ct.c_int, [_vp, ct.c_int64, _i32p]),
+    "astitch_graph_segments": (ct.c_int, [_vp, ct.c_int32, ct.c_int64, _i32p]),
+    "astitch_segments_layout": (ct.c_int, [ct.c_int32, ct.POINTER(ct.c_int64), _i32p, _i32p,
+                                           ct.POINTER(ct.c_int64), ct.POINTER(ct.c_int64)]),
     "astitch_graph_output": (ct.c_int, [_vp, ct.c_int32, ct.c_int, _i32p]),
     "astitch_plan": (ct.c_int, [_vp, ct.POINTER(PlanDesc), ct.POINTER(_vp)]),
     "astitch_plan_destroy": (ct.c_int, [_vp]),

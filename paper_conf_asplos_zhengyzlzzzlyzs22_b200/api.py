@@ -33,6 +33,7 @@ class Graph:
         check(lib.astitch_graph_create(ct.byref(h)), "astitch_graph_create")
         self._h = h
         self.names: dict[str, int] = {}
+        self.ragged = None  # (nseg, elems) once astitch_graph_segments was called
 
     def __del__(self):
         h = getattr(self, "_h", None)
@@ -56,6 +57,14 @@ class Graph:
     def lengths(self, rows_per_segment: int) -> int:
         v = self._out()
         check(lib.astitch_graph_lengths(self._h, int(rows_per_segment), ct.byref(v)), "astitch_graph_lengths")
+        return v.value
+
+    def segments(self, nseg: int, elems: int) -> int:
+        """Packed varlen rows (astitch_graph_segments): adds the int32 [nseg, 4]
+        segment-table input; FULL tensors then hold `elems` packed elements."""
+        v = self._out()
+        check(lib.astitch_graph_segments(self._h, int(nseg), int(elems), ct.byref(v)), "astitch_graph_segments")
+        self.ragged = (int(nseg), int(elems))
         return v.value
 
     def const(self, value: float) -> int:
@@ -99,6 +108,10 @@ class Graph:
             if kind == "LENGTHS":
                 assert mask is not None and mask["lengths"] == name
                 n[name] = g.lengths(mask["rows_per_segment"])
+            elif kind == "SEGMENTS":
+                seg = spec["segments"]
+                assert seg["table"] == name
+                n[name] = g.segments(len(seg["seg_rows"]), seg["elems"])
             else:
                 n[name] = g.input(kind, dtype)
         for op in spec["ops"]:
@@ -140,6 +153,7 @@ class Plan:
         check(lib.astitch_plan(graph.handle, ct.byref(d), ct.byref(h)), "astitch_plan")
         self._h = h
         self.rows, self.cols, self.device = int(rows), int(cols), int(device)
+        self.ragged = graph.ragged
         ni, no = ct.c_int32(), ct.c_int32()
         check(lib.astitch_plan_io_count(h, ct.byref(ni), ct.byref(no)), "astitch_plan_io_count")
         self.inputs = [self._io(0, i) for i in range(ni.value)]
@@ -196,7 +210,9 @@ class Plan:
     def io_shape(self, kind: str, rows: int | None = None, nseg: int | None = None):
         R = self.rows if rows is None else rows
         if kind == "FULL":
-            return (R, self.cols)
+            return (self.ragged[1],) if self.ragged else (R, self.cols)
+        if kind == "SEGMENTS":
+            return (self.ragged[0], 4)
         if kind == "ROWVEC":
             return (R,)
         if kind == "COLVEC":
@@ -259,6 +275,20 @@ def plan(graph: Graph, rows: int, cols: int, device: int = 0, flags: int = 0, **
     return Plan(graph, rows, cols, device=device, flags=flags, **kw)
 
 
+def segments_layout(seg_rows, seg_cols):
+    """astitch_segments_layout: canonical packed varlen table for segments of
+    seg_rows[s] x seg_cols[s] (pitch = cols rounded up to 8 elements).
+    Returns (table int32 [nseg, 4] as a list of rows, total rows, total elements)."""
+    nseg = len(seg_rows)
+    assert len(seg_cols) == nseg
+    r = (ct.c_int64 * nseg)(*[int(x) for x in seg_rows])
+    c = (ct.c_int32 * nseg)(*[int(x) for x in seg_cols])
+    t = (ct.c_int32 * (4 * nseg))()
+    rows, elems = ct.c_int64(), ct.c_int64()
+    check(lib.astitch_segments_layout(nseg, r, c, t, ct.byref(rows), ct.byref(elems)), "astitch_segments_layout")
+    return [list(t[4 * s: 4 * s + 4]) for s in range(nseg)], rows.value, elems.value
+
+
 def shard_rows(rows: int, world: int, rank: int) -> tuple[int, int]:
     b, c = ct.c_int64(), ct.c_int64()
     check(lib.astitch_shard_rows(int(rows), int(world), int(rank), ct.byref(b), ct.byref(c)), "astitch_shard_rows")
@@ -275,4 +305,4 @@ def bench_copy(device: int, src, dst, nbytes: int, stream=None) -> None:
                                  ct.c_void_p(_stream_ptr(stream))), "astitch_bench_copy")
 
 
-__all__ = ["Graph", "Plan", "plan", "shard_rows", "bench_barrier", "bench_copy", "AstitchError"]
+__all__ = ["Graph", "Plan", "plan", "segments_layout", "shard_rows", "bench_barrier", "bench_copy", "AstitchError"]

@@ -35,7 +35,7 @@ struct Gen {
   std::ostringstream o;
   int T, V, E, NE, RPB, U;
   long long C;
-  bool masked, exact;
+  bool masked, exact, ragged = false;
   int role;
 
   Gen(const Plan& pp, int r) : p(pp), g(pp.g), m(pp.map), role(r) {
@@ -46,7 +46,8 @@ struct Gen {
     RPB = m.rows_per_block;
     U = m.row_unroll;
     C = p.desc.cols;
-    masked = g.lengths_node >= 0;
+    ragged = g.segments_node >= 0;
+    masked = g.lengths_node >= 0 || ragged;  // varlen rows: masks of the row's own length
     exact = (static_cast<long long>(T) * V * E == C);
     split = (m.tmpl == Template::SplitRow);
     compute_precise();
@@ -179,9 +180,13 @@ struct Gen {
     for (size_t i = 0; i < g.nodes.size(); ++i)
       if (N(i).type == NodeType::Const && I(i).live)
         o << "  const float k" << i << " = " << flit(N(i).cval) << ";\n";
-    if (masked) {
+    if (g.lengths_node >= 0) {
       o << "  const int* __restrict__ Lp = (const int*)p.in[" << N(g.lengths_node).input_index << "];\n";
       o << "  constexpr long long RPS = " << g.rows_per_segment << "LL;\n";
+    }
+    if (ragged) {
+      o << "  const int4* __restrict__ SG = (const int4*)p.in[" << N(g.segments_node).input_index << "];\n";
+      o << "  constexpr int NSEG = " << g.nseg << ";\n";
     }
   }
 
@@ -303,8 +308,8 @@ struct Gen {
       std::string cond = act;
       if (!exact || masked) cond += " && c0 < " + lim;
       o << "      if (" << cond << ") r" << s << sfx << "[j] = "
-        << (st.ws_buf ? "as::ldg_cg(" : "as::ldg(") << "gs" << s << " + (" << row
-        << ") * CH + (j * T + lane));\n";
+        << (st.ws_buf ? "as::ldg_cg(" : "as::ldg(") << "gs" << s << " + " << rowbase(row, lim)
+        << " + (j * T + lane));\n";
       // chunks that are not loaded need no defined bits when the mask is
       // absorbed: the unpack step overwrites every invalid element with S
       if (!(absorb && !st.ws_buf)) o << "      else r" << s << sfx << "[j] = " << raw_t(st) << "{};\n";
@@ -816,7 +821,7 @@ struct Gen {
       if (nd.kind == ASTITCH_FULL) {
         std::string rt = "as::Raw<" + std::to_string(nb(dt)) + ">";
         o << "    if (" << act << ") {\n      " << rt << "* __restrict__ op_ = (" << rt << "*)p.out[" << k
-          << "] + (" << row << ") * CH;\n";
+          << "] + " << rowbase(row, lim) << ";\n";
         o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
         std::string val = ref(id, "(j * E + e)", sfx);
         o << "        float t_[E];\n";
@@ -827,7 +832,8 @@ struct Gen {
         } else {
           o << "#pragma unroll\n        for (int e = 0; e < E; ++e) t_[e] = " << val << ";\n";
         }
-        if (!exact) o << "        if ((long long)(j * T + lane) < CH)\n";
+        if (ragged) o << "        if ((j * T + lane) * E < " << lim << ")  // chunks of the row only (packed)\n";
+        else if (!exact) o << "        if ((long long)(j * T + lane) < CH)\n";
         o << "        as::stg(op_ + (j * T + lane), as::Conv<" << dt_code(dt) << ", E>::pack(t_));\n";
         o << "      }\n    }\n";
       } else if (nd.kind == ASTITCH_ROWVEC) {
@@ -857,6 +863,24 @@ struct Gen {
       }
     }
     (void)lim;
+  }
+
+  // declaration of the valid bound `lim` of row `row` (active flag `act`); for
+  // packed varlen rows also `lim`_b = the row's first chunk in every FULL tensor
+  std::string limdecl(const std::string& lim, const std::string& act, const std::string& row) const {
+    if (!ragged) {
+      if (!masked) return "const int " + lim + " = (int)C;";
+      return "const int " + lim + " = " + act + " ? " + lim_expr(row) + " : 0;";
+    }
+    return "const int4 " + lim + "_s = " + act + " ? as::seg_find<NSEG>(SG, (int)(" + row +
+           ")) : make_int4(0, 0, 0, 0);\n    const int " + lim + " = min(" + lim + "_s.y, (int)C);\n    const long long " +
+           lim + "_b = ((long long)" + lim + "_s.w * 8 + (long long)((" + row + ") - " + lim + "_s.x) * " + lim +
+           "_s.z) / E; (void)" + lim + "_b;";
+  }
+  // first chunk of row `row` in a FULL tensor (row-major [R, C] or packed varlen)
+  std::string rowbase(const std::string& row, const std::string& lim) const {
+    if (ragged) return lim + "_b";
+    return "(" + row + ") * CH";
   }
 
   std::string lim_expr(const std::string& row) const {
@@ -919,7 +943,7 @@ struct Gen {
     // register count on B200 (C3: 120 vs 80 regs, 153 vs 146 us), so the copy
     // form is the default; ASTITCH_PINGPONG=1 selects the other for experiments.
     const char* pp_env = getenv("ASTITCH_PINGPONG");
-    if (pf && pp_env && atoi(pp_env) == 1) {
+    if (pf && pp_env && atoi(pp_env) == 1 && !ragged) {
       // ping-pong buffers a / b
       for (int u = 0; u < U; ++u)
         for (const char* bf : {"a", "b"})
@@ -951,7 +975,7 @@ struct Gen {
         std::string s = su + std::to_string(u) + "n";
         for (size_t q = 0; q < streams.size(); ++q) o << "  " << raw_t(streams[q]) << " r" << q << s << "[V];\n";
         o << "  {\n    const bool pact = prow" << u << " < R;\n";
-        o << "    const int plim =" << (masked ? "pact ? " + lim_expr("prow" + std::to_string(u)) + " : 0" : "(int)C") << ";\n";
+        o << "    " << limdecl("plim", "pact", "prow" + std::to_string(u)) << "\n";
         o << "    (void)plim;\n";
         emit_loads("prow" + std::to_string(u), "pact", "plim", s, false);
         o << "  }\n";
@@ -962,7 +986,7 @@ struct Gen {
       std::string s = su + std::to_string(u);
       o << "    const " << rt << " row" << u << " = base + " << u << " * RPB + team;\n";
       o << "    const bool act" << u << " = row" << u << " < R;\n";
-      o << "    const int lim" << u << " = " << (masked ? "act" + std::to_string(u) + " ? " + lim_expr("row" + std::to_string(u)) + " : 0" : "(int)C") << ";\n";
+      o << "    " << limdecl("lim" + std::to_string(u), "act" + std::to_string(u), "row" + std::to_string(u)) << "\n";
       o << "    (void)lim" << u << ";\n";
     }
     if (pf) {
@@ -978,7 +1002,7 @@ struct Gen {
         o << "    {\n";
         o << "      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
         o << "      const bool pact = nrow < R;\n";
-        o << "      const int plim =" << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
+        o << "      " << limdecl("plim", "pact", "nrow") << "\n";
         o << "      (void)plim;\n";
         emit_loads("nrow", "pact", "plim", s, false);
         o << "    }\n";

@@ -3,6 +3,7 @@
 // unary/binary ops (broadcast is element-wise-like), row- and
 // column-reduce, plus the key-padding LENGTHS mask of BASELINE configs[2].
 #include <cmath>
+#include <cstdint>
 #include <string>
 
 #include "internal.h"
@@ -45,6 +46,7 @@ const char* kind_name(astitch_kind k) {
     case ASTITCH_COLVEC: return "COLVEC";
     case ASTITCH_SCALAR: return "SCALAR";
     case ASTITCH_LENGTHS: return "LENGTHS";
+    case ASTITCH_SEGMENTS: return "SEGMENTS";
   }
   return "?";
 }
@@ -139,7 +141,8 @@ astitch_status astitch_graph_lengths(astitch_graph_t g, int64_t rows_per_segment
                                      astitch_value_t* out) {
   if (!g || !out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL graph or out");
   if (rows_per_segment < 1) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "rows_per_segment < 1");
-  if (g->g.lengths_node >= 0) return fail(ASTITCH_ERR_INVALID_GRAPH, "graph already has a mask");
+  if (g->g.lengths_node >= 0 || g->g.segments_node >= 0)
+    return fail(ASTITCH_ERR_INVALID_GRAPH, "graph already has a mask or segments");
   if (g->g.inputs.size() >= static_cast<size_t>(kMaxIO))
     return fail(ASTITCH_ERR_UNSUPPORTED, "too many inputs (max 16)");
   Node n;
@@ -154,6 +157,53 @@ astitch_status astitch_graph_lengths(astitch_graph_t g, int64_t rows_per_segment
     g->g.rows_per_segment = rows_per_segment;
   }
   return s;
+}
+
+astitch_status astitch_graph_segments(astitch_graph_t g, int32_t nseg, int64_t elems,
+                                      astitch_value_t* out) {
+  if (!g || !out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL graph or out");
+  if (nseg < 1) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "nseg < 1");
+  if (elems < 0) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "elems < 0");
+  if (g->g.lengths_node >= 0 || g->g.segments_node >= 0)
+    return fail(ASTITCH_ERR_INVALID_GRAPH, "graph already has a mask or segments");
+  if (g->g.inputs.size() >= static_cast<size_t>(kMaxIO))
+    return fail(ASTITCH_ERR_UNSUPPORTED, "too many inputs (max 16)");
+  Node n;
+  n.type = NodeType::Input;
+  n.kind = ASTITCH_SEGMENTS;
+  n.dtype = ASTITCH_I32;
+  n.input_index = static_cast<int>(g->g.inputs.size());
+  astitch_status s = push(g->g, n, out);
+  if (s == ASTITCH_OK) {
+    g->g.inputs.push_back(*out);
+    g->g.segments_node = *out;
+    g->g.nseg = nseg;
+    g->g.seg_elems = elems;
+  }
+  return s;
+}
+
+astitch_status astitch_segments_layout(int32_t nseg, const int64_t* seg_rows, const int32_t* seg_cols,
+                                       int32_t* table, int64_t* rows, int64_t* elems) {
+  if (!seg_rows || !seg_cols || !table || !rows || !elems)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (nseg < 1) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "nseg < 1");
+  int64_t r = 0, off = 0;  // off in elements (always a multiple of 8)
+  for (int32_t s = 0; s < nseg; ++s) {
+    if (seg_rows[s] < 0 || seg_cols[s] < 1) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "segment rows < 0 or cols < 1");
+    const int64_t pitch = (static_cast<int64_t>(seg_cols[s]) + 7) / 8 * 8;
+    if (r > INT32_MAX || off / 8 > INT32_MAX) return fail(ASTITCH_ERR_SHAPE, "segment table overflows int32");
+    table[4 * s + 0] = static_cast<int32_t>(r);
+    table[4 * s + 1] = seg_cols[s];
+    table[4 * s + 2] = static_cast<int32_t>(pitch);
+    table[4 * s + 3] = static_cast<int32_t>(off / 8);
+    r += seg_rows[s];
+    off += seg_rows[s] * pitch;
+  }
+  if (r > INT32_MAX) return fail(ASTITCH_ERR_SHAPE, "segment table overflows int32");
+  *rows = r;
+  *elems = off;
+  return ASTITCH_OK;
 }
 
 astitch_status astitch_graph_const(astitch_graph_t g, double v, astitch_value_t* out) {
@@ -172,7 +222,8 @@ astitch_status astitch_graph_unary(astitch_graph_t g, astitch_unop op, astitch_v
   if (op < 0 || op >= ASTITCH_UNOP_COUNT) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad unop");
   if (!valid_value(g->g, a)) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad operand");
   astitch_kind k = g->g.nodes[a].kind;
-  if (k == ASTITCH_LENGTHS) return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS is not an operand");
+  if (k == ASTITCH_LENGTHS || k == ASTITCH_SEGMENTS)
+    return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS / SEGMENTS is not an operand");
   if (k == ASTITCH_SCALAR)
     return fail(ASTITCH_ERR_UNSUPPORTED, "unary op on a SCALAR constant (fold it on the host)");
   Node n;
@@ -190,8 +241,8 @@ astitch_status astitch_graph_binary(astitch_graph_t g, astitch_binop op, astitch
   if (!valid_value(g->g, a) || !valid_value(g->g, b))
     return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad operand");
   astitch_kind ka = g->g.nodes[a].kind, kb = g->g.nodes[b].kind;
-  if (ka == ASTITCH_LENGTHS || kb == ASTITCH_LENGTHS)
-    return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS is not an operand");
+  if (ka == ASTITCH_LENGTHS || kb == ASTITCH_LENGTHS || ka == ASTITCH_SEGMENTS || kb == ASTITCH_SEGMENTS)
+    return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS / SEGMENTS is not an operand");
   if (ka == ASTITCH_SCALAR && kb == ASTITCH_SCALAR)
     return fail(ASTITCH_ERR_UNSUPPORTED, "binary op on two SCALARs (fold it on the host)");
   if (ka != kb && ka != ASTITCH_SCALAR && kb != ASTITCH_SCALAR)
@@ -215,7 +266,8 @@ astitch_status astitch_graph_reduce(astitch_graph_t g, astitch_redop op, astitch
     return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad axis");
   if (!valid_value(g->g, a)) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad operand");
   astitch_kind k = g->g.nodes[a].kind;
-  if (k == ASTITCH_LENGTHS) return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS is not an operand");
+  if (k == ASTITCH_LENGTHS || k == ASTITCH_SEGMENTS)
+    return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS / SEGMENTS is not an operand");
   if (k != ASTITCH_FULL)
     return fail(ASTITCH_ERR_UNSUPPORTED,
                 std::string("reduce needs a FULL operand, got ") + kind_name(k));

@@ -46,6 +46,9 @@ struct Graph {
   std::vector<astitch_dtype> output_dtypes;
   int lengths_node = -1;
   int64_t rows_per_segment = 0;
+  int segments_node = -1;                   // packed varlen table (astitch_graph_segments)
+  int nseg = 0;
+  int64_t seg_elems = 0;                    // elements of every FULL tensor when ragged
 };
 
 int dtype_size(astitch_dtype d);

@@ -233,6 +233,21 @@ template <int DT, int E> struct Conv {
   }
 };
 
+// Packed varlen segments (astitch_graph_segments): the entry {row_start, cols,
+// pitch, offset8} of the segment owning `row` = the largest s with
+// row_start_s <= row (row_start increasing; empty segments share a start and
+// the search lands on the last of them, the one whose range holds the row).
+template <int NSEG> __device__ __forceinline__ int4 seg_find(const int4* __restrict__ sg, int row) {
+  int lo = 0, hi = NSEG - 1;
+#pragma unroll 1
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (__ldg(&sg[mid].x) <= row) lo = mid;
+    else hi = mid - 1;
+  }
+  return __ldg(sg + lo);
+}
+
 // scalar (ROWVEC / COLVEC element) load / store with dtype
 template <int DT> __device__ __forceinline__ float ld_scalar(const void* base, long long i) {
   if (DT == 0) return __ldg(reinterpret_cast<const float*>(base) + i);

@@ -104,6 +104,7 @@ void analyse(Plan& p) {
   };
   for (int o : g.outputs) mark(o);
   if (g.lengths_node >= 0) info[g.lengths_node].live = true;
+  if (g.segments_node >= 0) info[g.segments_node].live = true;
 
   // a1: classification
   for (int i = 0; i < n; ++i) {
@@ -152,6 +153,10 @@ void analyse(Plan& p) {
     info[i].post = lv > 0;
     p.max_level = std::max(p.max_level, lv);
   }
+  if (g.segments_node >= 0 && (!p.colreds.empty() || force_global || p.desc.shard_world > 1))
+    throw Error{ASTITCH_ERR_UNSUPPORTED,
+                "packed varlen segments support row-wise subgraphs only (no column reduction, "
+                "FORCE_GLOBAL or sharding)"};
   if (p.max_level > 4)
     throw Error{ASTITCH_ERR_UNSUPPORTED, "more than 4 dependent column reductions (grid barriers)"};
 
@@ -338,7 +343,9 @@ void select_mapping(Plan& p) {
   m.vec_elems = E;
   m.chunks = static_cast<int>((C + E - 1) / E);
   const int chunks = m.chunks;
-  const bool has_mask = g.lengths_node >= 0;
+  // packed varlen rows behave like masked rows of the maximum length
+  const bool ragged = g.segments_node >= 0;
+  const bool has_mask = g.lengths_node >= 0 || ragged;
   const bool has_colred = !p.colreds.empty();
   const int row_bytes_max = static_cast<int>(std::min<int64_t>(C * es_max, 1 << 30));
 
@@ -470,7 +477,7 @@ void select_mapping(Plan& p) {
     // one block per row is still faster (4.2 vs 4.7 us, latency-bound), on
     // <64,300000> (1.2 MB rows) a cluster of 8 is 5x faster; split from 256 KB.
     const bool force_split = (p.desc.flags & ASTITCH_FLAG_FORCE_SPLIT) != 0;
-    bool split_rule = !no_split && R < blocks_per_wave_1024 && C > 1024 &&
+    bool split_rule = !no_split && !ragged && R < blocks_per_wave_1024 && C > 1024 &&
                       (force_split || C * es_max >= 256 * 1024);
     if (packed_ok || team_tile_ok) {
       m.tmpl = Template::PackedTile;
@@ -634,7 +641,10 @@ uint64_t compulsory_bytes(const Plan& p) {
     const Node& nd = g.nodes[id];
     if (!p.info[id].live) continue;
     uint64_t es = dtype_size(nd.dtype);
-    if (nd.kind == ASTITCH_FULL) b += R * C * es;
+    // packed varlen: the whole packed buffer (incl. pitch padding: an upper bound)
+    if (nd.kind == ASTITCH_FULL && g.segments_node >= 0) b += static_cast<uint64_t>(g.seg_elems) * es;
+    else if (nd.kind == ASTITCH_SEGMENTS) b += 16ULL * g.nseg;
+    else if (nd.kind == ASTITCH_FULL) b += R * C * es;
     else if (nd.kind == ASTITCH_ROWVEC) b += R * es;
     else if (nd.kind == ASTITCH_COLVEC) b += C * es;
     else if (nd.kind == ASTITCH_LENGTHS)
@@ -643,7 +653,8 @@ uint64_t compulsory_bytes(const Plan& p) {
   for (size_t k = 0; k < g.outputs.size(); ++k) {
     uint64_t es = dtype_size(g.output_dtypes[k]);
     astitch_kind kd = g.nodes[g.outputs[k]].kind;
-    if (kd == ASTITCH_FULL) b += R * C * es;
+    if (kd == ASTITCH_FULL && g.segments_node >= 0) b += static_cast<uint64_t>(g.seg_elems) * es;
+    else if (kd == ASTITCH_FULL) b += R * C * es;
     else if (kd == ASTITCH_ROWVEC) b += R * es;
     else b += C * es;
   }
@@ -709,6 +720,8 @@ std::string describe_json(const Plan& p) {
   o << ",\"global_fulls\":[";
   for (size_t k = 0; k < p.global_fulls.size(); ++k) o << (k ? "," : "") << p.global_fulls[k];
   o << "],\"needs_sweep2\":" << (p.needs_sweep2 ? "true" : "false");
+  if (g.segments_node >= 0)
+    o << ",\"ragged\":{\"nseg\":" << g.nseg << ",\"elems\":" << g.seg_elems << "}";
   o << ",\"kernel_count\":" << p.kernels.size() << ",\"memsets_per_run\":0";
   o << ",\"kernels\":[";
   for (size_t k = 0; k < p.kernels.size(); ++k) {

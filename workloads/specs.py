@@ -13,8 +13,10 @@ Spec format (all strings upper-case as in the C-ABI enums)::
 
     {
       "name": str, "rows": int, "cols": int,
-      "inputs":  [(name, kind, dtype), ...]        kind in FULL|ROWVEC|COLVEC|LENGTHS
+      "inputs":  [(name, kind, dtype), ...]        kind in FULL|ROWVEC|COLVEC|LENGTHS|SEGMENTS
       "mask":    None | {"lengths": name, "rows_per_segment": int}
+      "segments": (packed varlen only) {"table": name, "batches", "heads", "min_len"}
+                 -> workloads.gen.ragged_spec adds "seg_rows", "seg_cols", "elems"
       "ops":     [(name, "const", value)
                   (name, "unary", UNOP, a)
                   (name, "binary", BINOP, a, b)
@@ -120,6 +122,23 @@ C3_ATTN_SOFTMAX = {
         ("zb", "broadcast", "ROW", "z"),
         ("p", "binary", "DIV", "e", "zb"),
     ],
+    "outputs": [("p", "BF16")],
+}
+
+# C3v: the same attention softmax on the PACKED varlen layout (SURVEY 8(f)
+# f2(ii); the paper's irregular shapes): batch b contributes
+# heads x L_b query rows of L_b keys each, stored back to back with no padding
+# (row pitch = L_b rounded up to 8 elements).  `rows` / the segment lists are
+# filled in by workloads.gen.ragged_spec from the seeded lengths (the same
+# draw as C3's L); cols = the maximum row length.
+C3V_ATTN_SOFTMAX_VARLEN = {
+    "name": "C3v_attention_softmax_varlen_bf16",
+    "rows": None,
+    "cols": 512,
+    "inputs": [("s", "FULL", "BF16"), ("S", "SEGMENTS", "I32")],
+    "mask": None,
+    "segments": {"table": "S", "batches": 64, "heads": 16, "min_len": 37},
+    "ops": [op for op in C3_ATTN_SOFTMAX["ops"]],
     "outputs": [("p", "BF16")],
 }
 
@@ -323,6 +342,7 @@ CONFIGS = {
 }
 
 EXTRA = {
+    "C3v": C3V_ATTN_SOFTMAX_VARLEN,
     "C5int": C5_INT_EXACT,
     "fig5": FIG5_POWER_BCAST_ADD,
     "fig7a": FIG7A_MIXED,
