@@ -867,15 +867,18 @@ struct Gen {
 
   // declaration of the valid bound `lim` of row `row` (active flag `act`); for
   // packed varlen rows also `lim`_b = the row's first chunk in every FULL tensor
-  std::string limdecl(const std::string& lim, const std::string& act, const std::string& row) const {
+  // seg: (ragged) an int4 expression holding the row's table entry already
+  // looked up (the prefetch of the previous iteration), else "" = look it up
+  std::string limdecl(const std::string& lim, const std::string& act, const std::string& row,
+                      const std::string& seg = "") const {
     if (!ragged) {
       if (!masked) return "const int " + lim + " = (int)C;";
       return "const int " + lim + " = " + act + " ? " + lim_expr(row) + " : 0;";
     }
-    return "const int4 " + lim + "_s = " + act + " ? as::seg_find<NSEG>(SG, (int)(" + row +
-           ")) : make_int4(0, 0, 0, 0);\n    const int " + lim + " = min(" + lim + "_s.y, (int)C);\n    const long long " +
-           lim + "_b = ((long long)" + lim + "_s.w * 8 + (long long)((" + row + ") - " + lim + "_s.x) * " + lim +
-           "_s.z) / E; (void)" + lim + "_b;";
+    std::string find = seg.empty() ? act + " ? as::seg_find<NSEG>(SG, (int)(" + row + ")) : make_int4(0, 0, 0, 0)" : seg;
+    return "const int4 " + lim + "_s = " + find + ";\n    const int " + lim + " = min(" + lim +
+           "_s.y, (int)C);\n    const long long " + lim + "_b = ((long long)" + lim + "_s.w * 8 + (long long)((" + row +
+           ") - " + lim + "_s.x) * " + lim + "_s.z) / E; (void)" + lim + "_b;";
   }
   // first chunk of row `row` in a FULL tensor (row-major [R, C] or packed varlen)
   std::string rowbase(const std::string& row, const std::string& lim) const {
@@ -974,8 +977,12 @@ struct Gen {
       for (int u = 0; u < U; ++u) {
         std::string s = su + std::to_string(u) + "n";
         for (size_t q = 0; q < streams.size(); ++q) o << "  " << raw_t(streams[q]) << " r" << q << s << "[V];\n";
+        // (ragged) the segment entry of the prefetched row, reused by the compute step
+        if (ragged) o << "  int4 nsg" << u << " = (prow" << u << " < R) ? as::seg_find<NSEG>(SG, (int)prow" << u
+                      << ") : make_int4(0, 0, 0, 0);\n";
         o << "  {\n    const bool pact = prow" << u << " < R;\n";
-        o << "    " << limdecl("plim", "pact", "prow" + std::to_string(u)) << "\n";
+        o << "    " << limdecl("plim", "pact", "prow" + std::to_string(u), ragged ? "nsg" + std::to_string(u) : "")
+          << "\n";
         o << "    (void)plim;\n";
         emit_loads("prow" + std::to_string(u), "pact", "plim", s, false);
         o << "  }\n";
@@ -986,7 +993,8 @@ struct Gen {
       std::string s = su + std::to_string(u);
       o << "    const " << rt << " row" << u << " = base + " << u << " * RPB + team;\n";
       o << "    const bool act" << u << " = row" << u << " < R;\n";
-      o << "    " << limdecl("lim" + std::to_string(u), "act" + std::to_string(u), "row" + std::to_string(u)) << "\n";
+      o << "    " << limdecl("lim" + std::to_string(u), "act" + std::to_string(u), "row" + std::to_string(u),
+                           (ragged && pf) ? "nsg" + std::to_string(u) : "") << "\n";
       o << "    (void)lim" << u << ";\n";
     }
     if (pf) {
@@ -1002,7 +1010,8 @@ struct Gen {
         o << "    {\n";
         o << "      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
         o << "      const bool pact = nrow < R;\n";
-        o << "      " << limdecl("plim", "pact", "nrow") << "\n";
+        if (ragged) o << "      nsg" << u << " = pact ? as::seg_find<NSEG>(SG, (int)nrow) : make_int4(0, 0, 0, 0);\n";
+        o << "      " << limdecl("plim", "pact", "nrow", ragged ? "nsg" + std::to_string(u) : "") << "\n";
         o << "      (void)plim;\n";
         emit_loads("nrow", "pact", "plim", s, false);
         o << "    }\n";

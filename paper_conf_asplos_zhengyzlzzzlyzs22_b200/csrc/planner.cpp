@@ -564,6 +564,10 @@ void select_mapping(Plan& p) {
       m.threads = m.team > 32 ? m.team : 256;
       m.rows_per_block = m.threads / m.team;
       m.row_unroll = 1;
+      if (const char* fu = getenv("ASTITCH_FORCE_UNROLL")) {  // tuning knob for experiments
+        int u = atoi(fu);
+        if (u >= 1 && u <= 8) m.row_unroll = u;
+      }
       why << "row team of " << m.team << " lanes x " << m.chunks_per_lane << " chunks ("
           << m.rows_per_block << " rows / block, packing), regional via shuffles" << (m.team > 32 ? "+smem" : "")
           << "; ";

@@ -32,6 +32,8 @@ def main():
     from workloads import gen, specs
 
     spec = specs.get(args.config, rows=args.rows, cols=args.cols)
+    if spec.get("segments"):  # packed varlen: seeded segment layout + table
+        spec = gen.ragged_spec(spec, gen.CONFIG_SEEDS.get(args.config, 0))
     R, C = spec["rows"], spec["cols"]
     g = torch.Generator(device="cuda").manual_seed(0)
     tdt = {"F32": torch.float32, "BF16": torch.bfloat16, "F16": torch.float16}
@@ -41,7 +43,12 @@ def main():
             L = gen.lengths_for(spec, gen.CONFIG_SEEDS.get(args.config, 0))
             ins.append(torch.from_numpy(L).cuda())
             continue
-        shape = {"FULL": (R, C), "ROWVEC": (R,), "COLVEC": (C,)}[kind]
+        if kind == "SEGMENTS":
+            t = gen.segment_table(spec["segments"]["seg_rows"], spec["segments"]["seg_cols"])
+            ins.append(torch.from_numpy(t).cuda())
+            continue
+        shape = {"FULL": (spec["segments"]["elems"],) if spec.get("segments") else (R, C),
+                 "ROWVEC": (R,), "COLVEC": (C,)}[kind]
         ins.append(torch.randn(shape, generator=g, device="cuda", dtype=torch.float32).to(tdt[dt]))
     plan = A.Plan(A.Graph.from_spec(spec), R, C, device=0, flags=args.flags)
     outs = plan.alloc_outputs()
