@@ -279,9 +279,7 @@ struct Gen {
         streams.push_back({id, true, ASTITCH_F32, static_cast<long long>(p.ws.globals + gbuf_offset(q))});
     }
   }
-  size_t gbuf_offset(size_t q) const {
-    return q * static_cast<size_t>(p.desc.rows) * static_cast<size_t>(C) * 4;
-  }
+  size_t gbuf_offset(size_t q) const { return p.gbuf_off[q]; }
 
   std::string raw_t(const Stream& s) const { return "as::Raw<" + std::to_string(nb(s.dt)) + ">"; }
 
@@ -937,7 +935,8 @@ struct Gen {
   void emit_sweep(bool post) {
     collect_streams(post);
     emit_stream_ptrs();
-    const bool pf = m.prefetch;
+    // prefetching the next row only pays when a team sweeps more than one row
+    const bool pf = m.prefetch && m.vertical_trips > 1;
     const std::string su = "_u";
     const std::string rt = rowt();
     o << "  const " << rt << " rstride = (" << rt << ")(NUNITS * RPB * " << U << ");\n";

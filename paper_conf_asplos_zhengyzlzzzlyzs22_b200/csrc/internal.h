@@ -148,7 +148,9 @@ struct Plan {
   Mapping map;
   std::vector<int> colreds;      // column reduce node ids (in order)
   std::vector<int> post_colvecs; // COLVEC values computed after the barrier (incl. colreds)
-  std::vector<int> global_fulls; // FULL values buffered in HBM across the barrier
+  std::vector<int> global_fulls; // FULL / ROWVEC values buffered in HBM across a barrier
+  std::vector<size_t> gbuf_off;  // byte offset of each one's buffer within ws.globals (a6 reuse)
+  int gbuf_slots = 0;            // distinct buffers after liveness-based reuse
   bool needs_sweep2 = false;     // FULL / ROWVEC work after the (first) grid barrier
   int max_level = 0;             // grid barriers needed by dependent column reductions
   std::vector<Kernel> kernels;   // kernels launched by astitch_run, in order

@@ -631,7 +631,50 @@ void plan_workspace(Plan& p) {
     w.colvals = off;
     off = align(off + std::max<size_t>(p.post_colvecs.size(), 1) * C * 4 + C * 4 * p.colreds.size());
     w.globals = off;
-    off = align(off + p.global_fulls.size() * static_cast<size_t>(R) * C * 4);
+    // a6 memory reuse: a global buffer is live from the sweep that
+    // writes it to the last sweep that reads it; a later value of the same
+    // kind whose writing sweep starts after that (a grid barrier in between)
+    // takes over the buffer (interval colouring in definition order, the
+    // role of the paper's dominance-tree data-flow analysis).  ROWVEC values
+    // need R floats, FULL values R x C floats.
+    const int n = static_cast<int>(p.g.nodes.size());
+    std::function<int(int)> last_read = [&](int v) {
+      int last = -1;
+      for (int u : p.info[v].consumers) {
+        if (!p.info[u].live) continue;
+        if (p.g.nodes[u].type == NodeType::Bcast) { last = std::max(last, last_read(u)); continue; }
+        int ph = p.info[u].cls == OpClass::ReduceCol ? p.info[p.g.nodes[u].a].level : p.info[u].level;
+        last = std::max(last, ph);
+      }
+      return last;
+    };
+    struct Slot { astitch_kind kind; int free_after; size_t off; };
+    std::vector<Slot> slots;
+    size_t goff = 0;
+    p.gbuf_off.assign(p.global_fulls.size(), 0);
+    std::vector<size_t> order(p.global_fulls.size());
+    std::iota(order.begin(), order.end(), 0);
+    std::stable_sort(order.begin(), order.end(), [&](size_t a, size_t b) {
+      return p.info[p.global_fulls[a]].level < p.info[p.global_fulls[b]].level;
+    });
+    for (size_t q : order) {
+      const int id = p.global_fulls[q];
+      const astitch_kind k = p.g.nodes[id].kind;
+      const int def = p.info[id].level;
+      int chosen = -1;
+      for (size_t s = 0; s < slots.size(); ++s)
+        if (slots[s].kind == k && slots[s].free_after < def) { chosen = static_cast<int>(s); break; }
+      if (chosen < 0) {
+        slots.push_back({k, -1, goff});
+        goff = align(goff + static_cast<size_t>(R) * (k == ASTITCH_FULL ? C : 1) * 4);
+        chosen = static_cast<int>(slots.size()) - 1;
+      }
+      slots[chosen].free_after = last_read(id);
+      p.gbuf_off[q] = slots[chosen].off;
+    }
+    (void)n;
+    p.gbuf_slots = static_cast<int>(slots.size());
+    off = align(off + goff);
   }
   w.total = off;
   p.ws = w;
@@ -723,7 +766,8 @@ std::string describe_json(const Plan& p) {
     << "}";
   o << ",\"global_fulls\":[";
   for (size_t k = 0; k < p.global_fulls.size(); ++k) o << (k ? "," : "") << p.global_fulls[k];
-  o << "],\"needs_sweep2\":" << (p.needs_sweep2 ? "true" : "false");
+  o << "],\"global_buffers\":" << p.gbuf_slots;
+  o << ",\"needs_sweep2\":" << (p.needs_sweep2 ? "true" : "false");
   if (g.segments_node >= 0)
     o << ",\"ragged\":{\"nseg\":" << g.nseg << ",\"elems\":" << g.seg_elems << "}";
   o << ",\"kernel_count\":" << p.kernels.size() << ",\"memsets_per_run\":0";

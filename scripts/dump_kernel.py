@@ -22,6 +22,9 @@ def main():
     import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
     from workloads import specs
     s = specs.get(a.config, rows=a.rows, cols=a.cols)
+    if s.get("segments"):
+        from workloads import gen
+        s = gen.ragged_spec(s, gen.CONFIG_SEEDS.get(a.config, 0))
     p = A.Plan(A.Graph.from_spec(s), s["rows"], s["cols"], device=-1, flags=a.flags)
     os.makedirs(a.outdir, exist_ok=True)
     base = os.path.join(a.outdir, f"{a.config}_f{a.flags}")

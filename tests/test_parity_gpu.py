@@ -164,6 +164,18 @@ def test_parity_force_global_ablation(cfg, rows, cols):
     _compare(spec, got, evaluate(spec, x))
 
 
+def test_parity_force_global_buffer_reuse():
+    """Four grid barriers and reused HBM buffers (double softmax, FORCE_GLOBAL)."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from tests.test_planner import DOUBLE_SOFTMAX
+    spec = dict(DOUBLE_SOFTMAX)
+    x = {"x": gen.generate("C1", specs.get("C1", rows=1000, cols=200))["x"]}
+    got, plan = run_gpu(spec, x, return_plan=True, flags=A.FLAG_FORCE_GLOBAL)
+    assert plan.describe()["global_buffers"] == 4
+    _compare(spec, got, evaluate(spec, x))
+    _compare(spec, run_gpu(spec, x), evaluate(spec, x))    # default (regional) plan
+
+
 @pytest.mark.parametrize("cfg,rows,cols,world", [("C5", 3001, 1024, 2), ("C5", 4099, 256, 8), ("fig7a", 1001, 96, 3),
                                                  ("C5int", 4096, 128, 4), ("C2", 777, 768, 4), ("C3", 4 * 512, 512, 4)])
 def test_virtual_shards(cfg, rows, cols, world):

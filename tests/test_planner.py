@@ -170,6 +170,35 @@ def test_force_global_ablation_demotes_row_reductions():
         describe("C1", flags=A.FLAG_NO_COMPILE | A.FLAG_FORCE_GLOBAL, shard_rank=0, shard_world=2)
 
 
+DOUBLE_SOFTMAX = {
+    "name": "double_softmax", "rows": 1000, "cols": 200,
+    "inputs": [("x", "FULL", "F32")], "mask": None,
+    "ops": [("m1", "reduce", "RMAX", "ROW", "x"), ("m1b", "broadcast", "ROW", "m1"),
+            ("d1", "binary", "SUB", "x", "m1b"), ("e1", "unary", "EXP", "d1"),
+            ("s1", "reduce", "SUM", "ROW", "e1"), ("s1b", "broadcast", "ROW", "s1"),
+            ("y1", "binary", "DIV", "e1", "s1b"),
+            ("m2", "reduce", "RMAX", "ROW", "y1"), ("m2b", "broadcast", "ROW", "m2"),
+            ("d2", "binary", "SUB", "y1", "m2b"), ("e2", "unary", "EXP", "d2"),
+            ("s2", "reduce", "SUM", "ROW", "e2"), ("s2b", "broadcast", "ROW", "s2"),
+            ("y2", "binary", "DIV", "e2", "s2b")],
+    "outputs": [("y2", "F32")],
+}
+
+
+def test_global_buffer_reuse_by_liveness():
+    """a6 memory reuse: FORCE_GLOBAL double softmax buffers m1, e1, s1,
+    y1, m2, e2, s2 in HBM across 4 barriers; a buffer whose last reader is an
+    earlier sweep is taken over (m2 <- m1, e2 <- e1, s2 <- s1): 4 buffers, not 7."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A2
+    g = A2.Graph.from_spec(DOUBLE_SOFTMAX)
+    p = A2.Plan(g, 1000, 200, device=-1, flags=A.FLAG_NO_COMPILE | A.FLAG_FORCE_GLOBAL)
+    d = p.describe()
+    assert len(d["global_fulls"]) == 7 and d["global_buffers"] == 4
+    assert p.source(0).count("as::grid_barrier(bar);") == 4
+    # FULL buffers hold R x C floats, ROWVEC buffers R floats
+    assert d["workspace"]["total"] - d["workspace"]["globals"] <= (2 * 1000 * 200 + 2 * 1000) * 4 + 4 * 256
+
+
 def test_no_pack_ablation():
     d, _, _ = describe("fig6a", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_PACK)
     assert d["mapping"]["team"] == 32
