@@ -54,6 +54,18 @@ struct Gen {
     compute_absorb();
   }
   bool split = false;
+  // chunk-count specialisation of masked rows: inside a `switch` on the
+  // row's number of fully valid team chunks KF (a compile-time constant in
+  // each case), chunk predicates fold at compile time, chunks past the
+  // boundary chunk vanish, and row reductions cover only NEV elements
+  bool kf = false;
+  std::string full_pred(const std::string& lim) const {
+    return kf ? "(j < KF)" : "((j + 1) * T * E <= " + lim + ")";
+  }
+  std::string live_pred(const std::string& lim) const {
+    return kf ? "(j <= KF)" : "(j * T * E < " + lim + ")";
+  }
+  std::string nev() const { return kf ? "NEV" : "NE"; }
   int rowred_index(int node) const {  // ordinal of a row reduction (cluster slot)
     int k = 0;
     for (int i = 0; i < node; ++i)
@@ -327,8 +339,8 @@ struct Gen {
       if (absorb && masked && !st.ws_buf && !lim.empty()) {
         // mask absorption: invalid elements take the substitute value
         // d_ = elements of this lane's chunk that are valid (may be <= 0)
-        o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n      if (!((j + 1) * T * E <= " << lim
-          << ")) {\n        const int d_ = " << lim << " - (j * T + lane) * E;\n#pragma unroll\n"
+        o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n      if (!" << full_pred(lim)
+          << ") {\n        const int d_ = " << lim << " - (j * T + lane) * E;\n#pragma unroll\n"
           << "        for (int e = 0; e < E; ++e) if (e >= d_) " << dst << "[j * E + e] = " << fconst(absorb_sub)
           << ";\n      }\n    }\n";
       }
@@ -489,7 +501,7 @@ struct Gen {
         if (check && !absorb) o << "(" << col_expr("(k / E)", "(k % E)") << " < " << lim << ") ? " << ref(nd.a, "k", sfx)
                      << " : 0.f;\n";
         else o << ref(nd.a, "k", sfx) << ";\n";
-        o << "      double r_ = as::TreeD<NE>::reduce(t_);\n";
+        o << "      double r_ = as::TreeD<" << nev() << ">::reduce(t_);\n";
         if (T <= 32) o << "      r_ = as::team_sum_d<T>(r_);\n";
         else if (split)
           o << "      r_ = as::cluster_team_sum_d<" << m.threads << ", " << m.split << ">(r_, red_scratch_d, &cl_slot_d["
@@ -523,7 +535,7 @@ struct Gen {
           // [j*T*E, (j+1)*T*E) across the team, so "fully valid" is uniform
           // over the team and only the boundary chunk pays per-element selects
           o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
-          o << "        if ((j + 1) * T * E <= " << lim << ") {\n#pragma unroll\n          for (int e = 0; e < E; ++e) { const int k = j * E + e; t_[k] = " << ref(src, "k", sfx) << "; }\n";
+          o << "        if (" << full_pred(lim) << ") {\n#pragma unroll\n          for (int e = 0; e < E; ++e) { const int k = j * E + e; t_[k] = " << ref(src, "k", sfx) << "; }\n";
           o << "        } else {\n#pragma unroll\n          for (int e = 0; e < E; ++e) { const int k = j * E + e; t_[k] = ("
             << col_expr("j", "e") << " < " << lim << ") ? " << ref(src, "k", sfx) << " : " << ident << "; }\n        }\n      }\n";
         } else {
@@ -532,7 +544,7 @@ struct Gen {
                        << " : " << ident << ";\n";
           else o << ref(src, "k", sfx) << ";\n";
         }
-        o << "      float r_ = as::Tree<NE, " << (mx ? "true" : "false") << ">::reduce(t_);\n";
+        o << "      float r_ = as::Tree<" << nev() << ", " << (mx ? "true" : "false") << ">::reduce(t_);\n";
         if (T <= 32) o << "      r_ = as::team_" << (mx ? "max" : "sum") << "<T>(r_);\n";
         else if (split)
           o << "      r_ = as::cluster_team_reduce<" << m.threads << ", " << m.split << ", " << (mx ? "true" : "false")
@@ -571,7 +583,7 @@ struct Gen {
         o << "    float v" << id << sfx << "[NE];\n";
         if (masked) {
           // chunks wholly past the valid length are not computed (team-uniform branch)
-          o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n      if (j * T * E < " << lim << ") {\n";
+          o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n      if (" << live_pred(lim) << ") {\n";
           o << "#pragma unroll\n        for (int e = 0; e < E; " << estep << ") { const int k = j * E + e; " << body
             << " }\n";
           std::string skip = (absorb && inval_known[i]) ? fconst(inval[i]) : "0.f";
@@ -824,13 +836,13 @@ struct Gen {
         std::string val = ref(id, "(j * E + e)", sfx);
         o << "        float t_[E];\n";
         if (masked) {
-          o << "        if ((j + 1) * T * E <= " << lim << ") {\n#pragma unroll\n          for (int e = 0; e < E; ++e) t_[e] = "
+          o << "        if (" << full_pred(lim) << ") {\n#pragma unroll\n          for (int e = 0; e < E; ++e) t_[e] = "
             << val << ";\n        } else {\n#pragma unroll\n          for (int e = 0; e < E; ++e) t_[e] = ("
             << col_expr("j", "e") << " < " << lim << ") ? " << val << " : 0.f;\n        }\n";
         } else {
           o << "#pragma unroll\n        for (int e = 0; e < E; ++e) t_[e] = " << val << ";\n";
         }
-        if (ragged) o << "        if ((j * T + lane) * E < " << lim << ")  // chunks of the row only (packed)\n";
+        if (ragged) o << "        if (" << live_pred(lim) << " && (j * T + lane) * E < " << lim << ")  // chunks of the row only (packed)\n";
         else if (!exact) o << "        if ((long long)(j * T + lane) < CH)\n";
         o << "        as::stg(op_ + (j * T + lane), as::Conv<" << dt_code(dt) << ", E>::pack(t_));\n";
         o << "      }\n    }\n";
@@ -1024,6 +1036,22 @@ struct Gen {
     for (int u = 0; u < U; ++u) {
       std::string s = su + std::to_string(u);
       std::string row = "row" + std::to_string(u), act = "act" + std::to_string(u), lim = "lim" + std::to_string(u);
+      emit_row_block(post, s, row, act, lim);
+    }
+    o << "  }\n";
+  }
+
+  // one row's compute (unpack, ops, stores).  Packed varlen row teams
+  // specialise it on KF = the number of fully valid team chunks (0..V), a
+  // warp-uniform switch for rows of one segment: per-chunk mask tests fold at
+  // compile time and chunks past the valid prefix cost nothing (measured on
+  // B200: C3v 81 vs 95 us; the padded C3 rows gain nothing: stores of the
+  // whole padded row dominate, and the 5x code loses 1-4%).
+  void emit_row_block(bool post, const std::string& s, const std::string& row, const std::string& act,
+                      const std::string& lim) {
+    const bool spec = ragged && m.tmpl == Template::RowTeam && V >= 2 && !split &&
+                      !(getenv("ASTITCH_NO_KF") && atoi(getenv("ASTITCH_NO_KF")) == 1);
+    if (!spec) {
       o << "    {\n";
       emit_unpack(s, lim);
       emit_colvecs(true);
@@ -1031,8 +1059,22 @@ struct Gen {
       emit_body(post, s, row, act, lim);
       emit_stores(post, s, row, act, lim);
       o << "    }\n";
+      return;
     }
-    o << "  }\n";
+    o << "    switch (min(" << lim << " / (T * E), V)) {\n";
+    kf = true;
+    for (int k = 0; k <= V; ++k) {
+      o << (k == V ? "    default" : "    case " + std::to_string(k)) << ": {\n";
+      o << "    constexpr int KF = " << k << ", NEV = " << std::min(k + 1, V) << " * E; (void)KF; (void)NEV;\n";
+      emit_unpack(s, lim);
+      emit_colvecs(true);
+      emit_rowvec_inputs(post, s, row, act);
+      emit_body(post, s, row, act, lim);
+      emit_stores(post, s, row, act, lim);
+      o << "    } break;\n";
+    }
+    kf = false;
+    o << "    }\n";
   }
 
   // ------------------------------------------------------------ global pieces

@@ -426,7 +426,10 @@ void select_mapping(Plan& p) {
     // chunk-uniform mask branches skip whole chunks past the valid length, so
     // a finer chunk (smaller team, more chunks per lane) wastes less work on
     // padding; it also puts several rows of one segment (same length) in a warp.
-    choose_team(1024, has_mask ? 32 : 16, 32);
+    // Packed varlen rows (measured on B200, C3v): T=8 x 8 chunks of 8 bf16 +
+    // the KF chunk-count specialisation (codegen) 81 us vs 95 us at T=16;
+    // padded masked rows (C3) are store-bound and keep T=16 without it.
+    choose_team(1024, ragged ? 64 : (has_mask ? 32 : 16), ragged ? 64 : 32);
     if (const char* ft = getenv("ASTITCH_FORCE_TEAM")) {  // tuning knob for experiments
       int t = atoi(ft);
       if (t >= 1 && t <= 1024 && ((t & (t - 1)) == 0 || t % 32 == 0)) {

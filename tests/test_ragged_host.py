@@ -94,10 +94,10 @@ def test_planner_ragged_row_team_and_describe():
     assert sv["rows"] == 16 * sum(sv["segments"]["seg_cols"])
     p = _plan(sv)
     d = p.describe()
-    assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 16
+    assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 8
     assert d["ragged"] == {"nseg": 64, "elems": sv["segments"]["elems"]}
     src = p.source(0)
-    assert "as::seg_find<NSEG>(SG" in src
+    assert "as::seg_find<NSEG>(SG" in src and "constexpr int KF = " in src
     assert "// chunks of the row only (packed)" in src     # no writes past a row
     assert "= (-AS_INF);" in src                            # mask absorption still applies
     assert p.io_shape("FULL") == (sv["segments"]["elems"],)
