@@ -565,6 +565,10 @@ void select_mapping(Plan& p) {
       m.tmpl = Template::RowTeam;
       // a multi-warp team reduces through block-wide smem: one team per block
       m.threads = m.team > 32 ? m.team : 256;
+      if (const char* ft = getenv("ASTITCH_FORCE_THREADS")) {  // tuning knob for experiments
+        int t = atoi(ft);
+        if (t >= m.team && t <= 1024 && t % m.team == 0 && t % 32 == 0) m.threads = t;
+      }
       m.rows_per_block = m.threads / m.team;
       m.row_unroll = 1;
       if (const char* fu = getenv("ASTITCH_FORCE_UNROLL")) {  // tuning knob for experiments
@@ -583,6 +587,7 @@ void select_mapping(Plan& p) {
     for (int i = 0; i < static_cast<int>(g.nodes.size()); ++i)
       if (p.info[i].live && !p.info[i].post && g.nodes[i].kind == ASTITCH_COLVEC) ++ncv;
     m.hoist_colvec = (ncv * m.chunks_per_lane * E) <= 48;
+    if (const char* fh = getenv("ASTITCH_HOIST")) m.hoist_colvec = atoi(fh) == 1;  // tuning knob
   }
 
   // a7: assume-relax-apply.  Assume the 32-register bound (full occupancy),
@@ -592,6 +597,10 @@ void select_mapping(Plan& p) {
   int by_threads = 2048 / m.threads;
   int by_smem = m.smem_bytes > 0 ? (228 * 1024) / (m.smem_bytes + 1024) : 32;
   m.blocks_per_sm = std::max(1, std::min({32, by_threads, by_smem}));
+  if (const char* fb = getenv("ASTITCH_FORCE_BPS")) {  // tuning knob: fixed occupancy target
+    int b = atoi(fb);
+    if (b >= 1 && b <= 32) m.blocks_per_sm = b;
+  }
   m.reg_cap = std::min(255, (65536 / (m.blocks_per_sm * m.threads)) & ~7);
 
   m.reason = why.str();

@@ -104,7 +104,7 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     if (!compile) return ASTITCH_OK;
     astitch_status st = compile_and_inspect(p, k, load);
     if (st != ASTITCH_OK) return st;
-    if (!may_relax) return ASTITCH_OK;
+    if (!may_relax || getenv("ASTITCH_FORCE_BPS")) return ASTITCH_OK;
     const int cur = p.map.blocks_per_sm;
     if (k.spill_bytes > 0 && cur == 1 && p.map.row_unroll > 1) {
       // even one block per SM spills: fewer rows in flight per team

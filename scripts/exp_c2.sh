@@ -1,7 +1,10 @@
 #!/bin/bash
-# C2 latency experiment: templates / teams / prefetch
-b() { timeout 120 python bench.py --config C2 --no-cpu-baseline "$@" > /tmp/o.json 2>/tmp/e.txt; python -c "import json; d=json.load(open('/tmp/o.json')); print('C2', '$*', '${ASTITCH_FORCE_TEAM}', d['value'], d['us_per_subgraph'], d['config']['template'], 'regs', d['config']['regs'], 'grid', d['config']['grid'])" 2>/dev/null || (echo "fail $*"; tail -2 /tmp/e.txt); }
-b; b --flags 32; b --flags 96
-ASTITCH_FORCE_TEAM=96 b --flags 32; ASTITCH_FORCE_TEAM=96 b --flags 96
-ASTITCH_FORCE_TEAM=64 b --flags 32; ASTITCH_FORCE_TEAM=64 b --flags 96
-ASTITCH_FORCE_TEAM=16 b --flags 96
+# C2 latency experiments: block size x occupancy target x colvec hoisting
+bash scripts/bench_brief.sh C2 --no-e2e
+for cfg in "128 4 0" "128 7 0" "128 8 0" "256 4 0" "128 7 1" "256 3 1"; do
+  set -- $cfg
+  echo -n "th=$1 bps=$2 hoist=$3  "
+  ASTITCH_FORCE_THREADS=$1 ASTITCH_FORCE_BPS=$2 ASTITCH_HOIST=$3 bash scripts/bench_brief.sh C2 --no-e2e
+done
+echo -n "T=16 "; ASTITCH_FORCE_TEAM=16 bash scripts/bench_brief.sh C2 --no-e2e
+echo -n "T=16 bps4 "; ASTITCH_FORCE_TEAM=16 ASTITCH_FORCE_BPS=4 bash scripts/bench_brief.sh C2 --no-e2e
