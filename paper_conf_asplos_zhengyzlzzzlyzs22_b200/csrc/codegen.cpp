@@ -49,7 +49,7 @@ struct Gen {
     ragged = g.segments_node >= 0;
     masked = g.lengths_node >= 0 || ragged;  // varlen rows: masks of the row's own length
     exact = (static_cast<long long>(T) * V * E == C);
-    split = (m.tmpl == Template::SplitRow);
+    split = (m.tmpl == Template::SplitRow) || (m.tmpl == Template::RowStream && m.split > 1);
     compute_precise();
     compute_absorb();
   }
@@ -203,8 +203,10 @@ struct Gen {
   }
 
   std::string col_expr(const std::string& j, const std::string& e) const {
+    if (!tile_off.empty()) return "((" + j + " * T + lane) * E + " + e + " + " + tile_off + ")";
     return "((" + j + " * T + lane) * E + " + e + ")";
   }
+  std::string tile_off;  // row_stream: column offset of the current tile ("" otherwise)
 
   // hoisted COLVEC values (pre-barrier): inputs and EW on them
   // in_loop: called inside the row loop (COLVEC operands re-read through L1
@@ -221,7 +223,7 @@ struct Gen {
         // chunk loads through L1 (the vector is re-read by every row team)
         std::string rt = "as::Raw<" + std::to_string(nb(nd.dtype)) + ">";
         o << "#pragma unroll\n  for (int j = 0; j < V; ++j) {\n";
-        o << "    const long long ch = (long long)j * T + lane;\n";
+        o << "    const long long ch = (long long)j * T + lane" << (tile_off.empty() ? "" : " + " + tile_off + " / E") << ";\n";
         o << "    const " << rt << " rc_ = (ch < CH) ? as::ldg_l1((const " << rt << "*)p.in[" << nd.input_index
           << "] + ch) : " << rt << "{};\n";
         o << "    as::Conv<" << dt_code(nd.dtype) << ", E>::unpack(rc_, c" << i << " + j * E);\n  }\n";
@@ -1394,10 +1396,229 @@ struct Gen {
     o << "}\n";
   }
 
+  // ------------------------------------------------------------ row stream
+  // Rows longer than the team's registers (planner: RowStream).  A team (a
+  // block, or a cluster when rows are few) owns a row and walks it in column
+  // tiles of T lanes x V chunks.  Row-local levels: rl(v) = number of row
+  // reductions on v's dependency path.  Pass p re-reads the tile's inputs,
+  // recomputes the FULL values of levels <= p, accumulates the row reductions
+  // of level p (per-lane fp32 / fp64 accumulators in tile order, then one
+  // team reduction) and stores the FULL outputs of level p; the row scalars
+  // of level p+1 are then computed in registers.  Deterministic (fixed tile
+  // order and trees).
+  std::vector<int> rl;
+  void compute_row_levels() {
+    const int n = static_cast<int>(g.nodes.size());
+    rl.assign(n, 0);
+    for (int i = 0; i < n; ++i) {
+      const Node& nd = N(i);
+      int lv = 0;
+      for (int a : {nd.a, nd.b}) {
+        if (a < 0) continue;
+        lv = std::max(lv, rl[a] + (I(a).cls == OpClass::ReduceRow ? 1 : 0));
+      }
+      rl[i] = lv;
+    }
+  }
+  // ROWVEC value i (not an input) computed from row scalars
+  void emit_stream_rowvec(int i) {
+    const Node& nd = N(i);
+    std::string id = std::to_string(i);
+    if (precise[i]) {
+      o << "    const double d" << id << " = ";
+      if (nd.type == NodeType::Unary) o << (nd.sub == ASTITCH_NEG ? "-" : "fabs") << "(" << dref(nd.a, "") << ");\n";
+      else o << dbinop(nd.sub, nd.a, nd.b, "") << ";\n";
+      emit_split(id, "");
+      return;
+    }
+    if (nd.type == NodeType::Unary) o << "    const float s" << id << " = " << unop(nd.sub, sref(nd.a, "")) << ";\n";
+    else o << "    const float s" << id << " = " << binop(nd.sub, nd.b, sref(nd.a, ""), sref(nd.b, "")) << ";\n";
+  }
+  void emit_stream_rowvec_output(int i) {
+    for (size_t k = 0; k < g.outputs.size(); ++k)
+      if (g.outputs[k] == i)
+        o << "    if (lane == 0) as::st_scalar<" << dt_code(g.output_dtypes[k]) << ">(p.out[" << k << "], row, s"
+          << i << ");\n";
+  }
+  void emit_stream(const std::string& name) {
+    header(name, false);
+    compute_row_levels();
+    const int n = static_cast<int>(g.nodes.size());
+    int P = 1;
+    for (int i = 0; i < n; ++i)
+      if (I(i).live && N(i).kind == ASTITCH_FULL && N(i).type != NodeType::Bcast) P = std::max(P, rl[i] + 1);
+    std::vector<int> fin;  // live FULL inputs
+    for (int id : g.inputs)
+      if (N(id).kind == ASTITCH_FULL && I(id).live) fin.push_back(id);
+    for (size_t s = 0; s < fin.size(); ++s) {
+      std::string rt = "as::Raw<" + std::to_string(nb(N(fin[s]).dtype)) + ">";
+      o << "  const " << rt << "* __restrict__ gs" << s << " = (const " << rt << "*)p.in[" << N(fin[s]).input_index
+        << "];\n";
+    }
+    emit_pre_colvec_outputs();
+    o << "  constexpr long long TCH = (long long)T * V;            // chunks per tile\n";
+    o << "  constexpr long long NT = (CH + TCH - 1) / TCH;          // tiles per row\n";
+    o << "  for (long long row = UNIT; row < (long long)R; row += NUNITS) {\n";
+    // ROWVEC inputs and level-0 row scalars
+    for (int id : g.inputs)
+      if (N(id).kind == ASTITCH_ROWVEC && I(id).live)
+        o << "    const float s" << id << " = as::ld_scalar<" << dt_code(N(id).dtype) << ">(p.in[" << N(id).input_index
+          << "], row);\n";
+    for (int i = 0; i < n; ++i)
+      if (I(i).live && N(i).kind == ASTITCH_ROWVEC && rl[i] == 0 && N(i).type != NodeType::Input &&
+          N(i).type != NodeType::Reduce)
+        emit_stream_rowvec(i);
+    for (int i = 0; i < n; ++i)
+      if (I(i).live && N(i).kind == ASTITCH_ROWVEC && rl[i] == 0 && N(i).type != NodeType::Reduce)
+        emit_stream_rowvec_output(i);
+    for (int pass = 0; pass < P; ++pass) {
+      // what this pass needs: its reductions' operands and its FULL outputs,
+      // closed backwards over FULL values (row / column scalars are at hand)
+      std::vector<bool> need(n, false);
+      std::vector<int> reds;
+      for (int i = 0; i < n; ++i) {
+        if (!I(i).live) continue;
+        if (I(i).cls == OpClass::ReduceRow && rl[i] == pass) { reds.push_back(i); need[N(i).a] = true; }
+      }
+      std::vector<int> fouts;
+      for (size_t k = 0; k < g.outputs.size(); ++k) {
+        int id = g.outputs[k];
+        if (N(id).kind == ASTITCH_FULL && rl[id] == pass) { need[id] = true; fouts.push_back(static_cast<int>(k)); }
+      }
+      std::vector<bool> need_cv(n, false);
+      for (int i = n - 1; i >= 0; --i) {
+        if (!need[i]) continue;
+        const Node& nd = N(i);
+        if (nd.type == NodeType::Bcast) {
+          if (nd.axis == ASTITCH_AXIS_COL) need_cv[nd.a] = true;
+          continue;
+        }
+        for (int a : {nd.a, nd.b}) {
+          if (a < 0) continue;
+          if (N(a).kind == ASTITCH_FULL) need[a] = true;
+          else if (N(a).kind == ASTITCH_COLVEC) need_cv[a] = true;
+        }
+      }
+      for (int i = n - 1; i >= 0; --i)  // COLVEC closure
+        if (need_cv[i])
+          for (int a : {N(i).a, N(i).b})
+            if (a >= 0 && N(a).kind == ASTITCH_COLVEC) need_cv[a] = true;
+      o << "    // ---- pass " << pass << ": " << reds.size() << " row reduction(s), " << fouts.size()
+        << " FULL output(s)\n";
+      for (int r : reds) {
+        if (precise[r]) o << "    double ad" << r << " = 0.0;\n";
+        else o << "    float a" << r << " = " << (N(r).sub == ASTITCH_RMAX ? "-AS_INF" : "0.f") << ";\n";
+      }
+      o << "    for (long long t = 0; t < NT; ++t) {\n";
+      o << "      const long long TOFF = t * TCH * E;  // first column of the tile\n";
+      tile_off = "TOFF";
+      for (size_t s = 0; s < fin.size(); ++s) {
+        int id = fin[s];
+        if (!need[id]) continue;
+        std::string rt = "as::Raw<" + std::to_string(nb(N(id).dtype)) + ">";
+        o << "      " << rt << " r" << s << "[V];\n";
+        o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
+        o << "        const long long ch = t * TCH + j * T + lane;\n";
+        o << "        r" << s << "[j] = (ch < CH) ? as::ldg(gs" << s << " + row * CH + ch) : " << rt << "{};\n";
+        o << "      }\n";
+        o << "      float v" << id << "[NE];\n";
+        o << "#pragma unroll\n      for (int j = 0; j < V; ++j) as::Conv<" << dt_code(N(id).dtype) << ", E>::unpack(r" << s
+          << "[j], v" << id << " + j * E);\n";
+      }
+      // COLVEC operands of the tile (inputs through L1, EW on them)
+      for (int i = 0; i < n; ++i) {
+        if (!need_cv[i] || !I(i).live) continue;
+        const Node& nd = N(i);
+        o << "      float c" << i << "[NE];\n";
+        if (nd.type == NodeType::Input) {
+          std::string rt = "as::Raw<" + std::to_string(nb(nd.dtype)) + ">";
+          o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
+          o << "        const long long ch = t * TCH + j * T + lane;\n";
+          o << "        const " << rt << " rc_ = (ch < CH) ? as::ldg_l1((const " << rt << "*)p.in[" << nd.input_index
+            << "] + ch) : " << rt << "{};\n";
+          o << "        as::Conv<" << dt_code(nd.dtype) << ", E>::unpack(rc_, c" << i << " + j * E);\n      }\n";
+        } else {
+          o << "#pragma unroll\n      for (int k = 0; k < NE; ++k) c" << i << "[k] = ";
+          if (nd.type == NodeType::Unary) o << unop(nd.sub, ref(nd.a, "k", "")) << ";\n";
+          else o << binop(nd.sub, nd.b, ref(nd.a, "k", ""), ref(nd.b, "k", "")) << ";\n";
+        }
+      }
+      // FULL values of levels <= pass (recomputed)
+      for (int i = 0; i < n; ++i) {
+        const Node& nd = N(i);
+        if (!need[i] || !I(i).live || nd.kind != ASTITCH_FULL || nd.type == NodeType::Input ||
+            nd.type == NodeType::Bcast)
+          continue;
+        o << "      float v" << i << "[NE];\n";
+        o << "#pragma unroll\n      for (int k = 0; k < NE; ++k) v" << i << "[k] = " << full_expr(i, "") << ";\n";
+      }
+      // row reductions of this level: per-lane accumulation in tile order
+      const bool tail = (C % (static_cast<long long>(m.team) * V * E)) != 0;
+      for (int r : reds) {
+        bool mx = N(r).sub == ASTITCH_RMAX;
+        std::string ident = mx ? "-AS_INF" : "0.f";
+        o << "      {\n        float t_[NE];\n#pragma unroll\n        for (int k = 0; k < NE; ++k) t_[k] = ";
+        if (tail) o << "(" << col_expr("(k / E)", "(k % E)") << " < C) ? " << ref(N(r).a, "k", "") << " : " << ident << ";\n";
+        else o << ref(N(r).a, "k", "") << ";\n";
+        if (precise[r]) o << "        ad" << r << " += as::TreeD<NE>::reduce(t_);\n";
+        else if (mx) o << "        a" << r << " = fmaxf(a" << r << ", as::Tree<NE, true>::reduce(t_));\n";
+        else o << "        a" << r << " += as::Tree<NE, false>::reduce(t_);\n";
+        o << "      }\n";
+      }
+      // FULL outputs of this level
+      for (int k : fouts) {
+        int id = g.outputs[k];
+        astitch_dtype dt = g.output_dtypes[k];
+        std::string rt = "as::Raw<" + std::to_string(nb(dt)) + ">";
+        o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
+        o << "        const long long ch = t * TCH + j * T + lane;\n";
+        o << "        float t_[E];\n#pragma unroll\n        for (int e = 0; e < E; ++e) t_[e] = " << ref(id, "(j * E + e)", "")
+          << ";\n";
+        o << "        if (ch < CH) as::stg((" << rt << "*)p.out[" << k << "] + row * CH + ch, as::Conv<" << dt_code(dt)
+          << ", E>::pack(t_));\n      }\n";
+      }
+      tile_off.clear();
+      o << "    }\n";
+      // team reductions -> row scalars of level pass+1
+      for (int r : reds) {
+        bool mx = N(r).sub == ASTITCH_RMAX;
+        std::string id = std::to_string(r);
+        if (precise[r]) {
+          o << "    double d" << id << ";\n    {\n      double r_ = ad" << id << ";\n";
+          if (split)
+            o << "      r_ = as::cluster_team_sum_d<" << m.threads << ", " << m.split << ">(r_, red_scratch_d, &cl_slot_d["
+              << rowred_index(r) << "]);\n";
+          else o << "      r_ = as::block_team_sum_d<T>(r_, red_scratch_d);\n";
+          o << "      d" << id << " = r_;\n    }\n";
+          emit_split(id, "");
+        } else {
+          o << "    float s" << id << ";\n    {\n      float r_ = a" << id << ";\n";
+          if (split)
+            o << "      r_ = as::cluster_team_reduce<" << m.threads << ", " << m.split << ", " << (mx ? "true" : "false")
+              << ">(r_, red_scratch, &cl_slot[" << rowred_index(r) << "]);\n";
+          else o << "      r_ = as::block_team_reduce<T, " << (mx ? "true" : "false") << ">(r_, red_scratch);\n";
+          o << "      s" << id << " = r_;\n    }\n";
+        }
+        emit_stream_rowvec_output(r);
+      }
+      for (int i = 0; i < n; ++i)
+        if (I(i).live && N(i).kind == ASTITCH_ROWVEC && rl[i] == pass + 1 && N(i).type != NodeType::Reduce &&
+            N(i).type != NodeType::Input) {
+          emit_stream_rowvec(i);
+          emit_stream_rowvec_output(i);
+        }
+    }
+    o << "  }\n}\n";
+  }
+
   // ------------------------------------------------------------ roles
   std::string run(const std::string& name) {
     if (m.tmpl == Template::PackedTile) {
       emit_packed(name);
+      return o.str();
+    }
+    if (m.tmpl == Template::RowStream) {
+      emit_stream(name);
       return o.str();
     }
     if (role == ROLE_SHARD_FINAL) {

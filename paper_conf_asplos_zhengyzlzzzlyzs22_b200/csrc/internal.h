@@ -85,7 +85,8 @@ enum class Template {
   RowTeam,     // row-reduce / EW: a team of lanes per row, registers + shuffles (regional)
   PackedTile,  // many tiny rows: TMA-bulk tiles in smem, thread per row (horizontal packing)
   GlobalSweep, // column reduce: vertical packing + block partials + grid barrier (global)
-  SplitRow     // few long rows: row split over a thread-block cluster (task splitting)
+  SplitRow,    // few long rows: row split over a thread-block cluster (task splitting)
+  RowStream    // rows longer than a team's registers: column tiles, one pass per row-reduction level
 };
 const char* template_name(Template t);
 

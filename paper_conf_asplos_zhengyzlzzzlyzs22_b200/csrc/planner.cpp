@@ -54,6 +54,7 @@ const char* template_name(Template t) {
     case Template::PackedTile: return "packed_tile";
     case Template::GlobalSweep: return "global_sweep";
     case Template::SplitRow: return "split_row";
+    case Template::RowStream: return "row_stream";
   }
   return "?";
 }
@@ -579,6 +580,38 @@ void select_mapping(Plan& p) {
           << m.rows_per_block << " rows / block, packing), regional via shuffles" << (m.team > 32 ? "+smem" : "")
           << "; ";
     }
+    // Rows longer than the team's registers (more than kStreamNE fp32 values
+    // per lane even with the largest team / cluster): stream the row in
+    // column tiles, one pass over the row per level of dependent row
+    // reductions (FULL values of lower levels are recomputed from the
+    // re-read inputs, L2-resident for a row in flight), the regional values
+    // (row scalars) stay in registers.  The paper's answer to a regional
+    // buffer over the on-chip limit is demotion to global; a
+    // per-row re-read keeps it in one pass of the grid with no barrier.
+    constexpr int kStreamNE = 128;
+    const bool stream_ok = !has_mask && p.global_fulls.empty() &&
+                           (m.tmpl == Template::RowTeam || m.tmpl == Template::SplitRow);
+    const bool force_stream = getenv("ASTITCH_FORCE_STREAM") && atoi(getenv("ASTITCH_FORCE_STREAM")) == 1;
+    if (stream_ok && (m.chunks_per_lane * E > kStreamNE || force_stream)) {
+      m.tmpl = Template::RowStream;
+      m.threads = 512;
+      m.split = 1;
+      if (!no_split && R < blocks_per_wave_1024) {
+        int64_t want = (blocks_per_wave_1024 + R - 1) / std::max<int64_t>(R, 1);
+        int k = 1;
+        while (k < want && k < 8) k *= 2;
+        m.split = k;
+      }
+      m.team = m.split * m.threads;
+      m.chunks_per_lane = std::max(1, 32 / E);  // V: 32 values per lane per tile
+      m.lane_util = 1.0;
+      m.rows_per_block = 1;
+      m.row_unroll = 1;
+      m.prefetch = false;
+      why << "row of " << C << " exceeds the team's registers -> streamed in tiles of " << m.team << " lanes x "
+          << m.chunks_per_lane << " chunks" << (m.split > 1 ? " over a cluster of " + std::to_string(m.split) + " CTAs" : "")
+          << ", one pass per row-reduction level; ";
+    }
   }
 
   // colvec operands: hoist in registers when the footprint is small (a6)
@@ -617,7 +650,7 @@ void retune_grid(Plan& p) {
   if (m.tmpl == Template::PackedTile) work_units = (R + m.tile_rows - 1) / m.tile_rows;
   else work_units = (R + (int64_t)m.rows_per_block * m.row_unroll - 1) / ((int64_t)m.rows_per_block * m.row_unroll);
   int64_t wave = static_cast<int64_t>(m.blocks_per_sm) * p.sm_count;
-  if (m.tmpl == Template::SplitRow) {
+  if (m.tmpl == Template::SplitRow || (m.tmpl == Template::RowStream && m.split > 1)) {
     // clusters of `split` CTAs, one row per cluster per iteration
     int64_t clusters = std::max<int64_t>(1, std::min(work_units, wave / m.split));
     m.grid = clusters * m.split;

@@ -406,7 +406,7 @@ astitch_status astitch_run_host_pipelined(astitch_plan_t h, const void* const* h
   // rows are the independent units: chunk them; a column reduction accumulates
   // its totals across chunks and its consumers run once at the end
   if (chunks <= 1 || R < static_cast<int64_t>(chunks) * 64 || (global && p.needs_sweep2) ||
-      p.desc.shard_world > 1 || p.map.tmpl == Template::SplitRow || p.device < 0 || p.g.segments_node >= 0)
+      p.desc.shard_world > 1 || p.map.tmpl == Template::SplitRow || p.map.tmpl == Template::RowStream || p.device < 0 || p.g.segments_node >= 0)
     return astitch_run_host(h, host_inputs, host_outputs, dev_inputs, dev_outputs, ws, stream);
   if (chunks > 64) chunks = 64;
   astitch_status s = check_io(p, dev_inputs, dev_outputs, ws);

@@ -347,3 +347,26 @@ def test_one_kernel_no_memset_per_run(cfg):
     other = [n for n in names if not n.startswith("astitch_")]
     assert len(kern) == 1, names
     assert not any("memset" in n.lower() or "memcpy" in n.lower() for n in other), names
+
+
+@pytest.mark.parametrize("cfg,rows,cols,force", [("C1", None, None, True), ("C2", 300, None, True),
+                                                 ("fig5", None, None, True), ("remote", None, None, True),
+                                                 ("C4", 37, 5000, True), ("fig6b", 64, 300000, True),
+                                                 ("C1", 16, 2_000_000, False), ("C4", 8, 1_000_003, False),
+                                                 ("fig6b", 3, 4_000_000, False)])
+def test_parity_row_stream(cfg, rows, cols, force, monkeypatch):
+    """Rows longer than a team's registers: streamed column tiles, one pass per
+    row-reduction level (forced on small shapes; chosen by the planner for
+    multi-MB rows)."""
+    if force:
+        monkeypatch.setenv("ASTITCH_FORCE_STREAM", "1")
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    x = gen.generate(cfg, spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    d = plan.describe()
+    assert d["mapping"]["template"] == "row_stream" and d["kernel_count"] == 1
+    assert d["kernels"][0]["spill_bytes"] == 0
+    _compare(spec, got, evaluate(spec, x))
+    again = run_gpu(spec, x, plan=plan)
+    for k in got:
+        assert np.array_equal(got[k], again[k])       # deterministic tile order

@@ -118,7 +118,8 @@ def test_fig6_selector_branches():
     d, _, _ = describe("fig6b", cols=300_000)  # 1.2 MB rows: split by default
     assert d["mapping"]["template"] == "split_row"
     d, _, _ = describe("fig6b", cols=300_000, flags=A.FLAG_NO_COMPILE | A.FLAG_NO_SPLIT)
-    assert d["mapping"]["template"] == "row_team"
+    # no splitting: a 1024-lane block would need 293 values per lane -> streamed by one block
+    assert d["mapping"]["template"] == "row_stream" and d["mapping"]["split"] == 1
 
 
 @pytest.mark.parametrize("cfg", ["C2", "C3", "C4"])
@@ -220,3 +221,17 @@ def test_sharded_plan_has_epilogue_kernels():
     assert d["kernel_count"] == 1 and d["shard_kernels"] == 2
     d, _, _ = describe("fig7a", flags=0, shard_rank=0, shard_world=2)
     assert d["shard_kernels"] == 3
+
+
+def test_row_stream_for_rows_beyond_registers():
+    """A row too long for a team's registers is streamed in column tiles (one
+    pass per row-reduction level: softmax = max | sum | output = 3 passes)."""
+    d, _, p = describe("C1", rows=16, cols=2_000_000)
+    m = d["mapping"]
+    assert m["template"] == "row_stream" and m["split"] == 8 and m["chunks_per_lane"] * m["vec_elems"] == 32
+    src = p.source(0)
+    assert src.count("// ---- pass ") == 3
+    d, _, _ = describe("C1")                       # short rows stay in registers
+    assert d["mapping"]["template"] == "row_team"
+    d, _, _ = describe("C4", rows=100_000, cols=200_000)  # many long rows: block per row, no cluster
+    assert d["mapping"]["template"] == "row_stream" and d["mapping"]["split"] == 1
