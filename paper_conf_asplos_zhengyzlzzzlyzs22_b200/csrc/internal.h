@@ -154,6 +154,7 @@ struct Plan {
   int gbuf_slots = 0;            // distinct buffers after liveness-based reuse
   bool needs_sweep2 = false;     // FULL / ROWVEC work after the (first) grid barrier
   int max_level = 0;             // grid barriers needed by dependent column reductions
+  bool stream_fallback = false;  // registers overflowed at 1 block/SM: stream the rows
   std::vector<Kernel> kernels;   // kernels launched by astitch_run, in order
   std::vector<Kernel> shard_kernels; // kernels of the sharded path (after the allreduce)
   // chunked host pipeline (astitch_run_host_pipelined): copy-in / compute /

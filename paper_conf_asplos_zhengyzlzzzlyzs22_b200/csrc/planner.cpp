@@ -590,9 +590,10 @@ void select_mapping(Plan& p) {
     // per-row re-read keeps it in one pass of the grid with no barrier.
     constexpr int kStreamNE = 128;
     const bool stream_ok = !has_mask && p.global_fulls.empty() &&
+                           !(getenv("ASTITCH_NO_STREAM") && atoi(getenv("ASTITCH_NO_STREAM")) == 1) &&
                            (m.tmpl == Template::RowTeam || m.tmpl == Template::SplitRow);
     const bool force_stream = getenv("ASTITCH_FORCE_STREAM") && atoi(getenv("ASTITCH_FORCE_STREAM")) == 1;
-    if (stream_ok && (m.chunks_per_lane * E > kStreamNE || force_stream)) {
+    if (stream_ok && (m.chunks_per_lane * E > kStreamNE || force_stream || p.stream_fallback)) {
       m.tmpl = Template::RowStream;
       m.threads = 512;
       m.split = 1;

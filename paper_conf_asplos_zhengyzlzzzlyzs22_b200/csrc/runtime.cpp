@@ -106,6 +106,17 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     if (st != ASTITCH_OK) return st;
     if (!may_relax || getenv("ASTITCH_FORCE_BPS")) return ASTITCH_OK;
     const int cur = p.map.blocks_per_sm;
+    if (k.spill_bytes > 0 && cur == 1 && !p.stream_fallback &&
+        !(getenv("ASTITCH_NO_STREAM") && atoi(getenv("ASTITCH_NO_STREAM")) == 1) &&
+        (p.map.tmpl == Template::RowTeam || p.map.tmpl == Template::SplitRow) && p.g.lengths_node < 0 &&
+        p.g.segments_node < 0 && p.global_fulls.empty()) {
+      // the row does not fit the team's registers even at one block per SM:
+      // re-plan it as a streamed row (column tiles, one pass per level)
+      p.stream_fallback = true;
+      select_mapping(p);
+      good = bad = 0;
+      continue;
+    }
     if (k.spill_bytes > 0 && cur == 1 && p.map.row_unroll > 1) {
       // even one block per SM spills: fewer rows in flight per team
       p.map.row_unroll /= 2;
