@@ -1051,7 +1051,8 @@ struct Gen {
   // whole padded row dominate, and the 5x code loses 1-4%).
   void emit_row_block(bool post, const std::string& s, const std::string& row, const std::string& act,
                       const std::string& lim) {
-    const bool spec = ragged && m.tmpl == Template::RowTeam && V >= 2 && !split &&
+    const bool kf_env = getenv("ASTITCH_KF") && atoi(getenv("ASTITCH_KF")) == 1;  // experiments: padded masks too
+    const bool spec = (ragged || (masked && kf_env)) && m.tmpl == Template::RowTeam && V >= 2 && !split &&
                       !(getenv("ASTITCH_NO_KF") && atoi(getenv("ASTITCH_NO_KF")) == 1);
     if (!spec) {
       o << "    {\n";
