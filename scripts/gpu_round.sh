@@ -4,10 +4,11 @@
 #   list of the bench command itself, dram traffic per launch, and one
 #   `ncu --set full` capture per HBM-bound config.
 mkdir -p gpurun_out
+python -m pytest tests/ -q -m gpu 2>&1 | tail -4 > gpurun_out/pytest_gpu.txt
 nproc > gpurun_out/nproc.txt
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.limit --format=csv > gpurun_out/gpu.txt
 python bench.py > gpurun_out/bench_C5.json 2> gpurun_out/bench_C5.err
-for c in C1 C2 C3 C4; do
+for c in C1 C2 C3 C4 C3v; do
   python bench.py --config $c --no-cpu-baseline > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err
 done
 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
@@ -15,11 +16,11 @@ python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_ref.jso
 timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
    --log-file gpurun_out/launches_bench_C5.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --e2e-steps 1 \
    > gpurun_out/ncu_bench_C5.out 2>&1
-for c in C1 C2 C3 C4 C5; do
+for c in C1 C2 C3 C4 C5 C3v; do
   timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv \
      --log-file gpurun_out/launches_$c.csv python scripts/profile_run.py --config $c --iters 5 > /dev/null 2>&1
 done
-for c in C3 C4 C5 C2; do
+for c in C3 C4 C5 C2 C3v; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:astitch_ -s 2 -c 1 \
      -o gpurun_out/prof_$c -f python scripts/profile_run.py --config $c --iters 3 > gpurun_out/ncu_$c.log 2>&1
 done

@@ -90,9 +90,9 @@ def main():
     if os.path.exists(gpu):
         lines += ["```", open(gpu).read().strip(), "```", ""]
     lines += ["## bench.py lines (CUDA-graph replay, events on the launch stream)", "",
-              "| cfg | GB/s | us/subgraph | % of 8 TB/s | frac of measured 6.54 TB/s | % of copy kernel | e2e GB/s | sm MHz | reasons |",
+              "| cfg | GB/s | us/subgraph | % of 8 TB/s | frac of measured peak | % of copy kernel | e2e GB/s | sm MHz | reasons |",
               "|---|---|---|---|---|---|---|---|---|"]
-    for c in ("C1", "C2", "C3", "C4", "C5"):
+    for c in ("C1", "C2", "C3", "C4", "C5", "C3v"):
         p = os.path.join(OUT, f"bench_{c}.json")
         if not os.path.exists(p):
             continue
@@ -102,14 +102,14 @@ def main():
             continue
         shutil.copy(p, os.path.join(PROF, f"{rnd}_bench_{c}.json"))
         lines.append(f"| {c} | {d['value']} | {d['us_per_subgraph']} | {d['pct_of_8TBps']} | {d['roofline']['frac']} | "
-                     f"{d['pct_of_copy_kernel']} | {d['e2e']['value']} | {d['clocks']['sm_mhz']} | {d['clocks']['reasons']} |")
+                     f"{d['pct_of_copy_kernel']} | {(d.get('e2e') or {}).get('value')} | {d['clocks']['sm_mhz']} | {d['clocks']['reasons']} |")
     ref = os.path.join(OUT, "bench_ref.json")
     if os.path.exists(ref):
         shutil.copy(ref, os.path.join(PROF, f"{rnd}_bench_reference.json"))
     traffic = {}
     lines += ["", "## ncu launch lists (`--metrics gpu__time_duration.sum,dram__bytes_*`, cold-cache, serialised)", "",
               "| cfg | kernel | launches | median us | DRAM read MB/launch | DRAM write MB/launch |", "|---|---|---|---|---|---|"]
-    for c in ("C1", "C2", "C3", "C4", "C5"):
+    for c in ("C1", "C2", "C3", "C4", "C5", "C3v"):
         p = os.path.join(OUT, f"launches_{c}.csv")
         if not os.path.exists(p):
             continue
