@@ -261,6 +261,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg (ablation sweeps)")
     ap.add_argument("--flags", type=int, default=0)
+    ap.add_argument("--exchange", default="fused", choices=["fused", "nccl"],
+                    help="N>1 column reductions: in-kernel exchange over peer memory (fused) or ncclAllReduce + epilogue")
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
     ap.add_argument("--rows", type=int, default=None, help="override the config's rows (experiments)")
     ap.add_argument("--cols", type=int, default=None, help="override the config's cols (experiments)")
@@ -307,6 +309,17 @@ def main():
     graph = A.Graph.from_spec(spec)
     comm = Comm.from_process_group(dev) if world > 1 else None
     sp = ShardedPlan(graph, R, C, 1 if ragged else world, 0 if ragged else rank, dev, comm=comm, flags=args.flags)
+    exchange = "none"
+    if world > 1 and not ragged and sp.needs_exchange():
+        exchange = "ncclAllReduce + epilogue"
+        if args.exchange == "fused":
+            from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import PeerExchange
+            try:
+                sp.peer = PeerExchange.from_process_group(sp.plan)
+                exchange = "in-kernel over peer memory (astitch_run_fused)"
+            except Exception as e:  # pragma: no cover - needs a multi-GPU box
+                print(f"[bench] fused exchange unavailable ({e}); using NCCL", file=sys.stderr)
+                sp.peer = None
     plan = sp.plan
     desc = plan.describe()
     r0, nr = sp.row_begin, sp.row_count
@@ -482,7 +495,7 @@ def main():
             "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": f"{cfg}: {WORKLOAD_NAMES.get(cfg, spec_name(cfg))}", "rows": R, "cols": C, "global_batch": R,
                        "io_dtype": "bf16" if any(d == "BF16" for _, _, d in spec["inputs"]) else "f32",
-                       "parallelism": f"dp{world} contiguous row shards" + (", 1 ncclAllReduce of fp32 column partials" if world > 1 and desc["shard_kernels"] else ""),
+                       "parallelism": f"dp{world} contiguous row shards" + (f", column totals exchanged {exchange}" if exchange != "none" else ""),
                        "l2": ("inputs > L2 (%.2f GB per rank vs %d MB L2)" % (nbytes / 1e9, l2 // 2**20)) if nsets == 1
                        else f"{nsets} rotating input sets >= 4x L2",
                        "timing": "cuda_graph_replay" if graph is not None else "eager",

@@ -268,6 +268,35 @@ astitch_status astitch_run_sharded(astitch_plan_t p, astitch_comm_t c, const voi
 astitch_status astitch_run_shard_stage(astitch_plan_t p, int32_t stage, const void* const* inputs,
                                        void* const* outputs, void* ws, void* stream);
 astitch_status astitch_plan_colpart(astitch_plan_t p, size_t* byte_offset, size_t* count);
+/* Fused sharded run: the column-reduction exchange happens
+ * INSIDE the stitched kernel over peer memory instead of an ncclAllReduce +
+ * epilogue launch.  Each rank owns an exchange buffer (astitch_peer_create:
+ * device memory, ~1 KB + 2 x world x ncolred x cols fp32, zeroed once) and maps
+ * every other rank's buffer: astitch_peer_open with that rank's 64-byte CUDA IPC
+ * handle (one process per GPU; peer access over NVLink / NVSwitch), or
+ * astitch_peer_link with its peer object (several ranks in one process, e.g.
+ * virtual ranks on one GPU).  astitch_run_fused then launches ONE cooperative
+ * kernel per rank: sweep -> block column partials -> grid barrier -> rank-local
+ * totals stored into slot [run parity][rank] of every rank's buffer (plain P2P
+ * stores) -> system fence -> grid barrier -> one release flag per rank -> wait
+ * for all ranks' flags of this run -> fixed-order (rank 0..world-1) combine ->
+ * column consumers (+ the FULL sweep after the barrier).  Results are bitwise
+ * identical on every rank.  Every rank must make the same sequence of
+ * astitch_run_fused calls; the ranks' kernels must be able to run at the same
+ * time (separate GPUs, or grids that fit together).  A rank that does not
+ * arrive within ~2 s makes the waiting kernels give up (no hang): their
+ * outputs are then invalid and astitch_peer_status reports timed_out = 1.
+ * Errors: ERR_INVALID_ARGUMENT (mismatched plan / peer, peer not mapped),
+ * ERR_UNSUPPORTED (> 64 ranks), ERR_CUDA (allocation, IPC, launch). */
+typedef struct astitch_peer_s* astitch_peer_t;
+astitch_status astitch_peer_create(astitch_plan_t p, astitch_peer_t* out, uint8_t ipc_handle[64]);
+astitch_status astitch_peer_open(astitch_peer_t x, int32_t rank, const uint8_t ipc_handle[64]);
+astitch_status astitch_peer_link(astitch_peer_t x, int32_t rank, astitch_peer_t other);
+/* Synchronous read of the buffer's error word (1 = a wait timed out). */
+astitch_status astitch_peer_status(astitch_peer_t x, int32_t* timed_out);
+astitch_status astitch_peer_destroy(astitch_peer_t x);
+astitch_status astitch_run_fused(astitch_plan_t p, astitch_peer_t x, const void* const* inputs,
+                                 void* const* outputs, void* ws, void* stream);
 /* Contiguous row partition: rows_k = floor(R/g) (+1 for the first R mod g ranks). */
 astitch_status astitch_shard_rows(int64_t rows, int32_t world, int32_t rank, int64_t* row_begin,
                                   int64_t* row_count);

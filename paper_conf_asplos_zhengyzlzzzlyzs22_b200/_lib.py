@@ -97,6 +97,12 @@ _sig = {
     "astitch_run_sharded": (ct.c_int, [_vp, _vp, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
     "astitch_run_shard_stage": (ct.c_int, [_vp, ct.c_int32, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
     "astitch_plan_colpart": (ct.c_int, [_vp, ct.POINTER(ct.c_size_t), ct.POINTER(ct.c_size_t)]),
+    "astitch_peer_create": (ct.c_int, [_vp, ct.POINTER(_vp), ct.c_char_p]),
+    "astitch_peer_open": (ct.c_int, [_vp, ct.c_int32, ct.c_char_p]),
+    "astitch_peer_link": (ct.c_int, [_vp, ct.c_int32, _vp]),
+    "astitch_peer_status": (ct.c_int, [_vp, _i32p]),
+    "astitch_peer_destroy": (ct.c_int, [_vp]),
+    "astitch_run_fused": (ct.c_int, [_vp, _vp, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
     "astitch_shard_rows": (ct.c_int, [ct.c_int64, ct.c_int32, ct.c_int32, ct.POINTER(ct.c_int64),
                                       ct.POINTER(ct.c_int64)]),
     "astitch_bench_barrier": (ct.c_int, [ct.c_int32, ct.c_int32, ct.c_int32, ct.c_int32, _vp, _vp]),

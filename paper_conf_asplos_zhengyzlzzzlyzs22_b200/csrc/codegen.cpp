@@ -156,7 +156,7 @@ struct Gen {
       if (std::string(q) == ".cs" || std::string(q) == ".wt" || std::string(q) == ".cg")
         o << "#define AS_STQ \"" << q << "\"\n";
     o << "#include \"astitch_device.cuh\"\n";
-    o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; };\n";
+    o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; void* xbuf; unsigned int gen; };\n";
     o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") ";
     if (split) o << "__cluster_dims__(" << m.split << ", 1, 1) ";
     o << name << "(const Params p) {\n";
@@ -1170,6 +1170,53 @@ struct Gen {
     o << "      }\n    }\n  }\n";
   }
 
+  // Fused sharded stage (astitch_run_fused, NEXT f1): the rank-local column
+  // totals of this block's columns (ws colpart) are pushed with plain stores
+  // into slot [gen parity][this rank] of EVERY rank's exchange buffer (peer
+  // memory over NVLink), published by a system fence + grid barrier + one
+  // release flag per rank; each block then waits for all ranks' flags (bounded)
+  // and combines the world slots in rank order 0..world-1 (identical on every
+  // rank: deterministic) before the column consumers.  One kernel, no NCCL.
+  void emit_fused_exchange() {
+    const int ncr = static_cast<int>(p.colreds.size());
+    const int XW = p.desc.shard_world, XR = p.desc.shard_rank;
+    const long long colpart = static_cast<long long>(p.ws.colvals + p.post_colvecs.size() * C * 4);
+    o << "  __syncthreads();\n";
+    o << "  {  // ---- fused exchange of the column totals over peer memory\n";
+    o << "    constexpr int XW = " << XW << ", XR = " << XR << ", NCR = " << ncr << ";\n";
+    o << "    unsigned char* X = (unsigned char*)p.xbuf;\n";
+    o << "    const float* colpart = (const float*)((const char*)p.ws + " << colpart << "LL);\n";
+    o << "    const int G = gridDim.x;\n    const long long W = (C + G - 1) / G;\n";
+    o << "    const long long c0 = (long long)blockIdx.x * W, c1 = min(C, c0 + W);\n";
+    o << "    const int par = (int)(p.gen & 1u);\n";
+    o << "    for (int q = 0; q < XW; ++q) {\n";
+    o << "      float* dst = (float*)(__ldcg((const unsigned long long*)X + q) + " << kXSlots
+      << "ULL) + ((long long)(par * XW + XR) * NCR) * C;\n";
+    o << "      for (long long col = c0 + threadIdx.x; col < c1; col += blockDim.x)\n";
+    o << "#pragma unroll\n        for (int r = 0; r < NCR; ++r) dst[r * C + col] = colpart[r * C + col];\n";
+    o << "    }\n";
+    o << "    __threadfence_system();\n";
+    o << "    as::grid_barrier(bar);\n";
+    o << "    if (blockIdx.x == 0 && threadIdx.x < XW)\n";
+    o << "      as::st_release_sys((unsigned int*)(__ldcg((const unsigned long long*)X + threadIdx.x) + " << kXFlags
+      << "ULL) + XR, p.gen);\n";
+    o << "    if (threadIdx.x == 0) as::wait_flags((const unsigned int*)(X + " << kXFlags << "), XW, p.gen, (unsigned int*)(X + "
+      << kXErr << "));\n";
+    o << "    __syncthreads();\n";
+    o << "    const float* slots = (const float*)(X + " << kXSlots << ") + (long long)par * XW * NCR * C;\n";
+    o << "    for (long long col = c0 + threadIdx.x; col < c1; col += blockDim.x) {\n";
+    for (int q = 0; q < ncr; ++q) {
+      int id = p.colreds[q];
+      bool mx = N(id).sub == ASTITCH_RMAX;
+      o << "      float t" << id << " = " << (mx ? "-AS_INF" : "0.f") << ";\n";
+      o << "      for (int q = 0; q < XW; ++q) { const float x_ = as::ld_cg(slots + ((long long)q * NCR + " << q
+        << ") * C + col); t" << id << " = " << (mx ? "fmaxf(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_")
+        << "; }\n";
+    }
+    emit_colvec_chain("t");
+    o << "    }\n  }\n";
+  }
+
   // COLVEC chain for one column `col` given totals t<id> of the column
   // reductions finalised at this barrier (level cur_level + 1); values of
   // earlier barriers are read back from the workspace, level-0 ones recomputed
@@ -1626,7 +1673,7 @@ struct Gen {
       // small epilogue: one thread per column, consumers of the all-reduced
       // column totals (sharded global stage)
       o << "#include \"astitch_device.cuh\"\n";
-      o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; };\n";
+      o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; void* xbuf; unsigned int gen; };\n";
       o << "extern \"C\" __global__ void __launch_bounds__(256) " << name << "(const Params p) {\n";
       o << "  constexpr long long C = " << C << "LL;\n";
       for (size_t i = 0; i < g.nodes.size(); ++i)
@@ -1685,6 +1732,10 @@ struct Gen {
         o << "  as::grid_barrier(bar);\n";
         if (role == ROLE_SHARD_MAIN) {
           emit_column_finalize(false);
+        } else if (role == ROLE_FUSED) {
+          emit_column_finalize(false);
+          emit_fused_exchange();
+          if (lv < D) o << "  as::grid_barrier(bar);\n";
         } else {
           emit_column_finalize(true);
           if (lv < D) o << "  as::grid_barrier(bar);\n";

@@ -11,6 +11,7 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <vector>
 
 #include "internal.h"
 #include "nccl.h"
@@ -75,7 +76,18 @@ struct astitch_comm_s {
   int world = 1, rank = 0, device = 0;
 };
 
+struct astitch_peer_s {
+  int world = 1, rank = 0, device = 0;
+  size_t bytes = 0;
+  void* local = nullptr;                  // this rank's exchange buffer (cuMemAlloc)
+  std::vector<void*> ptrs;                // every rank's buffer as addressed from this process
+  std::vector<bool> opened;               // ptrs[q] came from cuIpcOpenMemHandle (close on destroy)
+  bool table_dirty = true;
+  unsigned int gen = 0;
+};
+
 namespace astitch {
+astitch_status build_plan_kernel(Plan& p, int role, Kernel& k);
 astitch_status check_io(const Plan& p, const void* const* inputs, void* const* outputs, void* ws);
 KernelParams make_params(const Plan& p, const void* const* inputs, void* const* outputs, void* ws);
 astitch_status launch(const Plan& p, const Kernel& k, KernelParams& kp, void* stream);
@@ -161,6 +173,116 @@ astitch_status astitch_run_sharded(astitch_plan_t h, astitch_comm_t c, const voi
   for (size_t i = 1; i < p.shard_kernels.size(); ++i)
     if ((s = launch(p, p.shard_kernels[i], kp, stream)) != ASTITCH_OK) return s;
   return ASTITCH_OK;
+}
+
+// ---------------------------------------------------------------- fused sharded run (NEXT f1)
+astitch_status astitch_peer_create(astitch_plan_t h, astitch_peer_t* out, uint8_t ipc_handle[64]) {
+  if (!h || !out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan or out");
+  *out = nullptr;
+  const Plan& p = *h->p;
+  if (p.device < 0) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "host-only plan");
+  if (p.desc.shard_world > 64) return fail(ASTITCH_ERR_UNSUPPORTED, "fused exchange supports up to 64 ranks");
+  auto* x = new astitch_peer_s();
+  x->world = p.desc.shard_world;
+  x->rank = p.desc.shard_rank;
+  x->device = p.device;
+  x->bytes = xbuf_bytes(x->world, std::max<size_t>(p.colreds.size(), 1), p.desc.cols);
+  std::string err;
+  if (!drv_alloc_zero(x->device, x->bytes, &x->local, err)) {
+    delete x;
+    return fail(ASTITCH_ERR_CUDA, err);
+  }
+  x->ptrs.assign(x->world, nullptr);
+  x->opened.assign(x->world, false);
+  x->ptrs[x->rank] = x->local;
+  if (ipc_handle) {
+    memset(ipc_handle, 0, 64);
+    if (!drv_ipc_get(x->local, ipc_handle, err)) {
+      drv_free(x->local);
+      delete x;
+      return fail(ASTITCH_ERR_CUDA, err);
+    }
+  }
+  *out = x;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_peer_open(astitch_peer_t x, int32_t rank, const uint8_t ipc_handle[64]) {
+  if (!x || !ipc_handle) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL peer or handle");
+  if (rank < 0 || rank >= x->world) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "rank out of range");
+  if (rank == x->rank) return ASTITCH_OK;
+  std::string err;
+  void* ptr = nullptr;
+  if (!drv_ipc_open(x->device, ipc_handle, &ptr, err)) return fail(ASTITCH_ERR_CUDA, err);
+  if (x->opened[rank]) drv_ipc_close(x->ptrs[rank]);
+  x->ptrs[rank] = ptr;
+  x->opened[rank] = true;
+  x->table_dirty = true;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_peer_link(astitch_peer_t x, int32_t rank, astitch_peer_t other) {
+  if (!x || !other) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL peer");
+  if (rank < 0 || rank >= x->world || other->rank != rank || other->world != x->world || other->bytes != x->bytes)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "peer does not match (rank / world / plan)");
+  x->ptrs[rank] = other->local;
+  x->table_dirty = true;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_peer_status(astitch_peer_t x, int32_t* timed_out) {
+  if (!x || !timed_out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  uint32_t e = 0;
+  std::string err;
+  if (!drv_dtoh(&e, static_cast<char*>(x->local) + kXErr, 4, err)) return fail(ASTITCH_ERR_CUDA, err);
+  *timed_out = e ? 1 : 0;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_peer_destroy(astitch_peer_t x) {
+  if (!x) return ASTITCH_OK;
+  for (int q = 0; q < x->world; ++q)
+    if (x->opened[q]) drv_ipc_close(x->ptrs[q]);
+  drv_free(x->local);
+  delete x;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_run_fused(astitch_plan_t h, astitch_peer_t x, const void* const* inputs,
+                                 void* const* outputs, void* ws, void* stream) {
+  if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
+  Plan& p = *h->p;
+  if (p.colreds.empty() || p.desc.shard_world <= 1) return astitch_run(h, inputs, outputs, ws, stream);
+  if (!x) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "column reduction over shards needs a peer exchange");
+  if (x->world != p.desc.shard_world || x->rank != p.desc.shard_rank ||
+      x->bytes != xbuf_bytes(x->world, std::max<size_t>(p.colreds.size(), 1), p.desc.cols))
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "peer exchange does not match the plan's shard");
+  for (int q = 0; q < x->world; ++q)
+    if (!x->ptrs[q]) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "peer " + std::to_string(q) + " not opened / linked");
+  astitch_status s = check_io(p, inputs, outputs, ws);
+  if (s != ASTITCH_OK) return s;
+  std::string err;
+  if (p.fused_kernels.empty()) {
+    p.fused_kernels.resize(1);
+    if ((s = build_plan_kernel(p, ROLE_FUSED, p.fused_kernels[0])) != ASTITCH_OK) {
+      p.fused_kernels.clear();
+      return s;
+    }
+    Kernel& k = p.fused_kernels[0];
+    if (!k.module && !drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
+    k.grid = std::min<int64_t>(k.grid, static_cast<int64_t>(k.occupancy) * p.sm_count);
+  }
+  if (x->table_dirty) {  // device addresses of every rank's buffer, read by the kernel
+    std::vector<uint64_t> t(x->world);
+    for (int q = 0; q < x->world; ++q) t[q] = reinterpret_cast<uint64_t>(x->ptrs[q]);
+    if (!drv_htod(x->local, t.data(), 8 * t.size(), err)) return fail(ASTITCH_ERR_CUDA, err);
+    x->table_dirty = false;
+  }
+  KernelParams kp = make_params(p, inputs, outputs, ws);
+  kp.xbuf = x->local;
+  kp.gen = ++x->gen;
+  if (kp.gen == 0) kp.gen = ++x->gen;  // 0 is the initial flag value
+  return launch(p, p.fused_kernels[0], kp, stream);
 }
 
 astitch_status astitch_plan_colpart(astitch_plan_t h, size_t* byte_offset, size_t* count) {

@@ -5,6 +5,7 @@
 #include <cuda.h>
 #include <dlfcn.h>
 
+#include <cstring>
 #include <mutex>
 #include <string>
 
@@ -38,6 +39,14 @@ struct Driver {
   CUresult (*EventDestroy)(CUevent);
   CUresult (*EventRecord)(CUevent, CUstream);
   CUresult (*StreamWaitEvent)(CUstream, CUevent, unsigned int);
+  CUresult (*MemAlloc)(CUdeviceptr*, size_t);
+  CUresult (*MemFree)(CUdeviceptr);
+  CUresult (*MemsetD8)(CUdeviceptr, unsigned char, size_t);
+  CUresult (*MemcpyHtoD)(CUdeviceptr, const void*, size_t);
+  CUresult (*MemcpyDtoH)(void*, CUdeviceptr, size_t);
+  CUresult (*IpcGetMemHandle)(CUipcMemHandle*, CUdeviceptr);
+  CUresult (*IpcOpenMemHandle)(CUdeviceptr*, CUipcMemHandle, unsigned int);
+  CUresult (*IpcCloseMemHandle)(CUdeviceptr);
 };
 
 namespace {
@@ -99,6 +108,14 @@ Driver* driver(std::string& err) {
   SYM(EventDestroy, "cuEventDestroy_v2");
   SYM(EventRecord, "cuEventRecord");
   SYM(StreamWaitEvent, "cuStreamWaitEvent");
+  SYM(MemAlloc, "cuMemAlloc_v2");
+  SYM(MemFree, "cuMemFree_v2");
+  SYM(MemsetD8, "cuMemsetD8_v2");
+  SYM(MemcpyHtoD, "cuMemcpyHtoD_v2");
+  SYM(MemcpyDtoH, "cuMemcpyDtoH_v2");
+  SYM(IpcGetMemHandle, "cuIpcGetMemHandle");
+  SYM(IpcOpenMemHandle, "cuIpcOpenMemHandle_v2");
+  SYM(IpcCloseMemHandle, "cuIpcCloseMemHandle");
 #undef SYM
   CUresult r = d.Init(0);
   if (r != CUDA_SUCCESS) {
@@ -288,6 +305,65 @@ void drv_event_destroy(void* e) {
   std::string err;
   Driver* d = driver(err);
   if (d && e) d->EventDestroy(static_cast<CUevent>(e));
+}
+
+// ---- peer exchange buffers of the fused sharded run (comm.cpp)
+bool drv_alloc_zero(int device, size_t bytes, void** ptr, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  if (!ensure_ctx(d, device, err)) return false;
+  CUdeviceptr p = 0;
+  CUresult r = d->MemAlloc(&p, bytes);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuMemAlloc"); return false; }
+  r = d->MemsetD8(p, 0, bytes);
+  if (r != CUDA_SUCCESS) { d->MemFree(p); err = cu_err(d, r, "cuMemsetD8"); return false; }
+  *ptr = reinterpret_cast<void*>(p);
+  return true;
+}
+void drv_free(void* ptr) {
+  std::string err;
+  Driver* d = driver(err);
+  if (d && ptr) d->MemFree(reinterpret_cast<CUdeviceptr>(ptr));
+}
+bool drv_htod(void* dst, const void* src, size_t bytes, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUresult r = d->MemcpyHtoD(reinterpret_cast<CUdeviceptr>(dst), src, bytes);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuMemcpyHtoD"); return false; }
+  return true;
+}
+bool drv_dtoh(void* dst, const void* src, size_t bytes, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUresult r = d->MemcpyDtoH(dst, reinterpret_cast<CUdeviceptr>(src), bytes);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuMemcpyDtoH"); return false; }
+  return true;
+}
+bool drv_ipc_get(void* ptr, unsigned char handle[64], std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  CUipcMemHandle h;
+  CUresult r = d->IpcGetMemHandle(&h, reinterpret_cast<CUdeviceptr>(ptr));
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuIpcGetMemHandle"); return false; }
+  memcpy(handle, h.reserved, 64);
+  return true;
+}
+bool drv_ipc_open(int device, const unsigned char handle[64], void** ptr, std::string& err) {
+  Driver* d = driver(err);
+  if (!d) return false;
+  if (!ensure_ctx(d, device, err)) return false;
+  CUipcMemHandle h;
+  memcpy(h.reserved, handle, 64);
+  CUdeviceptr p = 0;
+  CUresult r = d->IpcOpenMemHandle(&p, h, CU_IPC_MEM_LAZY_ENABLE_PEER_ACCESS);
+  if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuIpcOpenMemHandle"); return false; }
+  *ptr = reinterpret_cast<void*>(p);
+  return true;
+}
+void drv_ipc_close(void* ptr) {
+  std::string err;
+  Driver* d = driver(err);
+  if (d && ptr) d->IpcCloseMemHandle(reinterpret_cast<CUdeviceptr>(ptr));
 }
 
 bool drv_sync(void* stream, std::string& err) {

@@ -157,6 +157,7 @@ struct Plan {
   bool stream_fallback = false;  // registers overflowed at 1 block/SM: stream the rows
   std::vector<Kernel> kernels;   // kernels launched by astitch_run, in order
   std::vector<Kernel> shard_kernels; // kernels of the sharded path (after the allreduce)
+  std::vector<Kernel> fused_kernels; // fused sharded path (P2P exchange in-kernel), built lazily
   // chunked host pipeline (astitch_run_host_pipelined): copy-in / compute /
   // copy-out streams, per-chunk events, and for global plans the row-chunk
   // kernels (shard-main with accumulation + column epilogue), built lazily
@@ -179,7 +180,18 @@ uint64_t compulsory_bytes(const Plan& p);
 
 // codegen.cpp
 std::string generate_kernel(const Plan& p, int role, const std::string& name);
-enum KernelRole { ROLE_MAIN = 0, ROLE_SHARD_MAIN = 1, ROLE_SHARD_FINAL = 2, ROLE_SHARD_SWEEP2 = 3 };
+enum KernelRole { ROLE_MAIN = 0, ROLE_SHARD_MAIN = 1, ROLE_SHARD_FINAL = 2, ROLE_SHARD_SWEEP2 = 3, ROLE_FUSED = 4 };
+
+// Peer exchange buffer of the fused sharded run (astitch_run_fused), one per
+// rank, device memory:  [peers: world x u64 device addresses of every rank's
+// buffer as mapped in this process] [flags: world x u32] [err: u32] ... then at
+// kXSlots: 2 (generation parity) x world x ncolred x cols fp32 slots.
+constexpr size_t kXFlags = 8 * 64;           // up to 64 ranks
+constexpr size_t kXErr = kXFlags + 4 * 64;
+constexpr size_t kXSlots = 1024;
+inline size_t xbuf_bytes(int world, size_t ncolred, int64_t cols) {
+  return kXSlots + 2 * static_cast<size_t>(world) * ncolred * static_cast<size_t>(cols) * 4;
+}
 
 // jit.cpp
 bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<char>& cubin,
@@ -203,6 +215,13 @@ bool drv_event_create(void** e, std::string& err);
 bool drv_event_record(void* e, void* s, std::string& err);
 bool drv_stream_wait(void* s, void* e, std::string& err);
 void drv_stream_destroy(void* s);
+bool drv_alloc_zero(int device, size_t bytes, void** ptr, std::string& err);
+void drv_free(void* ptr);
+bool drv_htod(void* dst, const void* src, size_t bytes, std::string& err);
+bool drv_dtoh(void* dst, const void* src, size_t bytes, std::string& err);
+bool drv_ipc_get(void* ptr, unsigned char handle[64], std::string& err);
+bool drv_ipc_open(int device, const unsigned char handle[64], void** ptr, std::string& err);
+void drv_ipc_close(void* ptr);
 void drv_event_destroy(void* e);
 
 // kernel parameter block (mirrors the struct emitted by codegen)
@@ -214,6 +233,8 @@ struct KernelParams {
   long long rows;
   long long row_offset;   // global row index of row 0 (chunked runs; mask segments)
   int flags;              // bit 0: accumulate column totals onto earlier chunks
+  void* xbuf;             // fused sharded run: this rank's peer exchange buffer
+  unsigned int gen;       // fused sharded run: generation of this run (flags)
 };
 
 }  // namespace astitch

@@ -474,6 +474,31 @@ template <int N, bool MAX> struct Tree {
   }
 };
 
+// ------------------------------------------------------------------ fused sharded exchange
+// System-scope release / acquire on flags that other GPUs write over NVLink
+// (peer memory); the data they guard is published with a system fence.
+__device__ __forceinline__ void st_release_sys(unsigned int* p, unsigned int v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned int ld_acquire_sys(const unsigned int* p) {
+  unsigned int v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+// Wait (thread 0 of a block) until every rank's flag holds `gen`; bounded
+// (~2 s) so a missing rank cannot hang the GPU: on timeout the error word is
+// set and the caller proceeds with whatever the slots hold.
+__device__ __forceinline__ void wait_flags(const unsigned int* flags, int world, unsigned int gen,
+                                           unsigned int* err) {
+  long long spins = 0;
+  for (int q = 0; q < world; ++q) {
+    while (ld_acquire_sys(flags + q) != gen) {
+      if (++spins > (1LL << 21)) { atomicOr(err, 1u); return; }
+      __nanosleep(100);
+    }
+  }
+}
+
 // ------------------------------------------------------------------ global: grid barrier
 // Generation-counted, self-resetting barrier for a co-resident (cooperative)
 // grid.  bar[0] = arrival count, bar[1] = generation.  No memset per run.

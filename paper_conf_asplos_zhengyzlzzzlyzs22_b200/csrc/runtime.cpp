@@ -53,6 +53,7 @@ const char* role_suffix(int role) {
     case ROLE_SHARD_MAIN: return "_shard";
     case ROLE_SHARD_FINAL: return "_shard_final";
     case ROLE_SHARD_SWEEP2: return "_shard_sweep2";
+    case ROLE_FUSED: return "_fused";
   }
   return "";
 }
@@ -99,7 +100,8 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     k.threads = (role == ROLE_SHARD_FINAL) ? 256 : p.map.threads;
     k.grid = (role == ROLE_SHARD_FINAL) ? std::max<int64_t>(1, (p.desc.cols + 255) / 256) : p.map.grid;
     k.smem = (role == ROLE_SHARD_FINAL) ? 0 : p.map.smem_bytes;
-    k.cooperative = (p.map.tmpl == Template::GlobalSweep) && (role == ROLE_MAIN || role == ROLE_SHARD_MAIN);
+    k.cooperative = (p.map.tmpl == Template::GlobalSweep) &&
+                    (role == ROLE_MAIN || role == ROLE_SHARD_MAIN || role == ROLE_FUSED);
     k.pdl = !k.cooperative && role != ROLE_SHARD_FINAL && (p.desc.flags & ASTITCH_FLAG_NO_PDL) == 0;
     if (!compile) return ASTITCH_OK;
     astitch_status st = compile_and_inspect(p, k, load);
@@ -140,6 +142,11 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
 }
 
 }  // namespace
+
+namespace astitch {
+// (comm.cpp) build one more kernel of a plan, e.g. the fused sharded role
+astitch_status build_plan_kernel(Plan& p, int role, Kernel& k) { return build_kernel(p, role, k); }
+}  // namespace astitch
 
 extern "C" {
 
@@ -228,6 +235,7 @@ astitch_status astitch_plan_destroy(astitch_plan_t h) {
   for (auto& k : h->p->kernels) drv_unload(k);
   for (auto& k : h->p->shard_kernels) drv_unload(k);
   for (auto& k : h->p->chunk_kernels) drv_unload(k);
+  for (auto& k : h->p->fused_kernels) drv_unload(k);
   for (void* s : h->p->pipe_streams) drv_stream_destroy(s);
   for (void* e : h->p->pipe_events) drv_event_destroy(e);
   delete h;

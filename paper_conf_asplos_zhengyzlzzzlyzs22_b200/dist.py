@@ -3,9 +3,11 @@
 One process per GPU.  torch.distributed is the plumbing only: it bootstraps
 the NCCL communicator of libastitch (the ncclUniqueId is broadcast through the
 process group) and provides barriers for timing.  The data path is entirely in
-libastitch: astitch_run_sharded launches the stitched kernel on the rank's row
-slice and, when the subgraph has a column reduction, ONE ncclAllReduce of the
-fp32 column partials followed by the column-consumer epilogue kernel.
+libastitch.  When the subgraph has a column reduction, the rank-local fp32
+column totals are combined either INSIDE the stitched kernel over peer memory
+(PeerExchange + astitch_run_fused: one kernel per rank, NVLink P2P stores and
+flags) or by ONE ncclAllReduce between the stitched kernel and the
+column-consumer epilogue (Comm + astitch_run_sharded).
 """
 
 from __future__ import annotations
@@ -52,28 +54,93 @@ class Comm:
         return self._h
 
 
+class PeerExchange:
+    """Exchange buffer of the fused sharded run (astitch_peer_*): this rank's
+    buffer plus the mapping of every other rank's (CUDA IPC handles between
+    processes, or direct links between ranks living in one process)."""
+
+    def __init__(self, plan: Plan):
+        h = ct.c_void_p()
+        buf = ct.create_string_buffer(64)
+        check(lib.astitch_peer_create(plan.handle, ct.byref(h), buf), "astitch_peer_create")
+        self._h = h
+        self.ipc_handle = buf.raw
+
+    def open(self, rank: int, ipc_handle: bytes) -> None:
+        check(lib.astitch_peer_open(self._h, int(rank), ipc_handle), "astitch_peer_open")
+
+    def link(self, rank: int, other: "PeerExchange") -> None:
+        check(lib.astitch_peer_link(self._h, int(rank), other._h), "astitch_peer_link")
+
+    def timed_out(self) -> bool:
+        v = ct.c_int32()
+        check(lib.astitch_peer_status(self._h, ct.byref(v)), "astitch_peer_status")
+        return bool(v.value)
+
+    @classmethod
+    def from_process_group(cls, plan: Plan, group=None) -> "PeerExchange":
+        """One process per GPU: all-gather the IPC handles and map every peer."""
+        import torch.distributed as dist
+        x = cls(plan)
+        handles = [None] * dist.get_world_size(group)
+        dist.all_gather_object(handles, x.ipc_handle, group=group)
+        me = dist.get_rank(group)
+        for r, hnd in enumerate(handles):
+            if r != me:
+                x.open(r, hnd)
+        return x
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value:
+            lib.astitch_peer_destroy(h)
+            self._h = None
+
+    @property
+    def handle(self):
+        return self._h
+
+
 class ShardedPlan:
-    """The rank's plan over its contiguous row slice of an [R, C] problem."""
+    """The rank's plan over its contiguous row slice of an [R, C] problem.
+
+    A column reduction over the shards is combined either inside the stitched
+    kernel over peer memory (`peer`: astitch_run_fused, one kernel) or with an
+    NCCL allreduce between the stitched kernel and an epilogue (`comm`:
+    astitch_run_sharded)."""
 
     def __init__(self, graph: Graph, rows: int, cols: int, world: int, rank: int, device: int,
-                 comm: Comm | None = None, flags: int = 0):
+                 comm: Comm | None = None, flags: int = 0, sm_count: int = 0):
         self.row_begin, self.row_count = shard_rows(rows, world, rank)
         self.plan = Plan(graph, self.row_count, cols, device=device, flags=flags, shard_rank=rank,
-                         shard_world=world)
+                         shard_world=world, sm_count=sm_count)
         self.comm = comm
+        self.peer: PeerExchange | None = None
         self.world, self.rank = world, rank
 
-    def run(self, inputs, outputs, ws=None, stream=None) -> None:
+    def needs_exchange(self) -> bool:
+        return self.world > 1 and self.plan.describe()["shard_kernels"] > 0
+
+    def _ws(self, ws, stream):
         p = self.plan
         if ws is None and p.workspace_bytes() > 0:
             if p._ws_cache is None:
                 p._ws_cache = p.alloc_workspace(stream)
             ws = p._ws_cache
+        return ws
+
+    def run(self, inputs, outputs, ws=None, stream=None) -> None:
+        p = self.plan
+        ws = self._ws(ws, stream)
         ins = ptr_array([t.data_ptr() for t in inputs])
         outs = ptr_array([t.data_ptr() for t in outputs])
-        check(lib.astitch_run_sharded(p.handle, self.comm.handle if self.comm else None, ins, outs,
-                                      ct.c_void_p(ws.data_ptr() if ws is not None else 0),
-                                      ct.c_void_p(_stream_ptr(stream))), "astitch_run_sharded")
+        w = ct.c_void_p(ws.data_ptr() if ws is not None else 0)
+        s = ct.c_void_p(_stream_ptr(stream))
+        if self.peer is not None:
+            check(lib.astitch_run_fused(p.handle, self.peer.handle, ins, outs, w, s), "astitch_run_fused")
+            return
+        check(lib.astitch_run_sharded(p.handle, self.comm.handle if self.comm else None, ins, outs, w, s),
+              "astitch_run_sharded")
 
     def run_stage(self, stage: int, inputs, outputs, ws, stream=None) -> None:
         """astitch_run_shard_stage: 0 = stitched kernel leaving rank-local column
@@ -92,7 +159,7 @@ class ShardedPlan:
 
     def kernels_per_run(self) -> int:
         d = self.plan.describe()
-        if self.world > 1 and d["shard_kernels"] > 0:
+        if self.world > 1 and d["shard_kernels"] > 0 and self.peer is None:
             return d["shard_kernels"]
         return d["kernel_count"]
 
@@ -114,4 +181,4 @@ def partition_by_weight(weights, world: int):
     return [(bounds[r], bounds[r + 1]) for r in range(world)]
 
 
-__all__ = ["Comm", "ShardedPlan", "partition_by_weight", "_lib"]
+__all__ = ["Comm", "PeerExchange", "ShardedPlan", "partition_by_weight", "_lib"]

@@ -370,3 +370,111 @@ def test_parity_row_stream(cfg, rows, cols, force, monkeypatch):
     again = run_gpu(spec, x, plan=plan)
     for k in got:
         assert np.array_equal(got[k], again[k])       # deterministic tile order
+
+
+# The whole op vocabulary of the IR (include/astitch.h astitch_unop /
+# astitch_binop) on FULL, ROWVEC and COLVEC values, fp32 and fp16 I/O.
+OPS_UNARY = {
+    "name": "ops_unary_f32", "rows": 1000, "cols": 200,
+    "inputs": [("x", "FULL", "F32")], "mask": None,
+    "ops": [("one", "const", 1.0), ("half", "const", 0.5), ("p15", "const", 1.5),
+            ("ax", "unary", "ABS", "x"), ("nx", "unary", "NEG", "x"),
+            ("ax1", "binary", "ADD", "ax", "one"), ("l", "unary", "LOG", "ax1"),
+            ("t", "unary", "TANH", "x"), ("er", "unary", "ERF", "x"), ("sq", "unary", "SQRT", "ax"),
+            ("x2", "binary", "MUL", "x", "x"), ("x21", "binary", "ADD", "x2", "one"), ("rs", "unary", "RSQRT", "x21"),
+            ("x2h", "binary", "ADD", "x2", "half"), ("rc", "unary", "RCP", "x2h"),
+            ("sg", "unary", "SIGMOID", "x"), ("ge", "unary", "GELU_ERF", "x"), ("gt", "unary", "GELU_TANH", "x"),
+            ("gg", "unary", "GELU_TANH_GRAD", "x"), ("e1", "unary", "EXP", "nx"),
+            ("axh", "binary", "ADD", "ax", "half"), ("pw", "binary", "POW", "axh", "p15")],
+    "outputs": [(n, "F32") for n in ("l", "t", "er", "sq", "rs", "rc", "sg", "ge", "gt", "gg", "e1", "pw")],
+}
+OPS_MIXED_F16 = {
+    "name": "ops_mixed_f16", "rows": 777, "cols": 96,
+    "inputs": [("x", "FULL", "F16"), ("v", "ROWVEC", "F16"), ("w", "COLVEC", "F16")], "mask": None,
+    "ops": [("one", "const", 1.0),
+            ("wb", "broadcast", "COL", "w"), ("vb", "broadcast", "ROW", "v"),
+            ("mn", "binary", "MIN", "x", "wb"), ("mx", "binary", "MAX", "x", "vb"),
+            ("v2", "binary", "MUL", "v", "v"), ("v21", "binary", "ADD", "v2", "one"), ("v21b", "broadcast", "ROW", "v21"),
+            ("dv", "binary", "DIV", "x", "v21b"), ("sg", "unary", "SIGMOID", "x"), ("rs", "reduce", "SUM", "ROW", "sg"),
+            ("aw", "unary", "ABS", "w"), ("w2", "unary", "SQRT", "aw"), ("rv", "unary", "TANH", "v"),
+            ("rm", "reduce", "RMAX", "ROW", "mn"), ("sub", "binary", "SUB", "mx", "mn")],
+    "outputs": [("mn", "F16"), ("mx", "F16"), ("dv", "F32"), ("rs", "F32"), ("w2", "F16"), ("rv", "F32"),
+                ("rm", "F32"), ("sub", "F16")],
+}
+
+
+def _subset(spec, names):
+    return dict(spec, outputs=[o for o in spec["outputs"] if o[0] in names])
+
+
+@pytest.mark.parametrize("spec,template", [
+    (OPS_UNARY, "row_stream"),                       # 12 live FULL outputs: streamed (scalar math)
+    (_subset(OPS_UNARY, ("l", "t", "er", "sq", "rs", "rc")), "row_team"),   # paired f32x2 math
+    (_subset(OPS_UNARY, ("sg", "ge", "gt", "gg", "e1", "pw")), "row_team"),
+    (OPS_MIXED_F16, "row_team")], ids=["unary_stream", "unary_a", "unary_b", "mixed_f16"])
+def test_parity_op_vocabulary(spec, template):
+    x = gen.generate("fig6a", spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    assert plan.describe()["mapping"]["template"] == template
+    _compare(spec, got, evaluate(spec, x))
+
+
+@pytest.mark.parametrize("cfg,rows,cols,world", [("C5", 3001, 1024, 2), ("C5", 4099, 256, 4), ("fig7a", 1001, 96, 2),
+                                                 ("C5int", 4096, 128, 2), ("bn", 1500, 64, 2)])
+def test_fused_exchange_virtual_ranks(cfg, rows, cols, world):
+    """astitch_run_fused (NEXT f1): every rank's ONE cooperative kernel pushes its
+    column totals into all ranks' exchange slots, flags them and combines the
+    slots in rank order.  Virtual ranks share one GPU (each plan sized for
+    148/world SMs so the kernels run together, one stream per rank); results
+    must match the oracle and be bitwise identical across ranks and runs."""
+    import torch
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import PeerExchange, ShardedPlan
+    from tests.harness import device_inputs, from_torch
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    x = gen.generate(cfg, spec)
+    g = A.Graph.from_spec(spec)
+    if cfg == "bn":  # two dependent column reductions: sharded plans support one level
+        with pytest.raises(A.AstitchError):
+            ShardedPlan(g, rows, cols, world, 0, 0)
+        return
+    ref = evaluate(spec, x)
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    ranks = []
+    for r in range(world):
+        sp = ShardedPlan(g, rows, cols, world, r, 0, sm_count=sms // world)
+        b, n = sp.row_begin, sp.row_count
+        xs = {k: (v[b:b + n] if getattr(v, "ndim", 0) == 2 or k == "p2" else v) for k, v in x.items()}
+        ins = device_inputs(dict(spec, rows=n), xs)
+        ranks.append([sp, ins, sp.plan.alloc_outputs(), sp.plan.alloc_workspace(), b, n, torch.cuda.Stream()])
+    for sp, *_ in ranks:
+        sp.peer = PeerExchange(sp.plan)
+    for sp, *_ in ranks:
+        for other, *_ in ranks:
+            if other is not sp:
+                sp.peer.link(other.rank, other.peer)
+    results = []
+    for it in range(3):
+        torch.cuda.synchronize()
+        for sp, ins, outs, ws, b, n, st in ranks:
+            sp.run(ins, outs, ws=ws, stream=st)
+        torch.cuda.synchronize()
+        for sp, *_ in ranks:
+            assert not sp.peer.timed_out(), "a rank's kernel timed out waiting for its peers"
+        got = {}
+        for name, _ in spec["outputs"]:
+            k = [o for o, _ in spec["outputs"]].index(name)
+            if ref[name].ndim == 2 or (ref[name].shape == (rows,)):
+                got[name] = np.concatenate([from_torch(rk[2][k]) for rk in ranks])
+            else:
+                vals = [from_torch(rk[2][k]) for rk in ranks]
+                for v in vals[1:]:
+                    assert np.array_equal(v, vals[0]), f"{name}: ranks disagree"
+                got[name] = vals[0]
+        results.append(got)
+    _compare(spec, results[0], ref)
+    for k in results[0]:
+        assert np.array_equal(results[0][k], results[1][k]) and np.array_equal(results[0][k], results[2][k])
+    if cfg == "C5int":
+        np.testing.assert_array_equal(results[0]["db"], ref["db"])
+    assert ranks[0][0].kernels_per_run() == 1
