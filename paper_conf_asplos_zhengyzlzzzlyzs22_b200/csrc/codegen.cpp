@@ -1692,6 +1692,9 @@ struct Gen {
     if (m.tmpl == Template::GlobalSweep) {
       o << "  unsigned int* bar = (unsigned int*)((char*)p.ws + " << p.ws.barrier << "LL);\n  (void)bar;\n";
     }
+    if (role == ROLE_FUSED)  // this run's wait status (set only after the grid barriers below)
+      o << "  if (blockIdx.x == 0 && threadIdx.x == 0) *(volatile unsigned int*)((unsigned char*)p.xbuf + " << kXErr
+        << ") = 0u;\n";
     if (role == ROLE_SHARD_SWEEP2) {  // sharded plans have one barrier level
       cur_level = 1;
       emit_colvecs(false);

@@ -182,6 +182,22 @@ astitch_status astitch_peer_create(astitch_plan_t h, astitch_peer_t* out, uint8_
   const Plan& p = *h->p;
   if (p.device < 0) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "host-only plan");
   if (p.desc.shard_world > 64) return fail(ASTITCH_ERR_UNSUPPORTED, "fused exchange supports up to 64 ranks");
+  // compile + load the fused kernel now: ranks must not JIT at different
+  // times inside the first exchange (a late peer looks like a missing one)
+  Plan& pm = *h->p;
+  if (!pm.colreds.empty() && pm.desc.shard_world > 1 && pm.fused_kernels.empty()) {
+    pm.fused_kernels.resize(1);
+    astitch_status s = build_plan_kernel(pm, ROLE_FUSED, pm.fused_kernels[0]);
+    std::string e2;
+    if (s == ASTITCH_OK && !pm.fused_kernels[0].module && !drv_load(pm, pm.fused_kernels[0], e2))
+      s = fail(ASTITCH_ERR_CUDA, e2);
+    if (s != ASTITCH_OK) {
+      pm.fused_kernels.clear();
+      return s;
+    }
+    Kernel& k = pm.fused_kernels[0];
+    k.grid = std::min<int64_t>(k.grid, static_cast<int64_t>(k.occupancy) * pm.sm_count);
+  }
   auto* x = new astitch_peer_s();
   x->world = p.desc.shard_world;
   x->rank = p.desc.shard_rank;

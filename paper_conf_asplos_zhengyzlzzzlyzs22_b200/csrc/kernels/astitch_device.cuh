@@ -485,16 +485,21 @@ __device__ __forceinline__ unsigned int ld_acquire_sys(const unsigned int* p) {
   asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 // Wait (thread 0 of a block) until every rank's flag holds `gen`; bounded
-// (~2 s) so a missing rank cannot hang the GPU: on timeout the error word is
-// set and the caller proceeds with whatever the slots hold.
+// (5 s of wall time) so a missing rank cannot hang the GPU: on timeout the
+// error word is set and the caller proceeds with whatever the slots hold.
 __device__ __forceinline__ void wait_flags(const unsigned int* flags, int world, unsigned int gen,
                                            unsigned int* err) {
-  long long spins = 0;
+  const unsigned long long t0 = globaltimer_ns();
   for (int q = 0; q < world; ++q) {
     while (ld_acquire_sys(flags + q) != gen) {
-      if (++spins > (1LL << 21)) { atomicOr(err, 1u); return; }
-      __nanosleep(100);
+      if (globaltimer_ns() - t0 > 5000000000ULL) { atomicOr(err, 1u); return; }
+      __nanosleep(200);
     }
   }
 }

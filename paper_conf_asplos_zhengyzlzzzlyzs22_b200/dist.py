@@ -92,7 +92,7 @@ class PeerExchange:
 
     def __del__(self):
         h = getattr(self, "_h", None)
-        if h is not None and h.value:
+        if h is not None and h.value and lib is not None:
             lib.astitch_peer_destroy(h)
             self._h = None
 
