@@ -91,6 +91,9 @@ def run_gpu(spec: dict, inputs: dict, flags: int = 0, plan=None, return_plan=Fal
         plan = A.Plan(g, spec["rows"], spec["cols"], device=torch.cuda.current_device(), flags=flags)
     ins = device_inputs(spec, inputs)
     outs = plan.alloc_outputs()
+    if spec.get("segments"):  # packed rows: elements past a row's 16-byte chunks are never written
+        for o in outs:
+            o.zero_()
     plan.run(ins, outs)
     torch.cuda.synchronize()
     res = {n: from_torch(t) for (n, _), t in zip(spec["outputs"], outs)}

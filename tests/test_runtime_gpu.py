@@ -180,3 +180,27 @@ def test_sharded_world1_equals_run():
     torch.cuda.synchronize()
     for (name, _), t in zip(spec["outputs"], outs):
         assert np.array_equal(from_torch(t), ref[name])
+
+
+def test_peer_exchange_misuse_errors():
+    import torch
+    """astitch_peer_* / astitch_run_fused argument checks (ERR_INVALID_ARGUMENT)."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import PeerExchange, ShardedPlan
+    from workloads import specs
+    spec = specs.get("C5", rows=1000, cols=64)
+    g = A.Graph.from_spec(spec)
+    s0, s1 = ShardedPlan(g, 1000, 64, 2, 0, 0), ShardedPlan(g, 1000, 64, 2, 1, 0)
+    x0, x1 = PeerExchange(s0.plan), PeerExchange(s1.plan)
+    with pytest.raises(A.AstitchError):
+        x0.link(0, x1)                    # x1 is rank 1, not 0
+    with pytest.raises(A.AstitchError):
+        x0.link(5, x1)                    # rank out of range
+    ins = [torch.zeros(s0.row_count, 64, dtype=torch.bfloat16, device="cuda"),
+           torch.zeros(s0.row_count, 64, dtype=torch.bfloat16, device="cuda"), torch.zeros(64, device="cuda")]
+    s0.peer = x0
+    with pytest.raises(A.AstitchError):   # peer 1 not mapped yet
+        s0.run(ins, s0.plan.alloc_outputs())
+    other = ShardedPlan(A.Graph.from_spec(specs.get("C5", rows=1000, cols=128)), 1000, 128, 2, 1, 0)
+    with pytest.raises(A.AstitchError):   # different plan (cols): buffer sizes differ
+        x0.link(1, PeerExchange(other.plan))
