@@ -1468,6 +1468,35 @@ struct Gen {
       rl[i] = lv;
     }
   }
+  // values pass `pass` of a streamed row needs: its reductions' operands and
+  // its FULL outputs, closed backwards over FULL values; COLVEC operands in *cv
+  std::vector<bool> stream_need(int pass, int n, std::vector<bool>* cv = nullptr) const {
+    std::vector<bool> need(n, false), need_cv(n, false);
+    for (int i = 0; i < n; ++i)
+      if (I(i).live && I(i).cls == OpClass::ReduceRow && rl[i] == pass) need[N(i).a] = true;
+    for (size_t k = 0; k < g.outputs.size(); ++k)
+      if (N(g.outputs[k]).kind == ASTITCH_FULL && rl[g.outputs[k]] == pass) need[g.outputs[k]] = true;
+    for (int i = n - 1; i >= 0; --i) {
+      if (!need[i]) continue;
+      const Node& nd = N(i);
+      if (nd.type == NodeType::Bcast) {
+        if (nd.axis == ASTITCH_AXIS_COL) need_cv[nd.a] = true;
+        continue;
+      }
+      for (int a : {nd.a, nd.b}) {
+        if (a < 0) continue;
+        if (N(a).kind == ASTITCH_FULL) need[a] = true;
+        else if (N(a).kind == ASTITCH_COLVEC) need_cv[a] = true;
+      }
+    }
+    for (int i = n - 1; i >= 0; --i)  // COLVEC closure
+      if (need_cv[i])
+        for (int a : {N(i).a, N(i).b})
+          if (a >= 0 && N(a).kind == ASTITCH_COLVEC) need_cv[a] = true;
+    if (cv) *cv = need_cv;
+    return need;
+  }
+
   // ROWVEC value i (not an input) computed from row scalars
   void emit_stream_rowvec(int i) {
     const Node& nd = N(i);
@@ -1504,8 +1533,30 @@ struct Gen {
         << "];\n";
     }
     emit_pre_colvec_outputs();
+    // (staged rows) first pass that reads each FULL input: it loads from HBM
+    // and keeps the lane's raw chunks in smem for the later passes
+    std::vector<int> first_pass(n, -1);
+    std::vector<long long> soff(fin.size(), 0);
+    if (m.stage_row) {
+      o << "  extern __shared__ __align__(16) unsigned char smem[];\n";
+      o << "  const u32 sbase = as::smem_addr(smem);\n";
+    }
     o << "  constexpr long long TCH = (long long)T * V;            // chunks per tile\n";
     o << "  constexpr long long NT = (CH + TCH - 1) / TCH;          // tiles per row\n";
+    if (m.stage_row) {
+      const long long tch = static_cast<long long>(m.team) * V;
+      const long long nt = (C / E + tch - 1) / tch;
+      long long off = 0;
+      for (size_t s = 0; s < fin.size(); ++s) {
+        soff[s] = off;
+        off += nt * V * m.threads * nb(N(fin[s]).dtype);
+      }
+      for (int pass = 0; pass < P; ++pass) {
+        std::vector<bool> need = stream_need(pass, n);
+        for (size_t s = 0; s < fin.size(); ++s)
+          if (need[fin[s]] && first_pass[fin[s]] < 0) first_pass[fin[s]] = pass;
+      }
+    }
     o << "  for (long long row = UNIT; row < (long long)R; row += NUNITS) {\n";
     // ROWVEC inputs and level-0 row scalars
     for (int id : g.inputs)
@@ -1522,35 +1573,16 @@ struct Gen {
     for (int pass = 0; pass < P; ++pass) {
       // what this pass needs: its reductions' operands and its FULL outputs,
       // closed backwards over FULL values (row / column scalars are at hand)
-      std::vector<bool> need(n, false);
+      std::vector<bool> need_cv;
+      std::vector<bool> need = stream_need(pass, n, &need_cv);
       std::vector<int> reds;
-      for (int i = 0; i < n; ++i) {
-        if (!I(i).live) continue;
-        if (I(i).cls == OpClass::ReduceRow && rl[i] == pass) { reds.push_back(i); need[N(i).a] = true; }
-      }
+      for (int i = 0; i < n; ++i)
+        if (I(i).live && I(i).cls == OpClass::ReduceRow && rl[i] == pass) reds.push_back(i);
       std::vector<int> fouts;
       for (size_t k = 0; k < g.outputs.size(); ++k) {
         int id = g.outputs[k];
-        if (N(id).kind == ASTITCH_FULL && rl[id] == pass) { need[id] = true; fouts.push_back(static_cast<int>(k)); }
+        if (N(id).kind == ASTITCH_FULL && rl[id] == pass) fouts.push_back(static_cast<int>(k));
       }
-      std::vector<bool> need_cv(n, false);
-      for (int i = n - 1; i >= 0; --i) {
-        if (!need[i]) continue;
-        const Node& nd = N(i);
-        if (nd.type == NodeType::Bcast) {
-          if (nd.axis == ASTITCH_AXIS_COL) need_cv[nd.a] = true;
-          continue;
-        }
-        for (int a : {nd.a, nd.b}) {
-          if (a < 0) continue;
-          if (N(a).kind == ASTITCH_FULL) need[a] = true;
-          else if (N(a).kind == ASTITCH_COLVEC) need_cv[a] = true;
-        }
-      }
-      for (int i = n - 1; i >= 0; --i)  // COLVEC closure
-        if (need_cv[i])
-          for (int a : {N(i).a, N(i).b})
-            if (a >= 0 && N(a).kind == ASTITCH_COLVEC) need_cv[a] = true;
       o << "    // ---- pass " << pass << ": " << reds.size() << " row reduction(s), " << fouts.size()
         << " FULL output(s)\n";
       for (int r : reds) {
@@ -1567,7 +1599,19 @@ struct Gen {
         o << "      " << rt << " r" << s << "[V];\n";
         o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
         o << "        const long long ch = t * TCH + j * T + lane;\n";
-        o << "        r" << s << "[j] = (ch < CH) ? as::ldg(gs" << s << " + row * CH + ch) : " << rt << "{};\n";
+        if (m.stage_row) {
+          const int nbs = nb(N(id).dtype);
+          o << "        const u32 sa = sbase + (u32)(" << soff[s] << "LL + ((t * V + j) * (long long)blockDim.x + threadIdx.x) * "
+            << nbs << ");\n";
+          if (first_pass[id] == pass) {
+            o << "        r" << s << "[j] = (ch < CH) ? as::ldg(gs" << s << " + row * CH + ch) : " << rt << "{};\n";
+            o << "        if (ch < CH) as::sts_chunk<" << nbs << ">(sa, r" << s << "[j]);  // stage for later passes\n";
+          } else {
+            o << "        r" << s << "[j] = (ch < CH) ? as::lds_chunk<" << nbs << ">(sa) : " << rt << "{};\n";
+          }
+        } else {
+          o << "        r" << s << "[j] = (ch < CH) ? as::ldg(gs" << s << " + row * CH + ch) : " << rt << "{};\n";
+        }
         o << "      }\n";
         o << "      float v" << id << "[NE];\n";
         o << "#pragma unroll\n      for (int j = 0; j < V; ++j) as::Conv<" << dt_code(N(id).dtype) << ", E>::unpack(r" << s

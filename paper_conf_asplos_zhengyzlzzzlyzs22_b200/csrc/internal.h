@@ -104,6 +104,7 @@ struct Mapping {
   int tile_rows = 0;        // PackedTile rows per stage
   int stages = 0;           // PackedTile pipeline stages
   int split = 1;            // CTAs per row (task splitting; 1 = none)
+  bool stage_row = false;   // row_stream: the row's inputs staged in shared memory (regional)
   int64_t grid = 1;
   int blocks_per_sm = 1;    // assume-relax-apply target
   int reg_cap = 255;

@@ -603,15 +603,42 @@ void select_mapping(Plan& p) {
         while (k < want && k < 8) k *= 2;
         m.split = k;
       }
-      m.team = m.split * m.threads;
       m.chunks_per_lane = std::max(1, 32 / E);  // V: 32 values per lane per tile
+      // Regional stitching proper: when the row's inputs fit the
+      // shared memory of a cluster (<= 160 KB per CTA, <= 8 CTAs), the first
+      // pass that reads an input stages the lane's raw chunks in its CTA's
+      // smem and the later passes re-read them from there (each lane reads
+      // back only its own chunks: no barrier); else the passes re-read L2/HBM.
+      int in_row_bytes = 0;
+      for (int id : g.inputs)
+        if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live)
+          in_row_bytes += static_cast<int>(std::min<int64_t>(C * dtype_size(g.nodes[id].dtype), 1 << 30));
+      const bool no_stage = getenv("ASTITCH_NO_STAGE") && atoi(getenv("ASTITCH_NO_STAGE")) == 1;
+      m.stage_row = false;
+      m.smem_bytes = 0;
+      if (!no_stage && in_row_bytes > 0) {
+        int k = m.split;
+        while (k < 8 && (in_row_bytes + k - 1) / k > 160 * 1024) k *= 2;
+        if ((in_row_bytes + k - 1) / k <= 160 * 1024 && !(no_split && k > 1)) {
+          m.split = k;
+          m.stage_row = true;
+          const int64_t tch = static_cast<int64_t>(k) * m.threads * m.chunks_per_lane;
+          const int64_t nt = (m.chunks + tch - 1) / tch;
+          int64_t sm = 0;
+          for (int id : g.inputs)
+            if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live)
+              sm += nt * m.chunks_per_lane * m.threads * E * dtype_size(g.nodes[id].dtype);
+          m.smem_bytes = static_cast<int>(sm);
+        }
+      }
+      m.team = m.split * m.threads;
       m.lane_util = 1.0;
       m.rows_per_block = 1;
       m.row_unroll = 1;
       m.prefetch = false;
       why << "row of " << C << " exceeds the team's registers -> streamed in tiles of " << m.team << " lanes x "
           << m.chunks_per_lane << " chunks" << (m.split > 1 ? " over a cluster of " + std::to_string(m.split) + " CTAs" : "")
-          << ", one pass per row-reduction level; ";
+          << ", one pass per row-reduction level" << (m.stage_row ? ", inputs staged in shared memory" : "") << "; ";
     }
   }
 
@@ -802,7 +829,8 @@ std::string describe_json(const Plan& p) {
     << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
     << ",\"prefetch\":" << (m.prefetch ? "true" : "false")
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
-    << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"grid\":" << m.grid
+    << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
+    << ",\"grid\":" << m.grid
     << ",\"blocks_per_sm\":" << m.blocks_per_sm << ",\"reg_cap\":" << m.reg_cap
     << ",\"vertical_trips\":" << m.vertical_trips << ",\"smem_bytes\":" << m.smem_bytes
     << ",\"lds128_conflict_ways\":" << m.bank_conflict_ways << ",\"reason\":\"" << esc(m.reason)

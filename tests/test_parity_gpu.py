@@ -353,7 +353,9 @@ def test_one_kernel_no_memset_per_run(cfg):
                                                  ("fig5", None, None, True), ("remote", None, None, True),
                                                  ("C4", 37, 5000, True), ("fig6b", 64, 300000, True),
                                                  ("C1", 16, 2_000_000, False), ("C4", 8, 1_000_003, False),
-                                                 ("fig6b", 3, 4_000_000, False)])
+                                                 ("fig6b", 3, 4_000_000, False),
+                                                 ("lmsoftmax", 64, None, False), ("C1", 37, 100_000, False),
+                                                 ("C2", 40, 100_000, False)])
 def test_parity_row_stream(cfg, rows, cols, force, monkeypatch):
     """Rows longer than a team's registers: streamed column tiles, one pass per
     row-reduction level (forced on small shapes; chosen by the planner for

@@ -310,6 +310,19 @@ BN_TRAIN_FWD = {
     "outputs": [("y", "F32"), ("mean", "F32"), ("var", "F32")],
 }
 
+# LM-head softmax over a 128K vocabulary, bf16 [4096 tokens, 128256]: rows of
+# 256 KB, longer than any team's registers -> the row_stream template (one
+# pass per row-reduction level: max | sum | normalise).
+LM_SOFTMAX = {
+    "name": "lm_head_softmax_bf16_4096x128256",
+    "rows": 4096,
+    "cols": 128256,
+    "inputs": [("x", "FULL", "BF16")],
+    "mask": None,
+    "ops": [op for op in C1_SOFTMAX["ops"]],
+    "outputs": [("y", "BF16")],
+}
+
 # Remote stitching: two subgraphs with no data dependency merged into
 # one stitch op (the "independent" scheme between them), one kernel.
 REMOTE_TWO_SUBGRAPHS = {
@@ -350,6 +363,7 @@ EXTRA = {
     "fig6b": FIG6B_FEW_LONG_ROWS,
     "remote": REMOTE_TWO_SUBGRAPHS,
     "bn": BN_TRAIN_FWD,
+    "lmsoftmax": LM_SOFTMAX,
 }
 
 ALL = {**CONFIGS, **EXTRA}
