@@ -613,13 +613,20 @@ void select_mapping(Plan& p) {
       for (int id : g.inputs)
         if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live)
           in_row_bytes += static_cast<int>(std::min<int64_t>(C * dtype_size(g.nodes[id].dtype), 1 << 30));
-      const bool no_stage = getenv("ASTITCH_NO_STAGE") && atoi(getenv("ASTITCH_NO_STAGE")) == 1;
+      // Measured on B200 (LM-head softmax 4096 x 128256 bf16: 741 us staged vs
+      // 660 us re-reading L2; fp32 4096 x 100000: 1896 vs 1049 us): staging
+      // costs occupancy (one 512-thread CTA per SM) that the L2-resident
+      // re-reads do not, so it is opt-in (ASTITCH_STAGE=1) until the staged
+      // pass pipelines its loads.
+      const bool no_stage = !(getenv("ASTITCH_STAGE") && atoi(getenv("ASTITCH_STAGE")) == 1);
       m.stage_row = false;
       m.smem_bytes = 0;
+      int stage_budget = 72 * 1024;  // per CTA: keeps 3 CTAs of 512 threads per SM
+      if (const char* sb = getenv("ASTITCH_STAGE_KB")) stage_budget = std::max(8, atoi(sb)) * 1024;
       if (!no_stage && in_row_bytes > 0) {
         int k = m.split;
-        while (k < 8 && (in_row_bytes + k - 1) / k > 160 * 1024) k *= 2;
-        if ((in_row_bytes + k - 1) / k <= 160 * 1024 && !(no_split && k > 1)) {
+        while (k < 8 && (in_row_bytes + k - 1) / k > stage_budget) k *= 2;
+        if ((in_row_bytes + k - 1) / k <= stage_budget && !(no_split && k > 1)) {
           m.split = k;
           m.stage_row = true;
           const int64_t tch = static_cast<int64_t>(k) * m.threads * m.chunks_per_lane;

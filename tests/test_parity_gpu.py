@@ -354,20 +354,24 @@ def test_one_kernel_no_memset_per_run(cfg):
                                                  ("C4", 37, 5000, True), ("fig6b", 64, 300000, True),
                                                  ("C1", 16, 2_000_000, False), ("C4", 8, 1_000_003, False),
                                                  ("fig6b", 3, 4_000_000, False),
-                                                 ("lmsoftmax", 64, None, False), ("C1", 37, 100_000, False),
-                                                 ("C2", 40, 100_000, False)])
+                                                 ("lmsoftmax", 64, None, False), ("C1", 37, 600_000, False),
+                                                 ("lmsoftmax", 64, None, "stage"), ("C2", 40, 100_000, "stage"),
+                                                 ("C4", 300, 60_000, "stage")])
 def test_parity_row_stream(cfg, rows, cols, force, monkeypatch):
     """Rows longer than a team's registers: streamed column tiles, one pass per
     row-reduction level (forced on small shapes; chosen by the planner for
-    multi-MB rows)."""
-    if force:
+    multi-MB rows; "stage": inputs kept in the cluster's shared memory)."""
+    if force is True:
         monkeypatch.setenv("ASTITCH_FORCE_STREAM", "1")
+    if force == "stage":
+        monkeypatch.setenv("ASTITCH_STAGE", "1")
     spec = specs.get(cfg, rows=rows, cols=cols)
     x = gen.generate(cfg, spec)
     got, plan = run_gpu(spec, x, return_plan=True)
     d = plan.describe()
     assert d["mapping"]["template"] == "row_stream" and d["kernel_count"] == 1
     assert d["kernels"][0]["spill_bytes"] == 0
+    assert d["mapping"]["stage_row"] == (force == "stage")
     _compare(spec, got, evaluate(spec, x))
     again = run_gpu(spec, x, plan=plan)
     for k in got:
