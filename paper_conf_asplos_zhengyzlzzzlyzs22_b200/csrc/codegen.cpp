@@ -582,6 +582,7 @@ struct Gen {
           body = "v" + id + sfx + "[k] = " + expr + ";";
         }
         const std::string estep = paired ? "e += 2" : "++e";
+        if (row_div(i)) o << "    " << row_div_decl(i, sfx) << "\n";
         o << "    float v" << id << sfx << "[NE];\n";
         if (masked) {
           // chunks wholly past the valid length are not computed (team-uniform branch)
@@ -745,6 +746,7 @@ struct Gen {
       }
     }
     if (nd.type == NodeType::Unary) return unop2(nd.sub, ref2(nd.a, sfx));
+    if (row_div(i)) return "as::mul2(" + ref2(nd.a, sfx) + ", as::bc2(rq" + std::to_string(i) + sfx + "))";
     std::string a = ref2(nd.a, sfx), b = ref2(nd.b, sfx);
     auto lo = [&](int v) { return "as::bc2(s" + std::to_string(N(v).a) + sfx + "lo)"; };
     if (nd.sub == ASTITCH_SUB && precise_bcast(nd.b)) return "as::sub2(as::sub2(" + a + ", " + b + "), " + lo(nd.b) + ")";
@@ -784,9 +786,21 @@ struct Gen {
       }
     }
     if (nd.type == NodeType::Unary) return unop(nd.sub, ref(nd.a, "k", sfx));
+    if (row_div(i)) return "(" + ref(nd.a, "k", sfx) + " * rq" + std::to_string(i) + sfx + ")";
     return full_binop(nd, sfx);
   }
 
+  // x / bcast_row(s): multiply by the row's reciprocal, computed once per
+  // row (rq<i>) instead of a MUFU.RCP per element (same arithmetic as fdiv)
+  bool row_div(int i) const {
+    const Node& nd = N(i);
+    if (nd.type != NodeType::Binary || nd.sub != ASTITCH_DIV || nd.kind != ASTITCH_FULL) return false;
+    const Node& b = N(nd.b);
+    return b.type == NodeType::Bcast && b.axis == ASTITCH_AXIS_ROW && !precise[b.a];
+  }
+  std::string row_div_decl(int i, const std::string& sfx) const {
+    return "const float rq" + std::to_string(i) + sfx + " = as::rcp(s" + std::to_string(N(N(i).b).a) + sfx + ");";
+  }
   bool precise_bcast(int v) const {
     const Node& nd = N(v);
     return nd.type == NodeType::Bcast && nd.axis == ASTITCH_AXIS_ROW && precise[nd.a];
@@ -1641,6 +1655,7 @@ struct Gen {
         if (!need[i] || !I(i).live || nd.kind != ASTITCH_FULL || nd.type == NodeType::Input ||
             nd.type == NodeType::Bcast)
           continue;
+        if (row_div(i)) o << "      " << row_div_decl(i, "") << "\n";
         o << "      float v" << i << "[NE];\n";
         o << "#pragma unroll\n      for (int k = 0; k < NE; ++k) v" << i << "[k] = " << full_expr(i, "") << ";\n";
       }
