@@ -9,7 +9,9 @@ on [1,048,576, 1024] bf16 (dz = dy * gelu'(z); db = col_sum(dz);
 b_new = b - 2^-7 db) — the config the metric is quoted on at 1/2/4/8 GPUs, run
 as ONE stitched kernel with global stitching (grid barrier).  At N > 1 the
 rows are sharded contiguously (strong scaling of the fixed problem) and the
-column partials are combined with one NCCL allreduce.
+column partials are exchanged inside the stitched kernel over peer memory
+(`--exchange fused`, default) or with one NCCL allreduce + epilogue
+(`--exchange nccl`, also the fallback when peer access is unavailable).
 
 A "step" is one execution of the whole subgraph (one astitch_run /
 astitch_run_sharded) over the resident synthetic inputs.  Timing: W warm-up

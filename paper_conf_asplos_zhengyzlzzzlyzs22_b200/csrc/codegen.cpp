@@ -329,15 +329,32 @@ struct Gen {
     }
   }
 
+  // unpack = convert (raw vectors -> fp32 registers) + mask (absorbed
+  // substitute for invalid elements).  The early-unpack row loop emits the
+  // convert step before the next row's prefetch is issued (the raw registers
+  // die there, so the prefetch reuses them: no register copies) and the
+  // mask step later, inside the (possibly KF-specialised) row block.
+  bool early_unpack = false;   // convert already emitted for the current row
   void emit_unpack(const std::string& sfx, const std::string& lim = "") {
+    if (!early_unpack) emit_unpack_convert(sfx, sfx);
+    emit_unpack_mask(sfx, lim);
+  }
+  void emit_unpack_convert(const std::string& sfx, const std::string& src) {
     for (size_t s = 0; s < streams.size(); ++s) {
       const Stream& st = streams[s];
       int id = st.node;
       std::string dst = "v" + std::to_string(id) + sfx;
       int dt = st.ws_buf ? 0 : dt_code(st.dt);
       o << "    float " << dst << "[NE];\n";
-      o << "#pragma unroll\n    for (int j = 0; j < V; ++j) as::Conv<" << dt << ", E>::unpack(r" << s << sfx
+      o << "#pragma unroll\n    for (int j = 0; j < V; ++j) as::Conv<" << dt << ", E>::unpack(r" << s << src
         << "[j], " << dst << " + j * E);\n";
+    }
+  }
+  void emit_unpack_mask(const std::string& sfx, const std::string& lim) {
+    for (size_t s = 0; s < streams.size(); ++s) {
+      const Stream& st = streams[s];
+      int id = st.node;
+      std::string dst = "v" + std::to_string(id) + sfx;
       if (absorb && masked && !st.ws_buf && !lim.empty()) {
         // mask absorption: invalid elements take the substitute value
         // d_ = elements of this lane's chunk that are valid (may be <= 0)
@@ -397,6 +414,39 @@ struct Gen {
       case ASTITCH_POW: return std::pow(a, b);
       default: return std::nan("");
     }
+  }
+
+  // a FULL value whose (transitive) consumers include a reduction
+  bool feeds_reduction(int i) const {
+    for (int u : I(i).consumers) {
+      if (!I(u).live) continue;
+      const Node& un = N(u);
+      if (un.type == NodeType::Reduce) return true;
+      if (un.kind == ASTITCH_FULL && feeds_reduction(u)) return true;
+    }
+    return false;
+  }
+  static bool env_on(const char* name) { return getenv(name) && atoi(getenv(name)) == 1; }
+  // FULL light op computed over every chunk of an absorbed-mask row (no
+  // live-chunk branch): its invalid elements take the known value inval[i]
+  // whenever the row's scalars are finite, i.e. whenever the row has a valid
+  // prefix; no reduction reads it (so fully-masked rows cannot leak a NaN into
+  // a row scalar) and it is not buffered across a barrier
+  bool light_unguarded(int i) const {
+    if (!absorb || kf || !inval_known[i] || env_on("ASTITCH_GUARD_LIGHT")) return false;
+    const Node& nd = N(i);
+    bool light = false;
+    if (nd.type == NodeType::Binary)
+      light = nd.sub == ASTITCH_ADD || nd.sub == ASTITCH_SUB || nd.sub == ASTITCH_MUL || nd.sub == ASTITCH_MAX ||
+              nd.sub == ASTITCH_MIN || row_div(i) || (nd.sub == ASTITCH_DIV && N(nd.b).type == NodeType::Const);
+    else if (nd.type == NodeType::Unary)
+      light = nd.sub == ASTITCH_NEG || nd.sub == ASTITCH_ABS;
+    return light && !feeds_reduction(i) && !I(i).global_full;
+  }
+  // FULL output whose invalid elements are known to be exactly 0 under the
+  // absorbed mask: stored without per-element selects
+  bool store_absorbed(int id) const {
+    return absorb && masked && inval_known[id] && inval[id] == 0.0 && !env_on("ASTITCH_STORE_SELECT");
   }
 
   // abstract evaluation for substitute S; returns true if every row (and
@@ -584,7 +634,12 @@ struct Gen {
         const std::string estep = paired ? "e += 2" : "++e";
         if (row_div(i)) o << "    " << row_div_decl(i, sfx) << "\n";
         o << "    float v" << id << sfx << "[NE];\n";
-        if (masked) {
+        if (masked && light_unguarded(i)) {
+          // absorbed mask, light op that no reduction reads: past the valid
+          // length it computes its known invalid value anyway, cheaper than a
+          // branch per chunk plus a zero fill
+          o << "#pragma unroll\n    for (int k = 0; k < NE; k += " << (paired ? 2 : 1) << ") " << body << "\n";
+        } else if (masked) {
           // chunks wholly past the valid length are not computed (team-uniform branch)
           o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n      if (" << live_pred(lim) << ") {\n";
           o << "#pragma unroll\n        for (int e = 0; e < E; " << estep << ") { const int k = j * E + e; " << body
@@ -848,10 +903,26 @@ struct Gen {
         std::string rt = "as::Raw<" + std::to_string(nb(dt)) + ">";
         o << "    if (" << act << ") {\n      " << rt << "* __restrict__ op_ = (" << rt << "*)p.out[" << k
           << "] + " << rowbase(row, lim) << ";\n";
-        o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
         std::string val = ref(id, "(j * E + e)", sfx);
+        const std::string cguard = exact ? "" : "        if ((long long)(j * T + lane) < CH)\n";
+        if (store_absorbed(id) && !ragged) {
+          // every invalid element already holds 0 (absorbed mask): no
+          // per-element selects; fully-masked rows (the only ones whose row
+          // scalars may be non-finite) store zeros on a team-uniform branch
+          o << "      if (" << lim << " > 0) {\n#pragma unroll\n      for (int j = 0; j < V; ++j) {\n        float t_[E];\n"
+            << "#pragma unroll\n        for (int e = 0; e < E; ++e) t_[e] = " << val << ";\n"
+            << cguard << "        as::stg(op_ + (j * T + lane), as::Conv<" << dt_code(dt) << ", E>::pack(t_));\n"
+            << "      }\n      } else {\n#pragma unroll\n      for (int j = 0; j < V; ++j) {\n"
+            << cguard << "        as::stg(op_ + (j * T + lane), " << rt << "{});\n      }\n      }\n    }\n";
+          continue;
+        }
+        o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
         o << "        float t_[E];\n";
-        if (masked) {
+        if (store_absorbed(id)) {
+          // packed varlen rows: only the row's own chunks are stored, and
+          // its invalid tail elements already hold 0
+          o << "#pragma unroll\n        for (int e = 0; e < E; ++e) t_[e] = " << val << ";\n";
+        } else if (masked) {
           o << "        if (" << full_pred(lim) << ") {\n#pragma unroll\n          for (int e = 0; e < E; ++e) t_[e] = "
             << val << ";\n        } else {\n#pragma unroll\n          for (int e = 0; e < E; ++e) t_[e] = ("
             << col_expr("j", "e") << " < " << lim << ") ? " << val << " : 0.f;\n        }\n";
@@ -1024,7 +1095,18 @@ struct Gen {
                            (ragged && pf) ? "nsg" + std::to_string(u) : "") << "\n";
       o << "    (void)lim" << u << ";\n";
     }
-    if (pf) {
+    // early unpack (default): convert the prefetched raw vectors to fp32
+    // before the next prefetch is issued into the same registers.  The copy
+    // form (ASTITCH_LATE_UNPACK=1) keeps a raw copy live across the prefetch;
+    // on B200 its register moves stall on the loads of the next row
+    // (long scoreboard at the loop back-edge, C3 ncu source view).
+    const bool early = pf && !(getenv("ASTITCH_LATE_UNPACK") && atoi(getenv("ASTITCH_LATE_UNPACK")) == 1);
+    if (pf && early) {
+      for (int u = 0; u < U; ++u) {
+        std::string s = su + std::to_string(u);
+        emit_unpack_convert(s, s + "n");
+      }
+    } else if (pf) {
       for (int u = 0; u < U; ++u) {
         std::string s = su + std::to_string(u);
         for (size_t q = 0; q < streams.size(); ++q) {
@@ -1032,6 +1114,8 @@ struct Gen {
           o << "#pragma unroll\n    for (int j = 0; j < V; ++j) r" << q << s << "[j] = r" << q << s << "n[j];\n";
         }
       }
+    }
+    if (pf) {
       for (int u = 0; u < U; ++u) {
         std::string s = su + std::to_string(u) + "n";
         o << "    {\n";
@@ -1049,11 +1133,13 @@ struct Gen {
         emit_loads("row" + std::to_string(u), "act" + std::to_string(u), "lim" + std::to_string(u), s, true);
       }
     }
+    early_unpack = pf && early;
     for (int u = 0; u < U; ++u) {
       std::string s = su + std::to_string(u);
       std::string row = "row" + std::to_string(u), act = "act" + std::to_string(u), lim = "lim" + std::to_string(u);
       emit_row_block(post, s, row, act, lim);
     }
+    early_unpack = false;
     o << "  }\n";
   }
 
