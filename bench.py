@@ -353,6 +353,8 @@ def main():
     for i in range(args.warmup):
         step(i)
     torch.cuda.synchronize()
+    if sp.peer is not None:
+        exchange = check_fused_exchange(sp, dev_in[0], plan, ws, exchange)
 
     # copy-kernel ceiling on the same number of bytes (practical roofline)
     half = (nbytes // 2) // 16 * 16
@@ -527,6 +529,36 @@ def main():
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def check_fused_exchange(sp, inputs, plan, ws, exchange):
+    """N>1 safety net for the in-kernel exchange: run the step once fused and
+    once through ncclAllReduce + epilogue on the same inputs and compare every
+    output (the fused combine sums the ranks in a fixed order, NCCL in its own:
+    equal within fp32 reassociation).  A bounded-wait timeout or a mismatch on
+    any rank switches every rank to the NCCL exchange."""
+    import torch
+    import torch.distributed as dist
+    out_f, out_n = plan.alloc_outputs(), plan.alloc_outputs()
+    sp.run(inputs, out_f, ws=ws)
+    torch.cuda.synchronize()
+    bad = 1.0 if sp.peer.timed_out() else 0.0
+    peer, sp.peer = sp.peer, None
+    sp.run(inputs, out_n, ws=ws)
+    torch.cuda.synchronize()
+    sp.peer = peer
+    for a, b in zip(out_f, out_n):
+        a, b = a.float(), b.float()
+        scale = float(b.pow(2).mean().sqrt()) if b.numel() else 0.0
+        if not bool(torch.isfinite(a).all()) or float((a - b).abs().max()) > 1e-5 * max(scale, 1e-30) + 1e-30:
+            bad = 1.0
+    flag = torch.tensor([bad], device=out_f[0].device)
+    dist.all_reduce(flag, op=dist.ReduceOp.MAX)
+    if float(flag.item()) > 0:
+        print("[bench] fused exchange failed its check against NCCL; using NCCL", file=sys.stderr)
+        sp.peer = None
+        return "ncclAllReduce + epilogue (fused exchange failed its check)"
+    return exchange + ", checked against NCCL"
 
 
 def _sharded_host(sp, host_in, host_out, dev_in, dev_out, ws):
