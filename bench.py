@@ -434,6 +434,23 @@ def main():
     peak, peak_src = _peaks()
     achieved = nbytes / (kern_ms * 1e-3) / 1e9
 
+    # eager per-call latency (no CUDA graph; host launch cost included):
+    # back-to-back pre-marshalled astitch_run calls (Plan.bind), rank-local
+    eager_us = None
+    if world == 1:
+        fns = [plan.bind(dev_in[i], dev_out[i], ws=ws) for i in range(min(nsets, args.steps))]
+        for f in fns[:3]:
+            f()
+        torch.cuda.synchronize()
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        q0.record(stream)
+        for i in range(args.steps):
+            fns[i % len(fns)]()
+        q1.record(stream)
+        torch.cuda.synchronize()
+        eager_us = q0.elapsed_time(q1) * 1e3 / args.steps
+        del fns
+
     # ---- e2e through the C ABI with pinned HOST buffers (H2D + kernel + D2H)
     host_in = [to_torch(x[n], d, None).pin_memory() for n, _, d in spec["inputs"]]
     host_out = [torch.empty(t.shape, dtype=t.dtype).pin_memory() for t in dev_out[0]]
@@ -506,6 +523,7 @@ def main():
                        "template": desc["mapping"]["template"], "grid": desc["kernels"][0]["grid"],
                        "threads": desc["mapping"]["threads"], "regs": desc["kernels"][0]["regs"]},
             "us_per_subgraph": round(ms_step * 1e3, 3),
+            "eager_us_per_call": round(eager_us, 3) if eager_us is not None else None,
             "pct_of_8TBps": round(100.0 * gbs / world / 8000.0, 2),
             "compulsory_bytes_per_step": int(total_bytes),
             "copy_kernel_gbs": round(copy_gbs, 1),

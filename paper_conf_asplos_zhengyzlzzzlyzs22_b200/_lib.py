@@ -123,7 +123,4 @@ def check(status: int, where: str) -> None:
 
 
 def ptr_array(ptrs) -> ct.Array:
-    arr = (_vp * max(1, len(ptrs)))()
-    for i, p in enumerate(ptrs):
-        arr[i] = p
-    return arr
+    return (_vp * max(1, len(ptrs)))(*ptrs)

@@ -241,14 +241,38 @@ class Plan:
 
     def run(self, inputs, outputs, ws=None, stream=None) -> None:
         """astitch_run on device tensors (in declaration order) on `stream`."""
-        if ws is None and self.workspace_bytes() > 0:
-            if self._ws_cache is None:
-                self._ws_cache = self.alloc_workspace(stream)
+        if ws is None and self._ws_cache is None and self.workspace_bytes() > 0:
+            self._ws_cache = self.alloc_workspace(stream)
+        if ws is None:
             ws = self._ws_cache
         ins = ptr_array([t.data_ptr() for t in inputs])
         outs = ptr_array([t.data_ptr() for t in outputs])
         check(lib.astitch_run(self._h, ins, outs, ct.c_void_p(ws.data_ptr() if ws is not None else 0),
                               ct.c_void_p(_stream_ptr(stream))), "astitch_run")
+
+    def bind(self, inputs, outputs, ws=None, stream=None):
+        """Pre-marshalled astitch_run for repeated eager calls on the same
+        buffers and stream: returns a no-argument callable whose only work per
+        call is the C-ABI call (pointer arrays, workspace and stream are
+        resolved once here; the tensors are kept alive by the callable)."""
+        if ws is None and self._ws_cache is None and self.workspace_bytes() > 0:
+            self._ws_cache = self.alloc_workspace(stream)
+        if ws is None:
+            ws = self._ws_cache
+        ins = ptr_array([t.data_ptr() for t in inputs])
+        outs = ptr_array([t.data_ptr() for t in outputs])
+        w = ct.c_void_p(ws.data_ptr() if ws is not None else 0)
+        s = ct.c_void_p(_stream_ptr(stream))
+        fn, h = lib.astitch_run, self._h
+        keep = (self, list(inputs), list(outputs), ws)
+
+        def run() -> None:
+            st = fn(h, ins, outs, w, s)
+            if st:
+                check(st, "astitch_run")
+
+        run.keep = keep
+        return run
 
     def run_host(self, host_inputs, host_outputs, dev_inputs, dev_outputs, ws=None, stream=None,
                  chunks: int = 1) -> None:

@@ -204,3 +204,27 @@ def test_peer_exchange_misuse_errors():
     other = ShardedPlan(A.Graph.from_spec(specs.get("C5", rows=1000, cols=128)), 1000, 128, 2, 1, 0)
     with pytest.raises(A.AstitchError):   # different plan (cols): buffer sizes differ
         x0.link(1, PeerExchange(other.plan))
+
+
+@pytest.mark.parametrize("cfg,rows,cols", [("C1", None, None), ("C5", 4099, 256), ("C3", 1024, None)])
+def test_bind_matches_run(cfg, rows, cols):
+    """Plan.bind(): the pre-marshalled eager call computes what run() does
+    (bitwise: same kernel, same buffers layout), repeatedly."""
+    import torch
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 256
+    x = gen.generate(cfg, spec)
+    p = A.Plan(A.Graph.from_spec(spec), spec["rows"], spec["cols"], device=0)
+    ins = device_inputs(spec, x)
+    o1, o2 = p.alloc_outputs(), p.alloc_outputs()
+    p.run(ins, o1)
+    f = p.bind(ins, o2)
+    for _ in range(3):
+        f()
+    torch.cuda.synchronize()
+    for a, b in zip(o1, o2):
+        assert torch.equal(a, b)
+    ref = evaluate(spec, x)
+    for (name, dt), t in zip(spec["outputs"], o2):
+        check_close(from_torch(t), ref[name], dt, spec_tol(spec), name=f"{cfg}:{name}")
