@@ -481,6 +481,23 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
     e2e_gbs = total_bytes / (e2e_ms * 1e-3) / 1e9 if args.e2e_steps else None
+    # the PCIe floor of that step: the same H2D bytes alone, the same D2H bytes alone
+    link = None
+    if args.e2e_steps:
+        def _copy_ms(pairs):
+            c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            c0.record(stream)
+            for dst_, src_ in pairs:
+                dst_.copy_(src_, non_blocking=True)
+            c1.record(stream)
+            torch.cuda.synchronize()
+            return c0.elapsed_time(c1)
+        _copy_ms(list(zip(dev_in[0], host_in)))
+        h2d_ms = _copy_ms(list(zip(dev_in[0], host_in)))
+        d2h_ms = _copy_ms(list(zip(host_out, dev_out[0])))
+        link = {"h2d_gbs": round(h2d / (h2d_ms * 1e-3) / 1e9, 2), "d2h_gbs": round(d2h / (d2h_ms * 1e-3) / 1e9, 2),
+                "floor_ms": round(max(h2d_ms, d2h_ms), 3),
+                "frac_of_floor": round(max(h2d_ms, d2h_ms) / e2e_ms, 4)}
 
     # ---- oracle on the host cores: bounded sample of the same workload (rank 0, N=1)
     cpu = None
@@ -537,7 +554,7 @@ def main():
                     "d2h_bytes_per_step": int(d2h), "ms_per_step": round(e2e_ms, 3),
                     "api": "astitch_run_host_pipelined" if (world == 1 and args.e2e_chunks > 1) else
                            ("astitch_run_host" if world == 1 else "torch H2D/D2H + astitch_run_sharded"),
-                    "chunks": args.e2e_chunks if world == 1 else 1},
+                    "chunks": args.e2e_chunks if world == 1 else 1, "pcie": link},
             "gpu_launches": int(args.steps * sp.kernels_per_run()),
             "clocks": clocks,
             "cpu_baseline": cpu,
