@@ -416,6 +416,13 @@ struct Gen {
     }
   }
 
+  // shifted fp32 form of a precise row sum: rows wholly inside one warp (or
+  // one thread), every column valid up to C (no masks: an invalid element
+  // would have to be excluded from both the terms and the count)
+  bool shifted_sum_ok() const {
+    return !masked && !split && T <= 32 && (m.tmpl == Template::RowTeam || m.tmpl == Template::PackedTile) &&
+           !env_on("ASTITCH_PRECISE_F64");
+  }
   // a FULL value whose (transitive) consumers include a reduction
   bool feeds_reduction(int i) const {
     for (int u : I(i).consumers) {
@@ -545,6 +552,32 @@ struct Gen {
         if (mx) o << "      if (" << okc << ") acc" << id << "[k] = fmaxf(acc" << id << "[k], " << val << ");\n";
         else o << "      if (" << okc << ") acc" << id << "[k] += " << val << ";\n";
         o << "    }\n";
+        continue;
+      }
+      if (nd.type == NodeType::Reduce && precise[i] && shifted_sum_ok()) {
+        // cancellation-prone row sum, shifted form: sum the row's values
+        // minus its first value x0 (team-uniform) in fp32, then
+        // d = C*x0 + sum(v - x0) in fp64 once per row.  The fp32 terms are of
+        // the size of the row's spread, not of its mean, so the mean is
+        // accurate to ~log2(C) ulps of the spread (as the fp64 tree, reading
+        // R7b) without an F2F + DADD per element.
+        const std::string v0 = ref(nd.a, "0", sfx);
+        o << "    double d" << id << sfx << ";\n    {\n";
+        o << "      const float x0_ = " << (T == 1 ? v0 : "__shfl_sync(0xffffffffu, " + v0 + ", 0, T)") << ";\n";
+        o << "      float t_[NE];\n";
+        if (check) {
+          o << "#pragma unroll\n      for (int k = 0; k < NE; ++k) t_[k] = (" << col_expr("(k / E)", "(k % E)") << " < " << lim
+            << ") ? " << ref(nd.a, "k", sfx) << " - x0_ : 0.f;\n";
+        } else if ((NE % 2) == 0) {
+          o << "#pragma unroll\n      for (int k = 0; k < NE; k += 2) { const as::f2 r_ = as::sub2(" << ref2(nd.a, sfx)
+            << ", as::bc2(x0_)); t_[k] = r_.x; t_[k + 1] = r_.y; }\n";
+        } else {
+          o << "#pragma unroll\n      for (int k = 0; k < NE; ++k) t_[k] = " << ref(nd.a, "k", sfx) << " - x0_;\n";
+        }
+        o << "      float r_ = as::Tree<NE, false>::reduce(t_);\n";
+        if (T > 1) o << "      r_ = as::team_sum<T>(r_);\n";
+        o << "      d" << id << sfx << " = fma((double)x0_, (double)C, (double)r_);\n    }\n";
+        emit_split(id, sfx);
         continue;
       }
       if (nd.type == NodeType::Reduce && precise[i]) {  // cancellation-prone row sum: fp64

@@ -484,3 +484,18 @@ def test_fused_exchange_virtual_ranks(cfg, rows, cols, world):
     if cfg == "C5int":
         np.testing.assert_array_equal(results[0]["db"], ref["db"])
     assert ranks[0][0].kernels_per_run() == 1
+
+
+@pytest.mark.parametrize("rows,cols,template", [(5003, 36, "packed_tile"), (300, 768, "row_team"),
+                                                (1000, 100, "row_team")])
+def test_parity_mean_far_from_spread(rows, cols, template):
+    """Row standardisation of rows whose mean (1000) is 1e5 times their spread
+    (0.01), fp32 I/O at the 1e-5 rule: a plain fp32 row sum loses the spread
+    (reading R7b); the shifted fp32 sum and the fp64 tree both keep it."""
+    spec = specs.get("C4", rows=rows, cols=cols)
+    x = gen.generate("C4", spec)
+    name = spec["inputs"][0][0]
+    x[name] = (1000.0 + 0.01 * x[name].astype(np.float64)).astype(np.float32)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    assert plan.describe()["mapping"]["template"] == template
+    _compare(spec, got, evaluate(spec, x))
