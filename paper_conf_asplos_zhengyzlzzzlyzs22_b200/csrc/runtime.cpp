@@ -128,7 +128,11 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
       retune_grid(p);
       continue;
     }
-    if (k.spill_bytes > 0 && cur > 1) bad = cur;
+    // a one-wave row team (every row its own team) tolerates a small spill
+    // at its target occupancy: measured on B200 (C2), 40 spilled bytes at
+    // 7 blocks/SM 6.8 us vs 7.1 us spill-free at 4 blocks/SM (two row trips)
+    const bool tolerable = p.map.single_wave_bps == cur && k.spill_bytes <= 64;
+    if (k.spill_bytes > 0 && cur > 1 && !tolerable) bad = cur;
     else good = cur;
     if (good == cur && (bad == 0 || bad - good <= 1)) return ASTITCH_OK;  // best found
     int next = good > 0 ? (good + bad) / 2 : std::max(1, bad / 2);

@@ -212,7 +212,10 @@ def test_generated_kernels_compile_for_sm100a(cfg):
     cub = p.cubin(0)
     assert len(cub) > 1000 and cub[:4] == b"\x7fELF"
     k = d["kernels"][0]
-    assert k["spill_bytes"] == 0, k
+    # a one-wave row team may keep a small spill at its target occupancy (C2:
+    # 40 bytes at 7 blocks/SM, measured faster than spill-free at 4)
+    allowed = 64 if d["mapping"].get("single_wave_bps", 0) > 0 else 0
+    assert k["spill_bytes"] <= allowed, k
     assert k["name"].startswith("astitch_")
 
 
