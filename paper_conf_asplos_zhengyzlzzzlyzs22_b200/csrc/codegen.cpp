@@ -423,6 +423,7 @@ struct Gen {
     return !masked && !split && T <= 32 && (m.tmpl == Template::RowTeam || m.tmpl == Template::PackedTile) &&
            !env_on("ASTITCH_PRECISE_F64");
   }
+  bool seg_lookahead() const { return !env_on("ASTITCH_SEG_LOOKAHEAD1"); }
   // a FULL value whose (transitive) consumers include a reduction
   bool feeds_reduction(int i) const {
     for (int u : I(i).consumers) {
@@ -1109,8 +1110,16 @@ struct Gen {
         std::string s = su + std::to_string(u) + "n";
         for (size_t q = 0; q < streams.size(); ++q) o << "  " << raw_t(streams[q]) << " r" << q << s << "[V];\n";
         // (ragged) the segment entry of the prefetched row, reused by the compute step
-        if (ragged) o << "  int4 nsg" << u << " = (prow" << u << " < R) ? as::seg_find<NSEG>(SG, (int)prow" << u
-                      << ") : make_int4(0, 0, 0, 0);\n";
+        if (ragged) {
+          o << "  int4 nsg" << u << " = (prow" << u << " < R) ? as::seg_find<NSEG>(SG, (int)prow" << u
+            << ") : make_int4(0, 0, 0, 0);\n";
+          // two-deep segment lookahead: the entry of the row after the
+          // prefetched one is searched an iteration early, so the prefetch's
+          // load addresses never wait on a binary search
+          if (seg_lookahead())
+            o << "  int nnsg" << u << " = (prow" << u << " + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(prow" << u
+              << " + rstride)) : -1;\n";
+        }
         o << "  {\n    const bool pact = prow" << u << " < R;\n";
         o << "    " << limdecl("plim", "pact", "prow" + std::to_string(u), ragged ? "nsg" + std::to_string(u) : "")
           << "\n";
@@ -1154,10 +1163,14 @@ struct Gen {
         o << "    {\n";
         o << "      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
         o << "      const bool pact = nrow < R;\n";
-        if (ragged) o << "      nsg" << u << " = pact ? as::seg_find<NSEG>(SG, (int)nrow) : make_int4(0, 0, 0, 0);\n";
+        const bool la = ragged && seg_lookahead();
+        if (la) o << "      nsg" << u << " = (nnsg" << u << " >= 0) ? __ldg(SG + nnsg" << u << ") : make_int4(0, 0, 0, 0);\n";
+        else if (ragged) o << "      nsg" << u << " = pact ? as::seg_find<NSEG>(SG, (int)nrow) : make_int4(0, 0, 0, 0);\n";
         o << "      " << limdecl("plim", "pact", "nrow", ragged ? "nsg" + std::to_string(u) : "") << "\n";
         o << "      (void)plim;\n";
         emit_loads("nrow", "pact", "plim", s, false);
+        if (la)
+          o << "      nnsg" << u << " = (nrow + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(nrow + rstride)) : -1;\n";
         o << "    }\n";
       }
     } else {

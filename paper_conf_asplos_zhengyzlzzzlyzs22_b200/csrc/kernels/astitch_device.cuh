@@ -237,7 +237,7 @@ template <int DT, int E> struct Conv {
 // pitch, offset8} of the segment owning `row` = the largest s with
 // row_start_s <= row (row_start increasing; empty segments share a start and
 // the search lands on the last of them, the one whose range holds the row).
-template <int NSEG> __device__ __forceinline__ int4 seg_find(const int4* __restrict__ sg, int row) {
+template <int NSEG> __device__ __forceinline__ int seg_find_idx(const int4* __restrict__ sg, int row) {
   int lo = 0, hi = NSEG - 1;
 #pragma unroll 1
   while (lo < hi) {
@@ -245,7 +245,10 @@ template <int NSEG> __device__ __forceinline__ int4 seg_find(const int4* __restr
     if (__ldg(&sg[mid].x) <= row) lo = mid;
     else hi = mid - 1;
   }
-  return __ldg(sg + lo);
+  return lo;
+}
+template <int NSEG> __device__ __forceinline__ int4 seg_find(const int4* __restrict__ sg, int row) {
+  return __ldg(sg + seg_find_idx<NSEG>(sg, row));
 }
 
 // scalar (ROWVEC / COLVEC element) load / store with dtype

@@ -125,4 +125,7 @@ def test_ragged_kernel_compiles_for_sm100a():
     sv = gen.ragged_spec(specs.get("C3v"), 3)
     p = _plan(sv, flags=0)
     d = p.describe()
-    assert p.cubin(0)[:4] == b"\x7fELF" and d["kernels"][0]["spill_bytes"] == 0
+    # a spill of a few registers (<= 32 bytes) is accepted rather than halving
+    # the occupancy (runtime.cpp, assume-relax-apply)
+    assert p.cubin(0)[:4] == b"\x7fELF" and d["kernels"][0]["spill_bytes"] <= 32
+    assert d["mapping"]["grid"] >= 2 * 148
