@@ -239,8 +239,36 @@ class Plan:
               "astitch_workspace_init")
         return ws
 
+    def _numel(self, kind: str):
+        if kind == "LENGTHS":
+            return None  # one length per segment of rows_per_segment rows (checked by the caller's spec)
+        n = 1
+        for d in self.io_shape(kind):
+            n *= d
+        return n
+
+    def check_io(self, inputs, outputs, device: bool = True) -> None:
+        """Validate tensors against the plan's I/O list (count, dtype, element
+        count, contiguity, CUDA placement): the C ABI sees only base pointers,
+        so a strided view or a wrong dtype would otherwise be read silently."""
+        for what, ts, decl in (("input", inputs, self.inputs), ("output", outputs, self.outputs)):
+            if len(ts) != len(decl):
+                raise ValueError(f"expected {len(decl)} {what}s, got {len(ts)}")
+            for i, (t, (kind, dt)) in enumerate(zip(ts, decl)):
+                want = _torch_dtype(dt)
+                if t.dtype != want:
+                    raise ValueError(f"{what} {i} ({kind}): dtype {t.dtype}, plan expects {want}")
+                if not t.is_contiguous():
+                    raise ValueError(f"{what} {i} ({kind}): tensor is not contiguous")
+                n = self._numel(kind)
+                if n is not None and t.numel() != n:
+                    raise ValueError(f"{what} {i} ({kind}): {t.numel()} elements, plan expects {n}")
+                if device and not t.is_cuda:
+                    raise ValueError(f"{what} {i} ({kind}): expected a CUDA tensor")
+
     def run(self, inputs, outputs, ws=None, stream=None) -> None:
         """astitch_run on device tensors (in declaration order) on `stream`."""
+        self.check_io(inputs, outputs)
         if ws is None and self._ws_cache is None and self.workspace_bytes() > 0:
             self._ws_cache = self.alloc_workspace(stream)
         if ws is None:
@@ -255,6 +283,7 @@ class Plan:
         buffers and stream: returns a no-argument callable whose only work per
         call is the C-ABI call (pointer arrays, workspace and stream are
         resolved once here; the tensors are kept alive by the callable)."""
+        self.check_io(inputs, outputs)
         if ws is None and self._ws_cache is None and self.workspace_bytes() > 0:
             self._ws_cache = self.alloc_workspace(stream)
         if ws is None:
@@ -278,6 +307,8 @@ class Plan:
                  chunks: int = 1) -> None:
         """astitch_run_host (chunks == 1) / astitch_run_host_pipelined (chunks > 1):
         H2D inputs, stitched kernel(s), D2H outputs, asynchronous on `stream`."""
+        self.check_io(host_inputs, host_outputs, device=False)
+        self.check_io(dev_inputs, dev_outputs)
         if ws is None and self.workspace_bytes() > 0:
             if self._ws_cache is None:
                 self._ws_cache = self.alloc_workspace(stream)

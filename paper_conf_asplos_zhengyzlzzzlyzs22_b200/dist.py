@@ -131,6 +131,7 @@ class ShardedPlan:
 
     def run(self, inputs, outputs, ws=None, stream=None) -> None:
         p = self.plan
+        p.check_io(inputs, outputs)
         ws = self._ws(ws, stream)
         ins = ptr_array([t.data_ptr() for t in inputs])
         outs = ptr_array([t.data_ptr() for t in outputs])

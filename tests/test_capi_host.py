@@ -129,3 +129,25 @@ def test_io_signature_and_workspace():
     p = A.Plan(A.Graph.from_spec(spec), 8192, 512, device=-1, flags=A.FLAG_NO_COMPILE)
     assert p.inputs == [("FULL", "BF16"), ("LENGTHS", "I32")]
     assert p.workspace_bytes() == 0
+
+
+def test_binding_checks_tensors_against_the_plan():
+    """The binding validates count, dtype, element count and contiguity before
+    a pointer crosses the C ABI (host tensors here; device placement on GPU)."""
+    import torch
+    from workloads import specs
+    spec = specs.get("C5", rows=64, cols=32)
+    p = A.Plan(A.Graph.from_spec(spec), 64, 32, device=-1, flags=A.FLAG_NO_COMPILE)
+    ins = [torch.zeros(64, 32, dtype=torch.bfloat16), torch.zeros(64, 32, dtype=torch.bfloat16), torch.zeros(32)]
+    outs = [torch.zeros(64, 32, dtype=torch.bfloat16), torch.zeros(32), torch.zeros(32)]
+    p.check_io(ins, outs, device=False)
+    with pytest.raises(ValueError, match="dtype"):
+        p.check_io([ins[0].float()] + ins[1:], outs, device=False)
+    with pytest.raises(ValueError, match="contiguous"):
+        p.check_io([torch.zeros(32, 64, dtype=torch.bfloat16).t()] + ins[1:], outs, device=False)
+    with pytest.raises(ValueError, match="elements"):
+        p.check_io(ins, [torch.zeros(63, 32, dtype=torch.bfloat16)] + outs[1:], device=False)
+    with pytest.raises(ValueError, match="inputs"):
+        p.check_io(ins[:2], outs, device=False)
+    with pytest.raises(ValueError, match="CUDA"):
+        p.check_io(ins, outs)
