@@ -322,6 +322,12 @@ def main():
             except Exception as e:  # pragma: no cover - needs a multi-GPU box
                 print(f"[bench] fused exchange unavailable ({e}); using NCCL", file=sys.stderr)
                 sp.peer = None
+            # every rank must take the same path (a fused kernel waits for all peers)
+            ok = torch.tensor([1.0 if sp.peer is not None else 0.0], device=f"cuda:{dev}")
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+            if float(ok.item()) < 1.0:
+                sp.peer = None
+                exchange = "ncclAllReduce + epilogue (peer mapping failed on a rank)"
     plan = sp.plan
     desc = plan.describe()
     r0, nr = sp.row_begin, sp.row_count
