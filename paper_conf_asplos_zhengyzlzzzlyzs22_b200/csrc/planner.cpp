@@ -386,6 +386,13 @@ void select_mapping(Plan& p) {
   // Blocks-per-wave reference for the paper's shape rule: the number
   // of 1024-thread-equivalent blocks the chip runs at once = 2 per SM.
   const int64_t blocks_per_wave_1024 = 2LL * sms;
+  // Cluster size for few long rows: the largest power of two K <= 8 with
+  // R * K <= SMs, i.e. every row's cluster resident in ONE wave of the
+  // 512-thread CTAs these templates use (one per SM at their register
+  // counts).  Measured on B200, <64, 300000> fp32 row sum: K = 8 (18
+  // clusters, 4 row trips) 29.1 us; one CTA per row, streamed, 20.8 us.
+  int k_wave = 1;
+  while (k_wave < 8 && R * (k_wave * 2) <= sms) k_wave *= 2;
 
   if (has_colred || p.max_level > 0) {
     // ---------------------------------------------------------- global sweep
@@ -541,10 +548,7 @@ void select_mapping(Plan& p) {
       // of K CTAs (K ~ blocks-per-wave / rows, power of two, <= 8 portable);
       // block partials combine through DSMEM in a fixed order.
       m.tmpl = Template::SplitRow;
-      int64_t want = (blocks_per_wave_1024 + R - 1) / std::max<int64_t>(R, 1);
-      int k = 2;
-      while (k < want && k < 8) k *= 2;
-      m.split = k;
+      m.split = std::max(2, k_wave);
       m.threads = 512;
       if (const char* fs = getenv("ASTITCH_FORCE_SPLIT")) {  // tuning knob: "K" or "K,threads"
         int kk = atoi(fs);
@@ -615,10 +619,7 @@ void select_mapping(Plan& p) {
       m.threads = 512;
       m.split = 1;
       if (!no_split && R < blocks_per_wave_1024) {
-        int64_t want = (blocks_per_wave_1024 + R - 1) / std::max<int64_t>(R, 1);
-        int k = 1;
-        while (k < want && k < 8) k *= 2;
-        m.split = k;
+        m.split = k_wave;
       }
       m.chunks_per_lane = std::max(1, 32 / E);  // V: 32 values per lane per tile
       // Regional stitching proper: when the row's inputs fit the
@@ -679,13 +680,27 @@ void select_mapping(Plan& p) {
   // compute blocks per SM from threads and smem, relax the register cap to the
   // largest value that keeps those blocks resident; the caller
   // recompiles with a lower target if ptxas reports spills.
-  // Register row teams keep the next row's loads in flight per warp, so 24
-  // resident warps per SM already cover HBM latency; more resident row
-  // streams only add DRAM page contention (measured on B200, C3 masked
-  // softmax: 24 warps/SM 146 us, 32 warps/SM 153.5 us, 16 warps/SM 163 us).
-  const int max_threads_sm = (m.tmpl == Template::RowTeam)
-                                 ? (m.single_wave_bps > 0 ? m.single_wave_bps * m.threads : 768)
-                                 : 2048;
+  // Register row teams that write whole rows: cap the resident warps at those
+  // needed for ~48 KB of row stores per SM per row step; more concurrent
+  // row-write streams only add DRAM page contention (measured on B200: C3
+  // masked softmax, 2 KB of stores per warp step: 24 warps/SM 146 us, 32
+  // warps 153.5 us, 16 warps 163 us).  Read-mostly rows (a row sum, fig6a:
+  // 64 B of stores per warp step) keep the full occupancy.
+  int max_threads_sm = 2048;
+  if (m.tmpl == Template::RowTeam) {
+    if (m.single_wave_bps > 0) {
+      max_threads_sm = m.single_wave_bps * m.threads;
+    } else {
+      int64_t out_row_bytes = 0;
+      for (size_t k = 0; k < g.outputs.size(); ++k)
+        if (g.nodes[g.outputs[k]].kind == ASTITCH_FULL)
+          out_row_bytes += std::min<int64_t>(C * dtype_size(g.output_dtypes[k]), 1 << 30);
+      const double bytes_per_warp = std::max<double>(1.0, static_cast<double>(out_row_bytes) * m.row_unroll * 32.0 / m.team);
+      const int cap_warps = static_cast<int>(std::min(64.0, std::max(4.0, std::ceil(48.0 * 1024 / bytes_per_warp))));
+      const int wpb = std::max(1, m.threads / 32);
+      max_threads_sm = std::min(2048, ((cap_warps + wpb - 1) / wpb) * m.threads);
+    }
+  }
   int by_threads = std::max(1, max_threads_sm / m.threads);
   int by_smem = m.smem_bytes > 0 ? (228 * 1024) / (m.smem_bytes + 1024) : 32;
   m.blocks_per_sm = std::max(1, std::min({32, by_threads, by_smem}));

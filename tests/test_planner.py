@@ -114,9 +114,11 @@ def test_fig6_selector_branches():
     assert d["mapping"]["template"] == "row_team" and d["mapping"]["team"] == 1024
     d, _, _ = describe("fig6b", flags=A.FLAG_NO_COMPILE | A.FLAG_FORCE_SPLIT)
     assert d["mapping"]["template"] == "split_row" and "split rule holds" in d["mapping"]["reason"]
-    assert d["mapping"]["split"] == 8 and d["mapping"]["grid"] % 8 == 0
-    d, _, _ = describe("fig6b", cols=300_000)  # 1.2 MB rows: split by default
-    assert d["mapping"]["template"] == "split_row"
+    # cluster of K CTAs: the largest power of two with rows * K <= SMs (one wave)
+    assert d["mapping"]["split"] == 2 and d["mapping"]["grid"] % 2 == 0
+    d, _, _ = describe("fig6b", cols=300_000)  # 1.2 MB rows: split by default (streamed over a cluster)
+    assert d["mapping"]["template"] == "row_stream" and d["mapping"]["split"] == 2
+    assert d["mapping"]["grid"] == 128
     d, _, _ = describe("fig6b", cols=300_000, flags=A.FLAG_NO_COMPILE | A.FLAG_NO_SPLIT)
     # no splitting: a 1024-lane block would need 293 values per lane -> streamed by one block
     assert d["mapping"]["template"] == "row_stream" and d["mapping"]["split"] == 1
