@@ -1074,11 +1074,15 @@ struct Gen {
     const std::string rt = rowt();
     o << "  const " << rt << " rstride = (" << rt << ")(NUNITS * RPB * " << U << ");\n";
     o << "  " << rt << " base = (" << rt << ")(UNIT * RPB * " << U << ");\n";
-    // The ping-pong form removes the per-row register copies but raised the
-    // register count on B200 (C3: 120 vs 80 regs, 153 vs 146 us), so the copy
-    // form is the default; ASTITCH_PINGPONG=1 selects the other for experiments.
+    // Ping-pong buffers (the loop body emitted twice, rows alternating between
+    // two raw register sets: no copies, and each prefetch has a whole row step
+    // to land) are the default for padded rows.  Measured on B200 against the
+    // early-unpack copy form: C3 143.8 vs 146.1 us (80 vs 72 registers), C2 at
+    // 32768 rows 29.1 vs 29.9 us, C5 and fig6a equal.  Packed varlen rows keep
+    // the copy form (their KF-specialised body would be emitted 2 x (V+1)
+    // times).  ASTITCH_PINGPONG=0 selects the copy form for experiments.
     const char* pp_env = getenv("ASTITCH_PINGPONG");
-    if (pf && pp_env && atoi(pp_env) == 1 && !ragged) {
+    if (pf && !(pp_env && atoi(pp_env) == 0) && !ragged) {
       // ping-pong buffers a / b
       for (int u = 0; u < U; ++u)
         for (const char* bf : {"a", "b"})
