@@ -1038,23 +1038,40 @@ struct Gen {
     const std::string su = "_u";
     const std::string rt = rowt();
     for (int u = 0; u < U; ++u) {
+      const std::string us = std::to_string(u);
       o << "    const " << rt << " row" << u << " = base + " << u << " * RPB + team;\n";
       o << "    const bool act" << u << " = row" << u << " < R;\n";
-      o << "    const int lim" << u << " = "
-        << (masked ? "act" + std::to_string(u) + " ? " + lim_expr("row" + std::to_string(u)) + " : 0" : "(int)C")
-        << ";\n    (void)lim" << u << ";\n";
+      if (ragged) {
+        o << "    " << limdecl("lim" + us, "act" + us, "row" + us, "nsg" + us + cu) << "\n";
+      } else {
+        o << "    const int lim" << u << " = "
+          << (masked ? "act" + us + " ? " + lim_expr("row" + us) + " : 0" : "(int)C") << ";\n";
+      }
+      o << "    (void)lim" << u << ";\n";
     }
     for (int u = 0; u < U; ++u) {
+      const std::string us = std::to_string(u);
       o << "    {\n      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
       o << "      const bool pact = nrow < R;\n";
-      o << "      const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
+      if (ragged) {
+        o << "      nsg" << us << nx << " = (nnsg" << us << " >= 0) ? __ldg(SG + nnsg" << us << ") : make_int4(0, 0, 0, 0);\n";
+        o << "      " << limdecl("plim", "pact", "nrow", "nsg" + us + nx) << "\n";
+      } else {
+        o << "      const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
+      }
       o << "      (void)plim;\n";
-      emit_loads("nrow", "pact", "plim", su + std::to_string(u) + nx, false);
+      emit_loads("nrow", "pact", "plim", su + us + nx, false);
+      if (ragged)
+        o << "      nnsg" << us << " = (nrow + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(nrow + rstride)) : -1;\n";
       o << "    }\n";
     }
     for (int u = 0; u < U; ++u) {
       std::string s = su + std::to_string(u) + cu;
       std::string row = "row" + std::to_string(u), act = "act" + std::to_string(u), lim = "lim" + std::to_string(u);
+      if (ragged) {
+        emit_row_block(post, s, row, act, lim);
+        continue;
+      }
       o << "    {\n";
       emit_unpack(s, lim);
       emit_colvecs(true);
@@ -1064,6 +1081,7 @@ struct Gen {
       o << "    }\n";
     }
   }
+
 
   void emit_sweep(bool post) {
     collect_streams(post);
@@ -1082,16 +1100,29 @@ struct Gen {
     // the copy form (their KF-specialised body would be emitted 2 x (V+1)
     // times).  ASTITCH_PINGPONG=0 selects the copy form for experiments.
     const char* pp_env = getenv("ASTITCH_PINGPONG");
-    if (pf && !(pp_env && atoi(pp_env) == 0) && !ragged) {
+    const bool pp_ragged = env_on("ASTITCH_PINGPONG_RAGGED");
+    if (pf && !(pp_env && atoi(pp_env) == 0) && (!ragged || pp_ragged)) {
       // ping-pong buffers a / b
       for (int u = 0; u < U; ++u)
         for (const char* bf : {"a", "b"})
           for (size_t q = 0; q < streams.size(); ++q)
             o << "  " << raw_t(streams[q]) << " r" << q << su << u << bf << "[V];\n";
+      if (ragged)
+        for (int u = 0; u < U; ++u)
+          o << "  int4 nsg" << u << "a, nsg" << u << "b; int nnsg" << u << ";\n";
       for (int u = 0; u < U; ++u) {
+        const std::string us = std::to_string(u);
         o << "  {\n    const " << rt << " nrow = base + " << u << " * RPB + team;\n";
         o << "    const bool pact = nrow < R;\n";
-        o << "    const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
+        if (ragged) {
+          // packed varlen rows: segment entries per buffer, the next row's
+          // segment index searched one step ahead (nnsg)
+          o << "    nsg" << us << "a = pact ? as::seg_find<NSEG>(SG, (int)nrow) : make_int4(0, 0, 0, 0);\n";
+          o << "    nnsg" << us << " = (nrow + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(nrow + rstride)) : -1;\n";
+          o << "    " << limdecl("plim", "pact", "nrow", "nsg" + us + "a") << "\n";
+        } else {
+          o << "    const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
+        }
         o << "    (void)plim;\n";
         emit_loads("nrow", "pact", "plim", su + std::to_string(u) + "a", false);
         o << "  }\n";
