@@ -240,3 +240,30 @@ def test_row_stream_for_rows_beyond_registers():
     assert d["mapping"]["template"] == "row_team"
     d, _, _ = describe("C4", rows=100_000, cols=200_000)  # many long rows: block per row, no cluster
     assert d["mapping"]["template"] == "row_stream" and d["mapping"]["split"] == 1
+
+
+def test_one_wave_row_teams_and_store_cap():
+    """Launch heuristics measured on B200: rows that need <= 28
+    warps per SM get one wave of 4-warp blocks (C2: 4096 rows -> 1024 blocks
+    of 128 threads, 7 per SM, every row its own team); row teams that write
+    whole rows keep ~48 KB of row stores per SM (C3: 3 blocks of 256);
+    read-mostly rows keep the full occupancy (fig6a)."""
+    d, _, _ = describe("C2")
+    m = d["mapping"]
+    assert m["single_wave_bps"] == 7 and m["threads"] == 128 and m["grid"] == 1024
+    assert m["vertical_trips"] == 1
+    d, _, _ = describe("C2", rows=300)                     # 2 warps per SM: default blocks
+    assert d["mapping"]["single_wave_bps"] == 0
+    d, _, _ = describe("C3")
+    assert d["mapping"]["blocks_per_sm"] == 3 and d["mapping"]["grid"] == 3 * 148
+    d, _, _ = describe("fig6a")
+    assert d["mapping"]["blocks_per_sm"] == 8
+
+
+def test_cluster_size_fills_one_wave():
+    """Few long rows: K = largest power of two <= 8 with R * K <= SMs."""
+    for rows, k in ((64, 2), (16, 8), (37, 4), (38, 2), (100, 1), (3, 8)):
+        d, _, _ = describe("C1", rows=rows, cols=2_000_000)
+        m = d["mapping"]
+        assert m["template"] == "row_stream" and m["split"] == k, (rows, m["split"])
+        assert rows * m["split"] <= 148 or m["split"] == 1
