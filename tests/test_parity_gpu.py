@@ -500,3 +500,22 @@ def test_parity_mean_far_from_spread(rows, cols, template):
     got, plan = run_gpu(spec, x, return_plan=True)
     assert plan.describe()["mapping"]["template"] == template
     _compare(spec, got, evaluate(spec, x))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_parity_random_shapes(seed):
+    """Seeded random (rows, cols) across the mapping space (one-wave row teams,
+    prefetching ping-pong sweeps, packed tiles, clusters, streamed rows), each
+    checked against the oracle."""
+    rng = np.random.default_rng(1000 + seed)
+    cfgs = ["C1", "C2", "C3", "C4", "C5", "fig7a"]
+    for cfg in cfgs:
+        rows = int(rng.choice([int(rng.integers(1, 64)), int(rng.integers(64, 6000)), int(rng.integers(6000, 20000))]))
+        cols = int(rng.choice([int(rng.integers(1, 128)), int(rng.integers(128, 1100)), int(rng.integers(1100, 5000))]))
+        cols = max(1, min(cols, 8_000_000 // rows))        # oracle time bound
+        spec = specs.get(cfg, rows=rows, cols=cols)
+        if spec.get("mask"):
+            spec["mask"]["rows_per_segment"] = int(rng.integers(1, 300))
+        x = gen.generate(cfg, spec)
+        got, plan = run_gpu(spec, x, return_plan=True)
+        _compare(spec, got, evaluate(spec, x))
