@@ -28,6 +28,7 @@ struct Driver {
   CUresult (*FuncSetAttribute)(CUfunction, CUfunction_attribute, int);
   CUresult (*FuncGetAttribute)(int*, CUfunction_attribute, CUfunction);
   CUresult (*Occupancy)(int*, CUfunction, int, size_t);
+  CUresult (*OccupancyClusters)(int*, CUfunction, const CUlaunchConfig*);
   CUresult (*LaunchKernelEx)(const CUlaunchConfig*, CUfunction, void**, void**);
   CUresult (*MemsetD8Async)(CUdeviceptr, unsigned char, size_t, CUstream);
   CUresult (*MemcpyAsync)(CUdeviceptr, CUdeviceptr, size_t, CUstream);
@@ -97,6 +98,7 @@ Driver* driver(std::string& err) {
   SYM(FuncSetAttribute, "cuFuncSetAttribute");
   SYM(FuncGetAttribute, "cuFuncGetAttribute");
   SYM(Occupancy, "cuOccupancyMaxActiveBlocksPerMultiprocessor");
+  SYM(OccupancyClusters, "cuOccupancyMaxActiveClusters");
   SYM(LaunchKernelEx, "cuLaunchKernelEx");
   SYM(MemsetD8Async, "cuMemsetD8Async");
   SYM(MemcpyAsync, "cuMemcpyAsync");
@@ -175,6 +177,22 @@ bool drv_load(Plan& p, Kernel& k, std::string& err) {
   if (k.smem > 48 * 1024) {
     r = d->FuncSetAttribute(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, k.smem);
     if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuFuncSetAttribute(smem)"); d->ModuleUnload(mod); return false; }
+  }
+  if (k.cluster > 8) {
+    // clusters of 9-16 CTAs are non-portable: opt in per function
+    r = d->FuncSetAttribute(fn, CU_FUNC_ATTRIBUTE_NON_PORTABLE_CLUSTER_SIZE_ALLOWED, 1);
+    if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuFuncSetAttribute(non-portable cluster)"); d->ModuleUnload(mod); return false; }
+  }
+  k.max_clusters = -1;
+  if (k.cluster > 1) {
+    CUlaunchConfig cfg{};
+    cfg.gridDimX = static_cast<unsigned>(k.grid);
+    cfg.gridDimY = cfg.gridDimZ = 1;
+    cfg.blockDimX = static_cast<unsigned>(k.threads);
+    cfg.blockDimY = cfg.blockDimZ = 1;
+    cfg.sharedMemBytes = static_cast<unsigned>(k.smem);
+    int nc = 0;
+    if (d->OccupancyClusters(&nc, fn, &cfg) == CUDA_SUCCESS) k.max_clusters = nc;
   }
   int regs = -1, local = -1;
   d->FuncGetAttribute(&regs, CU_FUNC_ATTRIBUTE_NUM_REGS, fn);

@@ -130,6 +130,8 @@ struct Kernel {
   int regs = -1;
   int spill_bytes = -1;
   int occupancy = -1;        // blocks per SM from the occupancy API
+  int cluster = 1;           // CTAs per cluster (compile-time __cluster_dims__)
+  int max_clusters = -1;     // co-resident clusters (cuOccupancyMaxActiveClusters), cluster kernels
   void* module = nullptr;    // CUmodule
   void* function = nullptr;  // CUfunction
 };
@@ -157,6 +159,7 @@ struct Plan {
   bool needs_sweep2 = false;     // FULL / ROWVEC work after the (first) grid barrier
   int max_level = 0;             // grid barriers needed by dependent column reductions
   bool stream_fallback = false;  // registers overflowed at 1 block/SM: stream the rows
+  bool portable_clusters = false; // 16-CTA clusters not co-resident in one wave: plan with <= 8
   std::vector<Kernel> kernels;   // kernels launched by astitch_run, in order
   std::vector<Kernel> shard_kernels; // kernels of the sharded path (after the allreduce)
   std::vector<Kernel> fused_kernels; // fused sharded path (P2P exchange in-kernel), built lazily

@@ -393,6 +393,11 @@ void select_mapping(Plan& p) {
   // clusters, 4 row trips) 29.1 us; one CTA per row, streamed, 20.8 us.
   int k_wave = 1;
   while (k_wave < 8 && R * (k_wave * 2) <= sms) k_wave *= 2;
+  // rows <= 9: non-portable clusters of 16 (validated at load time against
+  // cuOccupancyMaxActiveClusters, else back to 8)
+  if (k_wave == 8 && R * 16 <= sms && !p.portable_clusters &&
+      !(getenv("ASTITCH_PORTABLE_CLUSTERS") && atoi(getenv("ASTITCH_PORTABLE_CLUSTERS")) == 1))
+    k_wave = 16;
 
   if (has_colred || p.max_level > 0) {
     // ---------------------------------------------------------- global sweep

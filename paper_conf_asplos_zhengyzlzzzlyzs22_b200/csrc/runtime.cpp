@@ -103,9 +103,20 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     k.cooperative = (p.map.tmpl == Template::GlobalSweep) &&
                     (role == ROLE_MAIN || role == ROLE_SHARD_MAIN || role == ROLE_FUSED);
     k.pdl = !k.cooperative && role != ROLE_SHARD_FINAL && (p.desc.flags & ASTITCH_FLAG_NO_PDL) == 0;
+    const bool clustered = role != ROLE_SHARD_FINAL &&
+                           (p.map.tmpl == Template::SplitRow || p.map.tmpl == Template::RowStream) && p.map.split > 1;
+    k.cluster = clustered ? p.map.split : 1;
     if (!compile) return ASTITCH_OK;
     astitch_status st = compile_and_inspect(p, k, load);
     if (st != ASTITCH_OK) return st;
+    // non-portable clusters (9-16 CTAs): keep them only if every row's
+    // cluster is co-resident in one wave; else fall back to portable 8
+    if (k.cluster > 8 && load && k.max_clusters >= 0 && k.max_clusters * k.cluster < k.grid && !p.portable_clusters) {
+      p.portable_clusters = true;
+      select_mapping(p);  // re-plan the row's lanes / chunks for clusters of <= 8
+      good = bad = 0;
+      continue;
+    }
     if (!may_relax || getenv("ASTITCH_FORCE_BPS")) return ASTITCH_OK;
     const int cur = p.map.blocks_per_sm;
     // (measured on B200, fp32 softmax rows of 4096 x C: a 116-byte spill

@@ -261,8 +261,10 @@ def test_one_wave_row_teams_and_store_cap():
 
 
 def test_cluster_size_fills_one_wave():
-    """Few long rows: K = largest power of two <= 8 with R * K <= SMs."""
-    for rows, k in ((64, 2), (16, 8), (37, 4), (38, 2), (100, 1), (3, 8)):
+    """Few long rows: K = largest power of two <= 8 with R * K <= SMs; rows
+    <= 9 ask for non-portable clusters of 16 (validated when the kernel loads
+    on a GPU, else back to 8)."""
+    for rows, k in ((64, 2), (16, 8), (37, 4), (38, 2), (100, 1), (3, 16), (9, 16), (10, 8)):
         d, _, _ = describe("C1", rows=rows, cols=2_000_000)
         m = d["mapping"]
         assert m["template"] == "row_stream" and m["split"] == k, (rows, m["split"])
