@@ -155,6 +155,8 @@ struct Gen {
     if (const char* q = getenv("ASTITCH_ST_HINT"))  // experiments: output store cache qualifier
       if (std::string(q) == ".cs" || std::string(q) == ".wt" || std::string(q) == ".cg")
         o << "#define AS_STQ \"" << q << "\"\n";
+    if (const char* q = getenv("ASTITCH_LD_HINT"))  // experiments: streaming load qualifiers
+      o << "#define AS_LDQ \"" << (std::string(q) == "none" ? "" : q) << "\"\n";
     o << "#include \"astitch_device.cuh\"\n";
     o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; void* xbuf; unsigned int gen; };\n";
     o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") ";
@@ -1034,6 +1036,7 @@ struct Gen {
   // one ping-pong half of the software-pipelined row loop: loads of the rows
   // one stride ahead go to buffer `nx` while the rows of `base` are computed
   // from buffer `cu` (no register copies between the halves)
+  bool dyn = false;  // dynamic row tiles (m.dyn_tiles) in the ping-pong loop being emitted
   void emit_pingpong_half(bool post, const std::string& cu, const std::string& nx) {
     const std::string su = "_u";
     const std::string rt = rowt();
@@ -1051,7 +1054,8 @@ struct Gen {
     }
     for (int u = 0; u < U; ++u) {
       const std::string us = std::to_string(u);
-      o << "    {\n      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
+      o << "    {\n      const " << rt << " nrow = " << (dyn ? "nbase" : "base + rstride") << " + " << u
+        << " * RPB + team;\n";
       o << "      const bool pact = nrow < R;\n";
       if (ragged) {
         o << "      nsg" << us << nx << " = (nnsg" << us << " >= 0) ? __ldg(SG + nnsg" << us << ") : make_int4(0, 0, 0, 0);\n";
@@ -1065,6 +1069,9 @@ struct Gen {
         o << "      nnsg" << us << " = (nrow + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(nrow + rstride)) : -1;\n";
       o << "    }\n";
     }
+    // dynamic tiles: the index of the tile after next, grabbed while this
+    // tile computes (read after the step's barrier)
+    if (dyn) o << "    if (threadIdx.x == 0) dq_[" << (cu == "a" ? 0 : 1) << "] = (int)atomicAdd(dctr_, 1u);\n";
     for (int u = 0; u < U; ++u) {
       std::string s = su + std::to_string(u) + cu;
       std::string row = "row" + std::to_string(u), act = "act" + std::to_string(u), lim = "lim" + std::to_string(u);
@@ -1101,7 +1108,15 @@ struct Gen {
     // times).  ASTITCH_PINGPONG=0 selects the copy form for experiments.
     const char* pp_env = getenv("ASTITCH_PINGPONG");
     const bool pp_ragged = env_on("ASTITCH_PINGPONG_RAGGED");
+    dyn = false;
     if (pf && !(pp_env && atoi(pp_env) == 0) && (!ragged || pp_ragged)) {
+      dyn = m.dyn_tiles && !ragged && m.tmpl == Template::RowTeam;
+      if (dyn) {
+        o << "  unsigned int* dctr_ = (unsigned int*)((char*)p.ws + " << p.ws.barrier << "LL);\n";
+        o << "  __shared__ int dq_[2];\n  constexpr int TILE_ = RPB * " << U << ";\n";
+        o << "  if (threadIdx.x == 0) { dq_[0] = (int)atomicAdd(dctr_, 1u); dq_[1] = (int)atomicAdd(dctr_, 1u); }\n";
+        o << "  __syncthreads();\n  base = dq_[0] * TILE_;\n  " << rt << " nbase = dq_[1] * TILE_;\n  __syncthreads();\n";
+      }
       // ping-pong buffers a / b
       for (int u = 0; u < U; ++u)
         for (const char* bf : {"a", "b"})
@@ -1126,6 +1141,20 @@ struct Gen {
         o << "    (void)plim;\n";
         emit_loads("nrow", "pact", "plim", su + std::to_string(u) + "a", false);
         o << "  }\n";
+      }
+      if (dyn) {
+        o << "  while (base < R) {\n";
+        o << "   {\n";
+        emit_pingpong_half(post, "a", "b");
+        o << "   }\n    __syncthreads();\n    base = nbase;\n    nbase = dq_[0] * TILE_;\n    __syncthreads();\n"
+          << "    if (base >= R) break;\n";
+        o << "   {\n";
+        emit_pingpong_half(post, "b", "a");
+        o << "   }\n    __syncthreads();\n    base = nbase;\n    nbase = dq_[1] * TILE_;\n    __syncthreads();\n  }\n";
+        // the last CTA to finish resets the counters for the next run
+        o << "  if (threadIdx.x == 0) {\n    __threadfence();\n"
+          << "    if (atomicAdd(dctr_ + 1, 1u) == gridDim.x - 1) { dctr_[0] = 0u; dctr_[1] = 0u; __threadfence(); }\n  }\n";
+        return;
       }
       o << "  while (base < R) {\n";
       o << "   {\n";
@@ -1898,7 +1927,9 @@ struct Gen {
     if (role == ROLE_SHARD_FINAL) {
       // small epilogue: one thread per column, consumers of the all-reduced
       // column totals (sharded global stage)
-      o << "#include \"astitch_device.cuh\"\n";
+      if (const char* q = getenv("ASTITCH_LD_HINT"))  // experiments: streaming load qualifiers
+      o << "#define AS_LDQ \"" << (std::string(q) == "none" ? "" : q) << "\"\n";
+    o << "#include \"astitch_device.cuh\"\n";
       o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; void* xbuf; unsigned int gen; };\n";
       o << "extern \"C\" __global__ void __launch_bounds__(256) " << name << "(const Params p) {\n";
       o << "  constexpr long long C = " << C << "LL;\n";

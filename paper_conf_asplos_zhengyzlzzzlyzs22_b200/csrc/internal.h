@@ -101,6 +101,7 @@ struct Mapping {
   int row_unroll = 1;       // U: rows per team per iteration (vertical packing ILP)
   bool prefetch = true;     // software-pipeline the next row's loads
   int single_wave_bps = 0;  // RowTeam: blocks/SM that give every row its own team in one wave (0 = off)
+  bool dyn_tiles = false;   // RowTeam: row tiles taken in address order from a workspace counter
   bool hoist_colvec = true; // keep COLVEC operands in registers across rows
   int tile_rows = 0;        // PackedTile rows per stage
   int stages = 0;           // PackedTile pipeline stages

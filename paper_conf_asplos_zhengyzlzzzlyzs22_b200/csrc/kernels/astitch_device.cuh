@@ -48,15 +48,20 @@ __device__ __forceinline__ Raw<8> ldg(const Raw<8>* p) {
   asm volatile("ld.global.nc.L1::no_allocate.v2.b32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
   return r;
 }
+// load cache qualifiers of the streaming inputs (experiments: e.g. an L2
+// prefetch-size hint), selectable at JIT time like AS_STQ
+#ifndef AS_LDQ
+#define AS_LDQ ".L1::no_allocate"
+#endif
 __device__ __forceinline__ Raw<16> ldg(const Raw<16>* p) {
   Raw<16> r;
-  asm volatile("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+  asm volatile("ld.global.nc" AS_LDQ ".v4.b32 {%0,%1,%2,%3}, [%4];"
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
   return r;
 }
 __device__ __forceinline__ Raw<32> ldg(const Raw<32>* p) {
   Raw<32> r;
-  asm volatile("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+  asm volatile("ld.global.nc" AS_LDQ ".v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w), "=r"(r.a), "=r"(r.b), "=r"(r.c), "=r"(r.d)
                : "l"(p));
   return r;

@@ -339,7 +339,9 @@ void select_mapping(Plan& p) {
 
   // E: the widest power-of-two vector (<= 16 bytes of the narrowest tensor)
   // that divides C, so every chunk is aligned and never straddles a row.
-  int E = std::max(1, 16 / es_min);
+  int vec_bytes = 16;  // 128-bit vectors (ASTITCH_VEC_BYTES=32: 256-bit, experiments)
+  if (const char* vb = getenv("ASTITCH_VEC_BYTES")) vec_bytes = atoi(vb) == 32 ? 32 : 16;
+  int E = std::max(1, vec_bytes / es_min);
   while (E > 1 && (C % E) != 0) E /= 2;
   m.vec_elems = E;
   m.chunks = static_cast<int>((C + E - 1) / E);
@@ -734,10 +736,22 @@ void retune_grid(Plan& p) {
     int64_t clusters = std::max<int64_t>(1, std::min(work_units, wave / m.split));
     m.grid = clusters * m.split;
     m.vertical_trips = (work_units + clusters - 1) / clusters;
+  } else if (m.tmpl == Template::RowTeam && getenv("ASTITCH_NONPERSISTENT") && atoi(getenv("ASTITCH_NONPERSISTENT")) == 1) {
+    // experiments: one row group per CTA, the hardware scheduler streams CTAs
+    m.grid = std::max<int64_t>(1, work_units);
+    m.vertical_trips = 1;
   } else {
     m.grid = std::max<int64_t>(1, std::min(work_units, wave));
     m.vertical_trips = (work_units + m.grid - 1) / m.grid;
   }
+  // Dynamic row tiles: a persistent row team that sweeps several row steps
+  // takes its next tile (RPB x U rows) from a workspace counter, so CTAs
+  // stream through the rows in address order instead of drifting apart on
+  // static strides (measured on B200, 2 reads : 1 write bf16 stream: static
+  // grid-stride 6.4 TB/s, tiles in counter order 7.0 TB/s).  Rows are
+  // independent, so results do not depend on which CTA takes a tile.
+  m.dyn_tiles = m.tmpl == Template::RowTeam && m.prefetch && m.vertical_trips > 1 && p.g.segments_node < 0 &&
+                getenv("ASTITCH_DYN_TILES") && atoi(getenv("ASTITCH_DYN_TILES")) == 1;
   plan_workspace(p);
 }
 
@@ -747,6 +761,10 @@ void plan_workspace(Plan& p) {
   size_t off = 0;
   auto align = [](size_t x) { return (x + 255) & ~static_cast<size_t>(255); };
   const int64_t C = p.desc.cols, R = p.desc.rows;
+  if (p.map.tmpl == Template::RowTeam && p.map.dyn_tiles) {
+    w.barrier = off;               // [0] next tile, [1] CTAs done (self-resetting)
+    off = align(off + 256);
+  }
   if (p.map.tmpl == Template::GlobalSweep) {
     w.barrier = off;
     off = align(off + 256);
@@ -878,7 +896,7 @@ std::string describe_json(const Plan& p) {
     << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
     << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads
     << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
-    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps
+    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"dyn_tiles\":" << (m.dyn_tiles ? "true" : "false")
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
     << ",\"grid\":" << m.grid
