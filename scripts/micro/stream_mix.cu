@@ -33,6 +33,25 @@ __global__ void persistent(const V4* __restrict__ x, const V4* __restrict__ y, V
     for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) z[i] = addv(a[u], b[u]); }
   }
 }
+// (a') persistent grid-stride recording each CTA's finish time (globaltimer)
+template <int U>
+__global__ void persistent_t(const V4* __restrict__ x, const V4* __restrict__ y, V4* __restrict__ z, long long n,
+                             unsigned long long* t_end, unsigned int* smid) {
+  long long stride = (long long)gridDim.x * blockDim.x * U;
+  for (long long base = (long long)blockIdx.x * blockDim.x * U + threadIdx.x; base < n; base += stride) {
+    V4 a[U], b[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) { a[u] = ld(x + i); b[u] = ld(y + i); } }
+#pragma unroll
+    for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) z[i] = addv(a[u], b[u]); }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    unsigned int s; asm volatile("mov.u32 %0, %%smid;" : "=r"(s));
+    t_end[blockIdx.x] = t; smid[blockIdx.x] = s;
+  }
+}
 // (b) one tile per CTA (non-persistent), U vectors per thread
 template <int U>
 __global__ void tiled(const V4* __restrict__ x, const V4* __restrict__ y, V4* __restrict__ z, long long n) {
@@ -189,6 +208,25 @@ int main() {
     if (u == 1) rep(nm, timeit([&] { tiled<1><<<g, t>>>(x, y, z, n); }));
     if (u == 2) rep(nm, timeit([&] { tiled<2><<<g, t>>>(x, y, z, n); }));
     if (u == 4) rep(nm, timeit([&] { tiled<4><<<g, t>>>(x, y, z, n); }));
+  }
+  {  // finish-time spread of the static persistent sweep (tail effect?)
+    const int G = sms;
+    unsigned long long* t_end; unsigned int* smid;
+    cudaMalloc(&t_end, G * 8); cudaMalloc(&smid, G * 4);
+    unsigned long long t0h = 0;
+    for (int r = 0; r < 3; ++r) persistent_t<4><<<G, 512>>>(x, y, z, n, t_end, smid);
+    cudaDeviceSynchronize();
+    unsigned long long h[1024]; unsigned int sid[1024];
+    cudaMemcpy(h, t_end, G * 8, cudaMemcpyDeviceToHost); cudaMemcpy(sid, smid, G * 4, cudaMemcpyDeviceToHost);
+    unsigned long long mn = ~0ULL, mx = 0; double sum = 0;
+    for (int i = 0; i < G; ++i) { mn = h[i] < mn ? h[i] : mn; mx = h[i] > mx ? h[i] : mx; }
+    for (int i = 0; i < G; ++i) sum += (double)(h[i] - mn);
+    printf("static persistent t512 x 1/SM: CTA finish spread %.1f us (mean lag %.1f us)\n", (mx - mn) / 1e3, sum / G / 1e3);
+    // finish lag by SM id range (die halves)
+    double lo = 0, hi = 0; int nlo = 0, nhi = 0;
+    for (int i = 0; i < G; ++i) { if (sid[i] < 74) { lo += (double)(h[i] - mn); ++nlo; } else { hi += (double)(h[i] - mn); ++nhi; } }
+    printf("  mean lag SM 0-73: %.1f us, SM 74-147: %.1f us\n", lo / nlo / 1e3, hi / nhi / 1e3);
+    (void)t0h;
   }
   cudaError_t e = cudaGetLastError();
   printf("status %s\n", cudaGetErrorString(e));
