@@ -119,6 +119,34 @@ __global__ void persistent_pf(const V4* __restrict__ x, const V4* __restrict__ y
   }
 }
 
+// (g) dynamic COARSE tiles: S steps of blockDim x U vectors per grabbed tile,
+// swept in order inside the tile (the shape a deterministic per-tile column
+// partial needs: C5 rows of 2 KB, 128-row tiles = 256 KB per tensor)
+template <int U>
+__global__ void dynamic_coarse(const V4* __restrict__ x, const V4* __restrict__ y, V4* __restrict__ z, long long n,
+                               unsigned long long* counter, int S) {
+  __shared__ long long tq[2];
+  const long long step = (long long)blockDim.x * U, per = step * S, ntiles = (n + per - 1) / per;
+  if (threadIdx.x == 0) tq[0] = (long long)atomicAdd(counter, 1ULL);
+  __syncthreads();
+  long long cur = tq[0];
+  int k = 1;
+  while (cur < ntiles) {
+    if (threadIdx.x == 0) tq[k & 1] = (long long)atomicAdd(counter, 1ULL);  // next tile, read after the sweep
+    for (int s2 = 0; s2 < S; ++s2) {
+      long long base = cur * per + s2 * step + threadIdx.x;
+      V4 a[U], b[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) { a[u] = ld(x + i); b[u] = ld(y + i); } }
+#pragma unroll
+      for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) z[i] = addv(a[u], b[u]); }
+    }
+    __syncthreads();
+    cur = tq[k & 1];
+    __syncthreads();
+    ++k;
+  }
+}
 // (f) dynamic tiles + software pipeline: tile i+1's loads are in flight while
 // tile i is stored, and the index of tile i+2 is grabbed (atomic) one step
 // early, so neither the loads nor the grab sit on the critical path
@@ -208,6 +236,11 @@ int main() {
     if (u == 1) rep(nm, timeit([&] { tiled<1><<<g, t>>>(x, y, z, n); }));
     if (u == 2) rep(nm, timeit([&] { tiled<2><<<g, t>>>(x, y, z, n); }));
     if (u == 4) rep(nm, timeit([&] { tiled<4><<<g, t>>>(x, y, z, n); }));
+  }
+  for (int S : {1, 2, 4, 8, 16}) for (int bps : {1, 2}) {
+    char nm[128];
+    snprintf(nm, sizeof nm, "dynamic coarse S%d U4 t512 x %d/SM", S, bps);
+    rep(nm, timeit([&] { cudaMemsetAsync(ctr, 0, 8); dynamic_coarse<4><<<sms * bps, 512>>>(x, y, z, n, ctr, S); }));
   }
   {  // finish-time spread of the static persistent sweep (tail effect?)
     const int G = sms;
