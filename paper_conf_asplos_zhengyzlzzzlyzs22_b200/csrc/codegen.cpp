@@ -1300,6 +1300,9 @@ struct Gen {
     }
   }
 
+  // partial row written by this block: the CTA, or the counter-ordered tile
+  std::string part_idx = "blockIdx.x";
+  bool dyn_colred = false;  // counter-ordered tiles in the level-0 sweep (m.dyn_colred_rows)
   // block partial of every column reduction -> ws partial row blockIdx.x
   void emit_block_partials() {
     const int ncr = static_cast<int>(p.colreds.size());
@@ -1310,7 +1313,7 @@ struct Gen {
         if (phase_of(id) != cur_level) continue;
         o << "#pragma unroll\n    for (int k = 0; k < NE; ++k) {\n      const long long col = "
           << col_expr("(k / E)", "(k % E)") << ";\n";
-        o << "      if (col < C) part[((long long)blockIdx.x * " << ncr << " + " << q << ") * C + col] = acc" << id
+        o << "      if (col < C) part[((long long)" << part_idx << " * " << ncr << " + " << q << ") * C + col] = acc" << id
           << "[k];\n    }\n";
       }
     } else {
@@ -1327,7 +1330,7 @@ struct Gen {
         o << "    for (long long col = threadIdx.x; col < C; col += blockDim.x) {\n";
         o << "      float a_ = cp_smem[col];\n";
         o << "      for (int t = 1; t < RPB; ++t) a_ = " << (mx ? "fmaxf(a_, cp_smem[t * CC + col])" : "a_ + cp_smem[t * CC + col]") << ";\n";
-        o << "      part[((long long)blockIdx.x * " << ncr << " + " << q << ") * C + col] = a_;\n    }\n";
+        o << "      part[((long long)" << part_idx << " * " << ncr << " + " << q << ") * C + col] = a_;\n    }\n";
       }
     }
     o << "  }\n";
@@ -1343,6 +1346,7 @@ struct Gen {
     o << "    const int G = gridDim.x;\n";
     o << "    const long long W = (C + G - 1) / G;\n";
     o << "    const long long c0 = (long long)blockIdx.x * W;\n";
+    if (dyn_colred) o << "    const int NPART = NT_;\n";
     o << "    const long long c1 = min(C, c0 + W);\n";
     o << "    __shared__ float fin_smem[" << m.threads << "];\n";
     o << "    int P = 1; while (P * 2 * W <= blockDim.x && P * 2 <= 256) P *= 2;\n";
@@ -1356,7 +1360,7 @@ struct Gen {
       bool mx = N(id).sub == ASTITCH_RMAX;
       std::string ident = mx ? "-AS_INF" : "0.f";
       o << "      float t" << id << " = " << ident << ";\n";
-      o << "      if (own) for (int r = pi; r < G; r += P) { const float x_ = as::ld_cg(part + ((long long)r * " << ncr
+      o << "      if (own) for (int r = pi; r < " << (dyn_colred ? "NPART" : "G") << "; r += P) { const float x_ = as::ld_cg(part + ((long long)r * " << ncr
         << " + " << q << ") * C + col); t" << id << " = " << (mx ? "fmaxf(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_") << "; }\n";
       o << "      fin_smem[threadIdx.x] = t" << id << ";\n      __syncthreads();\n";
       o << "      for (int s = P / 2; s > 0; s /= 2) { if (pi < s) fin_smem[threadIdx.x] = "
@@ -1946,8 +1950,10 @@ struct Gen {
       return o.str();
     }
     header(name, m.tmpl == Template::GlobalSweep);
+    dyn_colred = m.tmpl == Template::GlobalSweep && role == ROLE_MAIN && m.dyn_colred_rows > 0;
     if (m.tmpl == Template::GlobalSweep) {
       o << "  unsigned int* bar = (unsigned int*)((char*)p.ws + " << p.ws.barrier << "LL);\n  (void)bar;\n";
+      if (dyn_colred) o << "  const int R_all_ = R;\n";
     }
     if (role == ROLE_FUSED)  // this run's wait status (set only after the grid barriers below)
       o << "  if (blockIdx.x == 0 && threadIdx.x == 0) *(volatile unsigned int*)((unsigned char*)p.xbuf + " << kXErr
@@ -1985,6 +1991,35 @@ struct Gen {
       if (!sweep_here && !colred_here) continue;
       o << "  {  // ---- level " << lv << "\n";
       if (lv > 0) emit_post_colvec_loads();
+      if (colred_here && lv == 0 && dyn_colred) {
+        // counter-ordered tiles of TR_ rows, one column partial per tile
+        const long long TR = m.dyn_colred_rows;
+        const long long NT = (p.desc.rows + TR - 1) / TR;
+        o << "  constexpr int TR_ = " << TR << ";\n  constexpr int NT_ = " << NT << ";\n";
+        o << "  unsigned int* tctr_ = bar + 8;\n  __shared__ int tq_[2];\n";
+        o << "  if (threadIdx.x == 0) tq_[0] = (int)atomicAdd(tctr_, 1u);\n  __syncthreads();\n";
+        o << "  int tile_ = tq_[0];\n  __syncthreads();\n  int tk_ = 0;\n";
+        o << "  while (tile_ < NT_) {\n";
+        o << "   if (threadIdx.x == 0) tq_[(tk_ + 1) & 1] = (int)atomicAdd(tctr_, 1u);\n";
+        o << "   {\n";
+        emit_colred_acc_decl();
+        // the tile is swept by this CTA alone: shadow the row bound and the
+        // unit numbering of the persistent sweep
+        o << "   const int R = min(R_all_, (tile_ + 1) * TR_);\n";
+        o << "   const long long UNIT = (long long)tile_ * (TR_ / (RPB * " << U << ")), NUNITS = 1;\n";
+        o << "   (void)UNIT; (void)NUNITS;\n";
+        emit_sweep(false);
+        part_idx = "tile_";
+        emit_block_partials();
+        part_idx = "blockIdx.x";
+        o << "   }\n   __syncthreads();\n   tile_ = tq_[(tk_ + 1) & 1];\n   __syncthreads();\n   ++tk_;\n  }\n";
+        o << "  as::grid_barrier(bar);\n";
+        o << "  if (blockIdx.x == 0 && threadIdx.x == 0) tctr_[0] = 0u;  // every CTA is past its last grab\n";
+        emit_column_finalize(true);
+        if (lv < D) o << "  as::grid_barrier(bar);\n";
+        o << "  }\n";
+        continue;
+      }
       if (colred_here) emit_colred_acc_decl();
       emit_sweep(lv > 0);
       if (colred_here) {

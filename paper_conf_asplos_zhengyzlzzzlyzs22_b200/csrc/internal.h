@@ -102,6 +102,7 @@ struct Mapping {
   bool prefetch = true;     // software-pipeline the next row's loads
   int single_wave_bps = 0;  // RowTeam: blocks/SM that give every row its own team in one wave (0 = off)
   bool dyn_tiles = false;   // RowTeam: row tiles taken in address order from a workspace counter
+  int dyn_colred_rows = 0;  // GlobalSweep (N=1): rows per counter-ordered tile with its own column partial (0 = off)
   bool hoist_colvec = true; // keep COLVEC operands in registers across rows
   int tile_rows = 0;        // PackedTile rows per stage
   int stages = 0;           // PackedTile pipeline stages

@@ -752,6 +752,19 @@ void retune_grid(Plan& p) {
   // independent, so results do not depend on which CTA takes a tile.
   m.dyn_tiles = m.tmpl == Template::RowTeam && m.prefetch && m.vertical_trips > 1 && p.g.segments_node < 0 &&
                 getenv("ASTITCH_DYN_TILES") && atoi(getenv("ASTITCH_DYN_TILES")) == 1;
+  // Global sweep of one column-reduction level on one GPU: counter-ordered
+  // tiles of 128 rows, each with its own column partial (tile-ordered final
+  // combine: deterministic, independent of which CTA took which tile)
+  m.dyn_colred_rows = 0;
+  if (m.tmpl == Template::GlobalSweep && p.max_level == 1 && p.desc.shard_world <= 1 &&
+      (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0 && !p.colreds.empty() &&
+      getenv("ASTITCH_DYN_COLRED") && atoi(getenv("ASTITCH_DYN_COLRED")) == 1) {
+    const int step = m.rows_per_block * m.row_unroll;
+    int tr = 128;
+    if (const char* e = getenv("ASTITCH_DYN_COLRED_ROWS")) tr = std::max(1, atoi(e));
+    tr = std::max(step, (tr / step) * step);
+    if ((R + tr - 1) / tr > m.grid) m.dyn_colred_rows = tr;  // more tiles than CTAs
+  }
   plan_workspace(p);
 }
 
@@ -769,7 +782,9 @@ void plan_workspace(Plan& p) {
     w.barrier = off;
     off = align(off + 256);
     w.partials = off;
-    off = align(off + static_cast<size_t>(p.map.grid) * p.colreds.size() * C * 4);
+    const int64_t nparts = p.map.dyn_colred_rows > 0 ? (R + p.map.dyn_colred_rows - 1) / p.map.dyn_colred_rows
+                                                     : p.map.grid;
+    off = align(off + static_cast<size_t>(nparts) * p.colreds.size() * C * 4);
     w.colvals = off;
     off = align(off + std::max<size_t>(p.post_colvecs.size(), 1) * C * 4 + C * 4 * p.colreds.size());
     w.globals = off;
@@ -896,7 +911,7 @@ std::string describe_json(const Plan& p) {
     << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
     << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads
     << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
-    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"dyn_tiles\":" << (m.dyn_tiles ? "true" : "false")
+    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"dyn_tiles\":" << (m.dyn_tiles ? "true" : "false") << ",\"dyn_colred_rows\":" << m.dyn_colred_rows
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
     << ",\"grid\":" << m.grid
