@@ -519,3 +519,15 @@ def test_parity_random_shapes(seed):
         x = gen.generate(cfg, spec)
         got, plan = run_gpu(spec, x, return_plan=True)
         _compare(spec, got, evaluate(spec, x))
+
+
+@pytest.mark.xfail(strict=False, reason="cancellation-prone column means are plain fp32 column sums "
+                                        "(column analogue of reading R7b: DESIGN.md NEXT)")
+def test_parity_batchnorm_two_rows_column_mean_cancellation():
+    """Known limitation found by scripts/fuzz_shapes.py (seed 244): BatchNorm
+    over 2 rows x 4513 fp32 columns; columns with |x1 - x2| << |x| lose
+    ~5e-5 relative accuracy in x - mean."""
+    spec = specs.get("bn", rows=2, cols=4513)
+    x = gen.generate("bn", spec)
+    got = run_gpu(spec, x)
+    _compare(spec, got, evaluate(spec, x))
