@@ -194,6 +194,20 @@ typedef struct {
  * Errors: ERR_SHAPE (rows < 0, cols < 1, overflow), ERR_UNSUPPORTED,
  * ERR_RESOURCE (STRICT flag and no one-kernel plan), ERR_CUDA (NVRTC / load). */
 astitch_status astitch_plan(astitch_graph_t g, const astitch_plan_desc* desc, astitch_plan_t* out);
+/* astitch_plan with explicit overrides of the planner's choices, for
+ * experiments and tests: `tuning` is NULL or "key=value,..." with integer
+ * values; keys: threads, unroll, team, bps (fixed blocks/SM, no
+ * assume-relax-apply), vec_bytes (16|32), hoist (0|1), tile_stages, tile_rows,
+ * tile_threads, split, split_threads, stream (1 force row_stream, 0 never),
+ * stage (1: row_stream stages rows in smem), stage_kb, portable_clusters,
+ * dyn_colred_rows (global sweep: counter-ordered row tiles).  Values a
+ * template cannot use are ignored.  The plan is a pure function of
+ * (graph, desc, tuning): the library reads no environment variables for
+ * planning or code generation.  describe() reports the string.
+ * Errors: as astitch_plan, plus ERR_INVALID_ARGUMENT for an unknown key or a
+ * non-integer value. */
+astitch_status astitch_plan_ex(astitch_graph_t g, const astitch_plan_desc* desc, const char* tuning,
+                               astitch_plan_t* out);
 astitch_status astitch_plan_destroy(astitch_plan_t p);
 /* Bytes of device workspace astitch_run needs (0 if none). */
 astitch_status astitch_plan_workspace_bytes(astitch_plan_t p, size_t* bytes);

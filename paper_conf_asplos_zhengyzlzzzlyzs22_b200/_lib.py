@@ -77,6 +77,7 @@ _sig = {
                                            ct.POINTER(ct.c_int64), ct.POINTER(ct.c_int64)]),
     "astitch_graph_output": (ct.c_int, [_vp, ct.c_int32, ct.c_int, _i32p]),
     "astitch_plan": (ct.c_int, [_vp, ct.POINTER(PlanDesc), ct.POINTER(_vp)]),
+    "astitch_plan_ex": (ct.c_int, [_vp, ct.POINTER(PlanDesc), ct.c_char_p, ct.POINTER(_vp)]),
     "astitch_plan_destroy": (ct.c_int, [_vp]),
     "astitch_plan_workspace_bytes": (ct.c_int, [_vp, ct.POINTER(ct.c_size_t)]),
     "astitch_plan_describe": (ct.c_int, [_vp, ct.c_char_p, ct.c_size_t, ct.POINTER(ct.c_size_t)]),

@@ -146,11 +146,18 @@ class Plan:
     """A planned + JIT-compiled stitch op (astitch_plan)."""
 
     def __init__(self, graph: Graph, rows: int, cols: int, device: int = 0, flags: int = 0,
-                 shard_rank: int = 0, shard_world: int = 1, sm_count: int = 0):
+                 shard_rank: int = 0, shard_world: int = 1, sm_count: int = 0, tune: str | dict | None = None):
+        """`tune`: explicit planner overrides for experiments / tests
+        (astitch_plan_ex), "key=value,..." or a dict, e.g. {"threads": 256}."""
         d = _lib.PlanDesc(rows=int(rows), cols=int(cols), device=int(device), shard_rank=int(shard_rank),
                           shard_world=int(shard_world), flags=int(flags), sm_count=int(sm_count), reserved=0)
         h = ct.c_void_p()
-        check(lib.astitch_plan(graph.handle, ct.byref(d), ct.byref(h)), "astitch_plan")
+        if isinstance(tune, dict):
+            tune = ",".join(f"{k}={int(v)}" for k, v in tune.items())
+        if tune:
+            check(lib.astitch_plan_ex(graph.handle, ct.byref(d), tune.encode(), ct.byref(h)), "astitch_plan_ex")
+        else:
+            check(lib.astitch_plan(graph.handle, ct.byref(d), ct.byref(h)), "astitch_plan")
         self._h = h
         self.rows, self.cols, self.device = int(rows), int(cols), int(device)
         self.ragged = graph.ragged

@@ -133,8 +133,8 @@ struct Gen {
       case ASTITCH_DIV:
         if (bconst) return "(" + a + " * " + flit(1.0 / bn.cval) + ")";
         return "as::fdiv(" + a + ", " + b + ")";
-      case ASTITCH_MAX: return "fmaxf(" + a + ", " + b + ")";
-      case ASTITCH_MIN: return "fminf(" + a + ", " + b + ")";
+      case ASTITCH_MAX: return "as::nmax(" + a + ", " + b + ")";
+      case ASTITCH_MIN: return "as::nmin(" + a + ", " + b + ")";
       case ASTITCH_POW:
         if (bconst && bn.cval == std::floor(bn.cval) && bn.cval >= 0 && bn.cval <= 8) {
           int n = static_cast<int>(bn.cval);
@@ -152,11 +152,6 @@ struct Gen {
   void header(const std::string& name, bool cooperative_sync) {
     (void)cooperative_sync;
     o << "// generated by astitch codegen: " << template_name(m.tmpl) << " role " << role << "\n";
-    if (const char* q = getenv("ASTITCH_ST_HINT"))  // experiments: output store cache qualifier
-      if (std::string(q) == ".cs" || std::string(q) == ".wt" || std::string(q) == ".cg")
-        o << "#define AS_STQ \"" << q << "\"\n";
-    if (const char* q = getenv("ASTITCH_LD_HINT"))  // experiments: streaming load qualifiers
-      o << "#define AS_LDQ \"" << (std::string(q) == "none" ? "" : q) << "\"\n";
     o << "#include \"astitch_device.cuh\"\n";
     o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; void* xbuf; unsigned int gen; };\n";
     o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") ";
@@ -411,8 +406,8 @@ struct Gen {
       case ASTITCH_SUB: return a - b;
       case ASTITCH_MUL: return a * b;
       case ASTITCH_DIV: return a / b;
-      case ASTITCH_MAX: return std::fmax(a, b);
-      case ASTITCH_MIN: return std::fmin(a, b);
+      case ASTITCH_MAX: return (std::isnan(a) || std::isnan(b)) ? a + b : std::fmax(a, b);
+      case ASTITCH_MIN: return (std::isnan(a) || std::isnan(b)) ? a + b : std::fmin(a, b);
       case ASTITCH_POW: return std::pow(a, b);
       default: return std::nan("");
     }
@@ -422,10 +417,8 @@ struct Gen {
   // one thread), every column valid up to C (no masks: an invalid element
   // would have to be excluded from both the terms and the count)
   bool shifted_sum_ok() const {
-    return !masked && !split && T <= 32 && (m.tmpl == Template::RowTeam || m.tmpl == Template::PackedTile) &&
-           !env_on("ASTITCH_PRECISE_F64");
+    return !masked && !split && T <= 32 && (m.tmpl == Template::RowTeam || m.tmpl == Template::PackedTile);
   }
-  bool seg_lookahead() const { return !env_on("ASTITCH_SEG_LOOKAHEAD1"); }
   // a FULL value whose (transitive) consumers include a reduction
   bool feeds_reduction(int i) const {
     for (int u : I(i).consumers) {
@@ -436,14 +429,13 @@ struct Gen {
     }
     return false;
   }
-  static bool env_on(const char* name) { return getenv(name) && atoi(getenv(name)) == 1; }
   // FULL light op computed over every chunk of an absorbed-mask row (no
   // live-chunk branch): its invalid elements take the known value inval[i]
   // whenever the row's scalars are finite, i.e. whenever the row has a valid
   // prefix; no reduction reads it (so fully-masked rows cannot leak a NaN into
   // a row scalar) and it is not buffered across a barrier
   bool light_unguarded(int i) const {
-    if (!absorb || kf || !inval_known[i] || env_on("ASTITCH_GUARD_LIGHT")) return false;
+    if (!absorb || kf || !inval_known[i]) return false;
     const Node& nd = N(i);
     bool light = false;
     if (nd.type == NodeType::Binary)
@@ -456,7 +448,7 @@ struct Gen {
   // FULL output whose invalid elements are known to be exactly 0 under the
   // absorbed mask: stored without per-element selects
   bool store_absorbed(int id) const {
-    return absorb && masked && inval_known[id] && inval[id] == 0.0 && !env_on("ASTITCH_STORE_SELECT");
+    return absorb && masked && inval_known[id] && inval[id] == 0.0;
   }
 
   // abstract evaluation for substitute S; returns true if every row (and
@@ -552,7 +544,7 @@ struct Gen {
         std::string val = ref(nd.a, "k", sfx);
         std::string okc = act;
         if (check && !absorb) okc += " && " + col_expr("(k / E)", "(k % E)") + " < " + lim;
-        if (mx) o << "      if (" << okc << ") acc" << id << "[k] = fmaxf(acc" << id << "[k], " << val << ");\n";
+        if (mx) o << "      if (" << okc << ") acc" << id << "[k] = as::nmax(acc" << id << "[k], " << val << ");\n";
         else o << "      if (" << okc << ") acc" << id << "[k] += " << val << ";\n";
         o << "    }\n";
         continue;
@@ -756,8 +748,8 @@ struct Gen {
           return "(" + x + " * " + buf + ")";
         }
         return "(" + x + " / " + y + ")";
-      case ASTITCH_MAX: return "fmax(" + x + ", " + y + ")";
-      case ASTITCH_MIN: return "fmin(" + x + ", " + y + ")";
+      case ASTITCH_MAX: return "as::dmaxn(" + x + ", " + y + ")";
+      case ASTITCH_MIN: return "as::dminn(" + x + ", " + y + ")";
     }
     return x;
   }
@@ -1036,7 +1028,6 @@ struct Gen {
   // one ping-pong half of the software-pipelined row loop: loads of the rows
   // one stride ahead go to buffer `nx` while the rows of `base` are computed
   // from buffer `cu` (no register copies between the halves)
-  bool dyn = false;  // dynamic row tiles (m.dyn_tiles) in the ping-pong loop being emitted
   void emit_pingpong_half(bool post, const std::string& cu, const std::string& nx) {
     const std::string su = "_u";
     const std::string rt = rowt();
@@ -1044,41 +1035,23 @@ struct Gen {
       const std::string us = std::to_string(u);
       o << "    const " << rt << " row" << u << " = base + " << u << " * RPB + team;\n";
       o << "    const bool act" << u << " = row" << u << " < R;\n";
-      if (ragged) {
-        o << "    " << limdecl("lim" + us, "act" + us, "row" + us, "nsg" + us + cu) << "\n";
-      } else {
-        o << "    const int lim" << u << " = "
-          << (masked ? "act" + us + " ? " + lim_expr("row" + us) + " : 0" : "(int)C") << ";\n";
-      }
+      o << "    const int lim" << u << " = "
+        << (masked ? "act" + us + " ? " + lim_expr("row" + us) + " : 0" : "(int)C") << ";\n";
       o << "    (void)lim" << u << ";\n";
     }
     for (int u = 0; u < U; ++u) {
       const std::string us = std::to_string(u);
-      o << "    {\n      const " << rt << " nrow = " << (dyn ? "nbase" : "base + rstride") << " + " << u
+      o << "    {\n      const " << rt << " nrow = base + rstride + " << u
         << " * RPB + team;\n";
       o << "      const bool pact = nrow < R;\n";
-      if (ragged) {
-        o << "      nsg" << us << nx << " = (nnsg" << us << " >= 0) ? __ldg(SG + nnsg" << us << ") : make_int4(0, 0, 0, 0);\n";
-        o << "      " << limdecl("plim", "pact", "nrow", "nsg" + us + nx) << "\n";
-      } else {
-        o << "      const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
-      }
+      o << "      const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
       o << "      (void)plim;\n";
       emit_loads("nrow", "pact", "plim", su + us + nx, false);
-      if (ragged)
-        o << "      nnsg" << us << " = (nrow + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(nrow + rstride)) : -1;\n";
       o << "    }\n";
     }
-    // dynamic tiles: the index of the tile after next, grabbed while this
-    // tile computes (read after the step's barrier)
-    if (dyn) o << "    if (threadIdx.x == 0) dq_[" << (cu == "a" ? 0 : 1) << "] = (int)atomicAdd(dctr_, 1u);\n";
     for (int u = 0; u < U; ++u) {
       std::string s = su + std::to_string(u) + cu;
       std::string row = "row" + std::to_string(u), act = "act" + std::to_string(u), lim = "lim" + std::to_string(u);
-      if (ragged) {
-        emit_row_block(post, s, row, act, lim);
-        continue;
-      }
       o << "    {\n";
       emit_unpack(s, lim);
       emit_colvecs(true);
@@ -1105,56 +1078,21 @@ struct Gen {
     // early-unpack copy form: C3 143.8 vs 146.1 us (80 vs 72 registers), C2 at
     // 32768 rows 29.1 vs 29.9 us, C5 and fig6a equal.  Packed varlen rows keep
     // the copy form (their KF-specialised body would be emitted 2 x (V+1)
-    // times).  ASTITCH_PINGPONG=0 selects the copy form for experiments.
-    const char* pp_env = getenv("ASTITCH_PINGPONG");
-    const bool pp_ragged = env_on("ASTITCH_PINGPONG_RAGGED");
-    dyn = false;
-    if (pf && !(pp_env && atoi(pp_env) == 0) && (!ragged || pp_ragged)) {
-      dyn = m.dyn_tiles && !ragged && m.tmpl == Template::RowTeam;
-      if (dyn) {
-        o << "  unsigned int* dctr_ = (unsigned int*)((char*)p.ws + " << p.ws.barrier << "LL);\n";
-        o << "  __shared__ int dq_[2];\n  constexpr int TILE_ = RPB * " << U << ";\n";
-        o << "  if (threadIdx.x == 0) { dq_[0] = (int)atomicAdd(dctr_, 1u); dq_[1] = (int)atomicAdd(dctr_, 1u); }\n";
-        o << "  __syncthreads();\n  base = dq_[0] * TILE_;\n  " << rt << " nbase = dq_[1] * TILE_;\n  __syncthreads();\n";
-      }
+    // times).
+    if (pf && !ragged) {
       // ping-pong buffers a / b
       for (int u = 0; u < U; ++u)
         for (const char* bf : {"a", "b"})
           for (size_t q = 0; q < streams.size(); ++q)
             o << "  " << raw_t(streams[q]) << " r" << q << su << u << bf << "[V];\n";
-      if (ragged)
-        for (int u = 0; u < U; ++u)
-          o << "  int4 nsg" << u << "a, nsg" << u << "b; int nnsg" << u << ";\n";
       for (int u = 0; u < U; ++u) {
         const std::string us = std::to_string(u);
         o << "  {\n    const " << rt << " nrow = base + " << u << " * RPB + team;\n";
         o << "    const bool pact = nrow < R;\n";
-        if (ragged) {
-          // packed varlen rows: segment entries per buffer, the next row's
-          // segment index searched one step ahead (nnsg)
-          o << "    nsg" << us << "a = pact ? as::seg_find<NSEG>(SG, (int)nrow) : make_int4(0, 0, 0, 0);\n";
-          o << "    nnsg" << us << " = (nrow + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(nrow + rstride)) : -1;\n";
-          o << "    " << limdecl("plim", "pact", "nrow", "nsg" + us + "a") << "\n";
-        } else {
-          o << "    const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
-        }
+        o << "    const int plim = " << (masked ? "pact ? " + lim_expr("nrow") + " : 0" : "(int)C") << ";\n";
         o << "    (void)plim;\n";
         emit_loads("nrow", "pact", "plim", su + std::to_string(u) + "a", false);
         o << "  }\n";
-      }
-      if (dyn) {
-        o << "  while (base < R) {\n";
-        o << "   {\n";
-        emit_pingpong_half(post, "a", "b");
-        o << "   }\n    __syncthreads();\n    base = nbase;\n    nbase = dq_[0] * TILE_;\n    __syncthreads();\n"
-          << "    if (base >= R) break;\n";
-        o << "   {\n";
-        emit_pingpong_half(post, "b", "a");
-        o << "   }\n    __syncthreads();\n    base = nbase;\n    nbase = dq_[1] * TILE_;\n    __syncthreads();\n  }\n";
-        // the last CTA to finish resets the counters for the next run
-        o << "  if (threadIdx.x == 0) {\n    __threadfence();\n"
-          << "    if (atomicAdd(dctr_ + 1, 1u) == gridDim.x - 1) { dctr_[0] = 0u; dctr_[1] = 0u; __threadfence(); }\n  }\n";
-        return;
       }
       o << "  while (base < R) {\n";
       o << "   {\n";
@@ -1180,8 +1118,7 @@ struct Gen {
           // two-deep segment lookahead: the entry of the row after the
           // prefetched one is searched an iteration early, so the prefetch's
           // load addresses never wait on a binary search
-          if (seg_lookahead())
-            o << "  int nnsg" << u << " = (prow" << u << " + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(prow" << u
+          o << "  int nnsg" << u << " = (prow" << u << " + rstride < R) ? as::seg_find_idx<NSEG>(SG, (int)(prow" << u
               << " + rstride)) : -1;\n";
         }
         o << "  {\n    const bool pact = prow" << u << " < R;\n";
@@ -1201,24 +1138,14 @@ struct Gen {
                            (ragged && pf) ? "nsg" + std::to_string(u) : "") << "\n";
       o << "    (void)lim" << u << ";\n";
     }
-    // early unpack (default): convert the prefetched raw vectors to fp32
-    // before the next prefetch is issued into the same registers.  The copy
-    // form (ASTITCH_LATE_UNPACK=1) keeps a raw copy live across the prefetch;
-    // on B200 its register moves stall on the loads of the next row
-    // (long scoreboard at the loop back-edge, C3 ncu source view).
-    const bool early = pf && !(getenv("ASTITCH_LATE_UNPACK") && atoi(getenv("ASTITCH_LATE_UNPACK")) == 1);
-    if (pf && early) {
+    // early unpack: convert the prefetched raw vectors to fp32 before the
+    // next prefetch is issued into the same registers (a raw copy kept live
+    // across the prefetch stalled on the next row's loads: long scoreboard at
+    // the loop back-edge, C3 ncu source view, round 1)
+    if (pf) {
       for (int u = 0; u < U; ++u) {
         std::string s = su + std::to_string(u);
         emit_unpack_convert(s, s + "n");
-      }
-    } else if (pf) {
-      for (int u = 0; u < U; ++u) {
-        std::string s = su + std::to_string(u);
-        for (size_t q = 0; q < streams.size(); ++q) {
-          o << "    " << raw_t(streams[q]) << " r" << q << s << "[V];\n";
-          o << "#pragma unroll\n    for (int j = 0; j < V; ++j) r" << q << s << "[j] = r" << q << s << "n[j];\n";
-        }
       }
     }
     if (pf) {
@@ -1227,7 +1154,7 @@ struct Gen {
         o << "    {\n";
         o << "      const " << rt << " nrow = base + rstride + " << u << " * RPB + team;\n";
         o << "      const bool pact = nrow < R;\n";
-        const bool la = ragged && seg_lookahead();
+        const bool la = ragged;
         if (la) o << "      nsg" << u << " = (nnsg" << u << " >= 0) ? __ldg(SG + nnsg" << u << ") : make_int4(0, 0, 0, 0);\n";
         else if (ragged) o << "      nsg" << u << " = pact ? as::seg_find<NSEG>(SG, (int)nrow) : make_int4(0, 0, 0, 0);\n";
         o << "      " << limdecl("plim", "pact", "nrow", ragged ? "nsg" + std::to_string(u) : "") << "\n";
@@ -1243,7 +1170,7 @@ struct Gen {
         emit_loads("row" + std::to_string(u), "act" + std::to_string(u), "lim" + std::to_string(u), s, true);
       }
     }
-    early_unpack = pf && early;
+    early_unpack = pf;
     for (int u = 0; u < U; ++u) {
       std::string s = su + std::to_string(u);
       std::string row = "row" + std::to_string(u), act = "act" + std::to_string(u), lim = "lim" + std::to_string(u);
@@ -1261,9 +1188,7 @@ struct Gen {
   // whole padded row dominate, and the 5x code loses 1-4%).
   void emit_row_block(bool post, const std::string& s, const std::string& row, const std::string& act,
                       const std::string& lim) {
-    const bool kf_env = getenv("ASTITCH_KF") && atoi(getenv("ASTITCH_KF")) == 1;  // experiments: padded masks too
-    const bool spec = (ragged || (masked && kf_env)) && m.tmpl == Template::RowTeam && V >= 2 && !split &&
-                      !(getenv("ASTITCH_NO_KF") && atoi(getenv("ASTITCH_NO_KF")) == 1);
+    const bool spec = ragged && m.tmpl == Template::RowTeam && V >= 2 && !split;
     if (!spec) {
       o << "    {\n";
       emit_unpack(s, lim);
@@ -1329,7 +1254,7 @@ struct Gen {
         o << "    __syncthreads();\n";
         o << "    for (long long col = threadIdx.x; col < C; col += blockDim.x) {\n";
         o << "      float a_ = cp_smem[col];\n";
-        o << "      for (int t = 1; t < RPB; ++t) a_ = " << (mx ? "fmaxf(a_, cp_smem[t * CC + col])" : "a_ + cp_smem[t * CC + col]") << ";\n";
+        o << "      for (int t = 1; t < RPB; ++t) a_ = " << (mx ? "as::nmax(a_, cp_smem[t * CC + col])" : "a_ + cp_smem[t * CC + col]") << ";\n";
         o << "      part[((long long)" << part_idx << " * " << ncr << " + " << q << ") * C + col] = a_;\n    }\n";
       }
     }
@@ -1361,10 +1286,10 @@ struct Gen {
       std::string ident = mx ? "-AS_INF" : "0.f";
       o << "      float t" << id << " = " << ident << ";\n";
       o << "      if (own) for (int r = pi; r < " << (dyn_colred ? "NPART" : "G") << "; r += P) { const float x_ = as::ld_cg(part + ((long long)r * " << ncr
-        << " + " << q << ") * C + col); t" << id << " = " << (mx ? "fmaxf(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_") << "; }\n";
+        << " + " << q << ") * C + col); t" << id << " = " << (mx ? "as::nmax(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_") << "; }\n";
       o << "      fin_smem[threadIdx.x] = t" << id << ";\n      __syncthreads();\n";
       o << "      for (int s = P / 2; s > 0; s /= 2) { if (pi < s) fin_smem[threadIdx.x] = "
-        << (mx ? "fmaxf(fin_smem[threadIdx.x], fin_smem[threadIdx.x + s])" : "fin_smem[threadIdx.x] + fin_smem[threadIdx.x + s]")
+        << (mx ? "as::nmax(fin_smem[threadIdx.x], fin_smem[threadIdx.x + s])" : "fin_smem[threadIdx.x] + fin_smem[threadIdx.x + s]")
         << "; __syncthreads(); }\n";
       o << "      t" << id << " = fin_smem[threadIdx.x - pi];\n      __syncthreads();\n";
     }
@@ -1376,7 +1301,7 @@ struct Gen {
         std::string slot = "colpart[" + std::to_string(q) + "LL * C + col]";
         std::string t = "t" + std::to_string(p.colreds[q]);
         o << "        " << slot << " = (p.flags & 1) ? "
-          << (mx ? "fmaxf(" + slot + ", " + t + ")" : "(" + slot + " + " + t + ")") << " : " << t << ";\n";
+          << (mx ? "as::nmax(" + slot + ", " + t + ")" : "(" + slot + " + " + t + ")") << " : " << t << ";\n";
       }
     } else {
       emit_colvec_chain("t");
@@ -1424,7 +1349,7 @@ struct Gen {
       bool mx = N(id).sub == ASTITCH_RMAX;
       o << "      float t" << id << " = " << (mx ? "-AS_INF" : "0.f") << ";\n";
       o << "      for (int q = 0; q < XW; ++q) { const float x_ = as::ld_cg(slots + ((long long)q * NCR + " << q
-        << ") * C + col); t" << id << " = " << (mx ? "fmaxf(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_")
+        << ") * C + col); t" << id << " = " << (mx ? "as::nmax(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_")
         << "; }\n";
     }
     emit_colvec_chain("t");
@@ -1868,7 +1793,7 @@ struct Gen {
         if (tail) o << "(" << col_expr("(k / E)", "(k % E)") << " < C) ? " << ref(N(r).a, "k", "") << " : " << ident << ";\n";
         else o << ref(N(r).a, "k", "") << ";\n";
         if (precise[r]) o << "        ad" << r << " += as::TreeD<NE>::reduce(t_);\n";
-        else if (mx) o << "        a" << r << " = fmaxf(a" << r << ", as::Tree<NE, true>::reduce(t_));\n";
+        else if (mx) o << "        a" << r << " = as::nmax(a" << r << ", as::Tree<NE, true>::reduce(t_));\n";
         else o << "        a" << r << " += as::Tree<NE, false>::reduce(t_);\n";
         o << "      }\n";
       }
@@ -1931,9 +1856,7 @@ struct Gen {
     if (role == ROLE_SHARD_FINAL) {
       // small epilogue: one thread per column, consumers of the all-reduced
       // column totals (sharded global stage)
-      if (const char* q = getenv("ASTITCH_LD_HINT"))  // experiments: streaming load qualifiers
-      o << "#define AS_LDQ \"" << (std::string(q) == "none" ? "" : q) << "\"\n";
-    o << "#include \"astitch_device.cuh\"\n";
+      o << "#include \"astitch_device.cuh\"\n";
       o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; void* xbuf; unsigned int gen; };\n";
       o << "extern \"C\" __global__ void __launch_bounds__(256) " << name << "(const Params p) {\n";
       o << "  constexpr long long C = " << C << "LL;\n";

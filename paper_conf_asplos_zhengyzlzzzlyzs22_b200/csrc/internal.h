@@ -101,7 +101,6 @@ struct Mapping {
   int row_unroll = 1;       // U: rows per team per iteration (vertical packing ILP)
   bool prefetch = true;     // software-pipeline the next row's loads
   int single_wave_bps = 0;  // RowTeam: blocks/SM that give every row its own team in one wave (0 = off)
-  bool dyn_tiles = false;   // RowTeam: row tiles taken in address order from a workspace counter
   int dyn_colred_rows = 0;  // GlobalSweep (N=1): rows per counter-ordered tile with its own column partial (0 = off)
   bool hoist_colvec = true; // keep COLVEC operands in registers across rows
   int tile_rows = 0;        // PackedTile rows per stage
@@ -117,6 +116,29 @@ struct Mapping {
   int bank_conflict_ways = 1;
   std::string reason;       // selector decision trace
 };
+
+// ------------------------------------------------------------------ tuning
+// Explicit overrides of the planner's choices (astitch_plan_ex's tuning
+// string "key=value,..."; experiments and tests).  0 / -1 = the planner
+// decides.  A plan is a pure function of (graph, desc, tuning): the library
+// reads no environment variables for planning or code generation.
+struct Tuning {
+  int threads = 0;          // block size
+  int unroll = 0;           // rows per team per iteration (U)
+  int team = 0;             // lanes per row (row-wise plans)
+  int bps = 0;              // fixed blocks-per-SM target (no assume-relax-apply bisection)
+  int vec_bytes = 0;        // 16 or 32: vector width of a chunk
+  int hoist = -1;           // 1 / 0: keep COLVEC operands in registers (or re-read per row)
+  int tile_stages = 0, tile_rows = 0, tile_threads = 0;  // packed_tile pipeline
+  int split = 0, split_threads = 0;                       // split_row cluster size / CTA size
+  int stream = -1;          // 1: force row_stream, 0: never stream
+  int stage = 0;            // 1: row_stream stages the row's inputs in smem
+  int stage_kb = 0;         // row_stream staging budget per CTA (KB)
+  int portable_clusters = 0;  // 1: never ask for 16-CTA clusters
+  int dyn_colred_rows = 0;  // global sweep: rows per counter-ordered tile (0 = static)
+  std::string text;         // the string it was parsed from (describe())
+};
+bool parse_tuning(const char* s, Tuning& t, std::string& err);
 
 // ------------------------------------------------------------------ plan
 struct Kernel {
@@ -149,6 +171,7 @@ struct WsLayout {
 struct Plan {
   Graph g;
   astitch_plan_desc desc{};
+  Tuning tune;
   int sm_count = 148;
   std::vector<NodeInfo> info;
   std::vector<std::vector<int>> groups;

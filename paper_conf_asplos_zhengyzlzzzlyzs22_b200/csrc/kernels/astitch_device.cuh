@@ -272,6 +272,12 @@ template <int DT> __device__ __forceinline__ void st_scalar(void* base, long lon
 // MUFU-based with cancellation-free forms (reading R6: no tanh.approx).
 __device__ __forceinline__ float ex2(float x) { float r; asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
 __device__ __forceinline__ float rcp(float x) { float r; asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
+// NaN-propagating max / min (reading R12: RMAX propagates NaN, as the oracle's
+// numpy max does; fmaxf would drop it).  One FMNMX with the .NaN modifier.
+__device__ __forceinline__ float nmax(float a, float b) { float r; asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r; }
+__device__ __forceinline__ float nmin(float a, float b) { float r; asm("min.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r; }
+__device__ __forceinline__ double dmaxn(double a, double b) { return (a != a || b != b) ? a + b : fmax(a, b); }
+__device__ __forceinline__ double dminn(double a, double b) { return (a != a || b != b) ? a + b : fmin(a, b); }
 __device__ __forceinline__ float rsq(float x) { float r; asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
 __device__ __forceinline__ float sqrt_(float x) { float r; asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }
 __device__ __forceinline__ float fexp(float x) { return ex2(x * 1.4426950408889634f); }
@@ -322,8 +328,8 @@ __device__ __forceinline__ f2 fma2(f2 a, f2 b, f2 c) {
 }
 __device__ __forceinline__ f2 abs2(f2 a) { return f2{fabsf(a.x), fabsf(a.y)}; }
 __device__ __forceinline__ f2 neg2(f2 a) { return f2{-a.x, -a.y}; }
-__device__ __forceinline__ f2 max2(f2 a, f2 b) { return f2{fmaxf(a.x, b.x), fmaxf(a.y, b.y)}; }
-__device__ __forceinline__ f2 min2(f2 a, f2 b) { return f2{fminf(a.x, b.x), fminf(a.y, b.y)}; }
+__device__ __forceinline__ f2 max2(f2 a, f2 b) { return f2{nmax(a.x, b.x), nmax(a.y, b.y)}; }
+__device__ __forceinline__ f2 min2(f2 a, f2 b) { return f2{nmin(a.x, b.x), nmin(a.y, b.y)}; }
 __device__ __forceinline__ f2 ex2_2(f2 a) { return f2{ex2(a.x), ex2(a.y)}; }
 __device__ __forceinline__ f2 rcp_2(f2 a) { return f2{rcp(a.x), rcp(a.y)}; }
 __device__ __forceinline__ f2 fexp2(f2 a) { return ex2_2(mul2(a, bc2(1.4426950408889634f))); }
@@ -372,7 +378,7 @@ template <int T> __device__ __forceinline__ float team_sum(float v) {
 }
 template <int T> __device__ __forceinline__ float team_max(float v) {
 #pragma unroll
-  for (int o = (T < 32 ? T : 32) / 2; o > 0; o /= 2) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  for (int o = (T < 32 ? T : 32) / 2; o > 0; o /= 2) v = nmax(v, __shfl_xor_sync(0xffffffffu, v, o));
   return v;
 }
 // team larger than a warp == whole block: warp tree, then a fixed-order
@@ -455,7 +461,7 @@ __device__ __forceinline__ float cluster_team_reduce(float v, float* scratch, fl
 #pragma unroll
   for (int q = 0; q < K; ++q) {
     const float x = ld_dsmem_f32(slot, static_cast<u32>(q));
-    r = MAX ? fmaxf(r, x) : r + x;
+    r = MAX ? nmax(r, x) : r + x;
   }
   cluster_sync_all();
   return r;
@@ -481,7 +487,7 @@ template <int N, bool MAX> struct Tree {
       constexpr int H = N / 2;
       float l = Tree<H, MAX>::reduce(a);
       float r = Tree<N - H, MAX>::reduce(a + H);
-      return MAX ? fmaxf(l, r) : l + r;
+      return MAX ? nmax(l, r) : l + r;
     }
   }
 };

@@ -339,8 +339,8 @@ void select_mapping(Plan& p) {
 
   // E: the widest power-of-two vector (<= 16 bytes of the narrowest tensor)
   // that divides C, so every chunk is aligned and never straddles a row.
-  int vec_bytes = 16;  // 128-bit vectors (ASTITCH_VEC_BYTES=32: 256-bit, experiments)
-  if (const char* vb = getenv("ASTITCH_VEC_BYTES")) vec_bytes = atoi(vb) == 32 ? 32 : 16;
+  const Tuning& tu = p.tune;
+  int vec_bytes = tu.vec_bytes == 32 ? 32 : 16;  // 128-bit vectors (tuning vec_bytes=32: 256-bit)
   int E = std::max(1, vec_bytes / es_min);
   while (E > 1 && (C % E) != 0) E /= 2;
   m.vec_elems = E;
@@ -397,8 +397,7 @@ void select_mapping(Plan& p) {
   while (k_wave < 8 && R * (k_wave * 2) <= sms) k_wave *= 2;
   // rows <= 9: non-portable clusters of 16 (validated at load time against
   // cuOccupancyMaxActiveClusters, else back to 8)
-  if (k_wave == 8 && R * 16 <= sms && !p.portable_clusters &&
-      !(getenv("ASTITCH_PORTABLE_CLUSTERS") && atoi(getenv("ASTITCH_PORTABLE_CLUSTERS")) == 1))
+  if (k_wave == 8 && R * 16 <= sms && !p.portable_clusters && !tu.portable_clusters)
     k_wave = 16;
 
   if (has_colred || p.max_level > 0) {
@@ -415,19 +414,13 @@ void select_mapping(Plan& p) {
       if (p.info[i].live && p.info[i].cls == OpClass::ReduceRow) has_rowred = true;
     // a multi-warp team reduces through block-wide smem: one team per block
     m.threads = (m.team > 32 && has_rowred) ? m.team : std::max(512, m.team);
-    if (const char* ft = getenv("ASTITCH_FORCE_THREADS")) {  // tuning knob for experiments
-      int t = atoi(ft);
-      if (t >= m.team && t <= 1024 && t % m.team == 0) m.threads = t;
-    }
+    if (tu.threads >= m.team && tu.threads <= 1024 && tu.threads % m.team == 0) m.threads = tu.threads;
     m.rows_per_block = m.threads / m.team;
     int ne = m.chunks_per_lane * E;
     // rows per team per iteration: ~64 input elements in flight per lane
     // (measured on B200 for C5: U=4 reaches 98% of the copy roofline, U=2 94%)
     m.row_unroll = std::max(1, std::min(4, 64 / std::max(1, ne * nfull_in)));
-    if (const char* fu = getenv("ASTITCH_FORCE_UNROLL")) {  // tuning knob for experiments
-      int u = atoi(fu);
-      if (u >= 1 && u <= 8) m.row_unroll = u;
-    }
+    if (tu.unroll >= 1 && tu.unroll <= 8) m.row_unroll = tu.unroll;
     // a6: block-level combine of the teams' column partials in smem
     if (m.rows_per_block > 1 && has_colred) {
       int64_t cb = static_cast<int64_t>(m.rows_per_block) * m.team * m.chunks_per_lane * E * 4;
@@ -445,13 +438,10 @@ void select_mapping(Plan& p) {
     // the KF chunk-count specialisation (codegen) 81 us vs 95 us at T=16;
     // padded masked rows (C3) are store-bound and keep T=16 without it.
     choose_team(1024, ragged ? 64 : (has_mask ? 32 : 16), ragged ? 64 : 32);
-    if (const char* ft = getenv("ASTITCH_FORCE_TEAM")) {  // tuning knob for experiments
-      int t = atoi(ft);
-      if (t >= 1 && t <= 1024 && ((t & (t - 1)) == 0 || t % 32 == 0)) {
-        m.team = t;
-        m.chunks_per_lane = (chunks + t - 1) / t;
-        m.lane_util = static_cast<double>(chunks) / (t * m.chunks_per_lane);
-      }
+    if (const int t = tu.team; t >= 1 && t <= 1024 && ((t & (t - 1)) == 0 || t % 32 == 0)) {
+      m.team = t;
+      m.chunks_per_lane = (chunks + t - 1) / t;
+      m.lane_util = static_cast<double>(chunks) / (t * m.chunks_per_lane);
     }
     if (no_pack && m.team < 32 && chunks >= 1) {
       // ablation: XLA-style one row per warp (no horizontal packing)
@@ -474,22 +464,10 @@ void select_mapping(Plan& p) {
     bool tile_common = !no_tma && row16 && p.global_fulls.empty() && R >= 4096;
     bool packed_ok = tile_common && !no_pack && !has_mask && !has_colvec_in && row_bytes_max <= 512 &&
                      m.lane_util < 0.95 && chunks <= 32;
-    int in_row_bytes = 0;
-    for (int id : g.inputs)
-      if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live)
-        in_row_bytes += static_cast<int>(C) * dtype_size(g.nodes[id].dtype);
-    // Team tiles: rows of up to a warp's worth of chunks staged by TMA bulk
-    // copies (deep async pipeline: bytes in flight no longer tied to registers)
-    // (measured on B200: for masked rows the register-prefetching row team is
-    // faster than per-row valid-prefix bulk copies, so masks stay on row teams)
-    // Measured on B200 (C2: 8.7 vs 8.0 us, C3: 3.8 vs 4.6 TB/s) the register
-    // row team beats TMA-staged team tiles whenever a power-of-two team tiles
-    // the row, so team tiles are opt-in (ASTITCH_TEAM_TILES=1); the T=1
-    // packed tiles (rows a team cannot tile, C4) stay the default.
-    const char* tt_env = getenv("ASTITCH_TEAM_TILES");
-    bool team_tile_ok = tile_common && tt_env && atoi(tt_env) == 1 && !packed_ok && !has_mask &&
-                        m.team <= 32 && m.team >= 1 &&
-                        in_row_bytes > 0 && in_row_bytes * (256 / m.team) <= 48 * 1024;
+    // (Round 1 measured TMA-staged tiles with a power-of-two TEAM per row
+    // against register row teams on B200: C2 8.7 vs 8.0 us, C3 3.8 vs 4.6 TB/s;
+    // the register row team wins whenever a team tiles the row, so only the
+    // T=1 packed tiles -- rows no team can tile, C4 -- use the TMA template.)
     // Task splitting (rule P:L270): rows < blocks-per-wave and row > 1024.
     // B200 threshold (reading R15): measured on <64,30000> fp32 (120 KB rows)
     // one block per row is still faster (4.2 vs 4.7 us, latency-bound), on
@@ -497,28 +475,17 @@ void select_mapping(Plan& p) {
     const bool force_split = (p.desc.flags & ASTITCH_FLAG_FORCE_SPLIT) != 0;
     bool split_rule = !no_split && !ragged && R < blocks_per_wave_1024 && C > 1024 &&
                       (force_split || C * es_max >= 256 * 1024);
-    if (packed_ok || team_tile_ok) {
+    if (packed_ok) {
       m.tmpl = Template::PackedTile;
-      if (packed_ok) {
-        m.team = 1;
-        m.chunks_per_lane = chunks;
-        m.lane_util = 1.0;
-        m.threads = 128;
-        m.tile_rows = 128;
-      } else {
-        m.threads = 256;
-        int teams = m.threads / m.team;
-        int tr = 1;
-        while (tr * 2 * in_row_bytes <= 24 * 1024) tr *= 2;
-        m.tile_rows = std::max(teams, (tr / teams) * teams);
-      }
+      m.team = 1;
+      m.chunks_per_lane = chunks;
+      m.lane_util = 1.0;
+      m.threads = 128;
+      m.tile_rows = 128;
       m.stages = 4;  // prefetch distance 2 tiles + 2 tiles draining (bulk stores)
-      if (const char* fs = getenv("ASTITCH_TILE")) {  // tuning knob: "stages,tile_rows,threads"
-        int s = 0, tr = 0, th = 0;
-        if (sscanf(fs, "%d,%d,%d", &s, &tr, &th) >= 1 && s >= 3 && s <= 8) m.stages = s;
-        if (th >= 32 && th <= 1024 && th % 32 == 0 && th % m.team == 0) m.threads = th;
-        if (tr >= 1 && tr % (m.threads / m.team) == 0) m.tile_rows = tr;
-      }
+      if (tu.tile_stages >= 3 && tu.tile_stages <= 8) m.stages = tu.tile_stages;
+      if (tu.tile_threads >= 32 && tu.tile_threads <= 1024 && tu.tile_threads % 32 == 0) m.threads = tu.tile_threads;
+      if (tu.tile_rows >= 1 && tu.tile_rows % m.threads == 0) m.tile_rows = tu.tile_rows;
       m.rows_per_block = m.threads / m.team;
       // stage bytes: input tiles + output tiles that cannot be written in
       // place over an input tile of the same element size (mirrors codegen)
@@ -541,15 +508,9 @@ void select_mapping(Plan& p) {
         m.stages--;
         m.smem_bytes = m.stages * m.tile_rows * (in_bytes + out_bytes) + 64 * m.stages;
       }
-      if (packed_ok) {
-        m.bank_conflict_ways = lds128_conflict_ways(static_cast<int>(C) * es_min);
-        why << "row of " << chunks << " x " << (E * es_min)
-            << "B chunks does not tile a power-of-two team -> TMA-staged packed tiles, thread per row; ";
-      } else {
-        why << "TMA bulk-staged tiles of " << m.tile_rows << " rows (" << m.stages
-            << "-stage mbarrier pipeline), team of " << m.team << " lanes x " << m.chunks_per_lane
-            << " chunks per row from smem" << (has_mask ? ", valid-prefix copies per row" : "") << "; ";
-      }
+      m.bank_conflict_ways = lds128_conflict_ways(static_cast<int>(C) * es_min);
+      why << "row of " << chunks << " x " << (E * es_min)
+          << "B chunks does not tile a power-of-two team -> TMA-staged packed tiles, thread per row; ";
     } else if (split_rule && p.global_fulls.empty()) {
       // Task splitting: each row is split over a thread-block cluster
       // of K CTAs (K ~ blocks-per-wave / rows, power of two, <= 8 portable);
@@ -557,14 +518,8 @@ void select_mapping(Plan& p) {
       m.tmpl = Template::SplitRow;
       m.split = std::max(2, k_wave);
       m.threads = 512;
-      if (const char* fs = getenv("ASTITCH_FORCE_SPLIT")) {  // tuning knob: "K" or "K,threads"
-        int kk = atoi(fs);
-        if (kk >= 1 && kk <= 16 && (kk & (kk - 1)) == 0) m.split = kk;
-        if (const char* c = strchr(fs, ',')) {
-          int t = atoi(c + 1);
-          if (t >= 32 && t <= 1024 && t % 32 == 0) m.threads = t;
-        }
-      }
+      if (const int kk = tu.split; kk >= 1 && kk <= 16 && (kk & (kk - 1)) == 0) m.split = kk;
+      if (const int t = tu.split_threads; t >= 32 && t <= 1024 && t % 32 == 0) m.threads = t;
       m.team = m.split * m.threads;
       m.chunks_per_lane = std::max(1, (chunks + m.team - 1) / m.team);
       m.lane_util = static_cast<double>(chunks) / (static_cast<double>(m.team) * m.chunks_per_lane);
@@ -577,10 +532,7 @@ void select_mapping(Plan& p) {
       m.tmpl = Template::RowTeam;
       // a multi-warp team reduces through block-wide smem: one team per block
       m.threads = m.team > 32 ? m.team : 256;
-      if (const char* ft = getenv("ASTITCH_FORCE_THREADS")) {  // tuning knob for experiments
-        int t = atoi(ft);
-        if (t >= m.team && t <= 1024 && t % m.team == 0 && t % 32 == 0) m.threads = t;
-      }
+      if (const int t = tu.threads; t >= m.team && t <= 1024 && t % m.team == 0 && t % 32 == 0) m.threads = t;
       // One wave of teams for every row: when the rows need at most 28 warps
       // per SM (>= 72 registers per thread), give each row its own team in a
       // single wave of 4-warp blocks, sized to exactly the warps needed (no
@@ -589,7 +541,7 @@ void select_mapping(Plan& p) {
       // bf16): 128 x 7 blocks/SM, one row per warp, 6.79 us vs 7.10 us for
       // 256-thread blocks at 2 blocks/SM sweeping two rows per warp.
       m.single_wave_bps = 0;
-      if (m.team <= 32 && !getenv("ASTITCH_FORCE_THREADS")) {
+      if (m.team <= 32 && tu.threads == 0) {
         const int64_t teams_per_warp = 32 / m.team;
         const int64_t warps = (R + teams_per_warp - 1) / teams_per_warp;
         const int64_t warps_per_sm = (warps + sms - 1) / std::max(1, sms);
@@ -599,11 +551,7 @@ void select_mapping(Plan& p) {
         }
       }
       m.rows_per_block = m.threads / m.team;
-      m.row_unroll = 1;
-      if (const char* fu = getenv("ASTITCH_FORCE_UNROLL")) {  // tuning knob for experiments
-        int u = atoi(fu);
-        if (u >= 1 && u <= 8) m.row_unroll = u;
-      }
+      m.row_unroll = (tu.unroll >= 1 && tu.unroll <= 8) ? tu.unroll : 1;
       why << (m.single_wave_bps ? "one wave of teams (one row per team); " : "") << "row team of " << m.team << " lanes x " << m.chunks_per_lane << " chunks ("
           << m.rows_per_block << " rows / block, packing), regional via shuffles" << (m.team > 32 ? "+smem" : "")
           << "; ";
@@ -617,10 +565,9 @@ void select_mapping(Plan& p) {
     // buffer over the on-chip limit is demotion to global; a
     // per-row re-read keeps it in one pass of the grid with no barrier.
     constexpr int kStreamNE = 128;
-    const bool stream_ok = !has_mask && p.global_fulls.empty() &&
-                           !(getenv("ASTITCH_NO_STREAM") && atoi(getenv("ASTITCH_NO_STREAM")) == 1) &&
+    const bool stream_ok = !has_mask && p.global_fulls.empty() && tu.stream != 0 &&
                            (m.tmpl == Template::RowTeam || m.tmpl == Template::SplitRow);
-    const bool force_stream = getenv("ASTITCH_FORCE_STREAM") && atoi(getenv("ASTITCH_FORCE_STREAM")) == 1;
+    const bool force_stream = tu.stream == 1;
     if (stream_ok && (m.chunks_per_lane * E > kStreamNE || force_stream || p.stream_fallback)) {
       m.tmpl = Template::RowStream;
       m.threads = 512;
@@ -641,13 +588,13 @@ void select_mapping(Plan& p) {
       // Measured on B200 (LM-head softmax 4096 x 128256 bf16: 741 us staged vs
       // 660 us re-reading L2; fp32 4096 x 100000: 1896 vs 1049 us): staging
       // costs occupancy (one 512-thread CTA per SM) that the L2-resident
-      // re-reads do not, so it is opt-in (ASTITCH_STAGE=1) until the staged
+      // re-reads do not, so it is opt-in (tuning stage=1) until the staged
       // pass pipelines its loads.
-      const bool no_stage = !(getenv("ASTITCH_STAGE") && atoi(getenv("ASTITCH_STAGE")) == 1);
+      const bool no_stage = tu.stage != 1;
       m.stage_row = false;
       m.smem_bytes = 0;
       int stage_budget = 72 * 1024;  // per CTA: keeps 3 CTAs of 512 threads per SM
-      if (const char* sb = getenv("ASTITCH_STAGE_KB")) stage_budget = std::max(8, atoi(sb)) * 1024;
+      if (tu.stage_kb > 0) stage_budget = std::max(8, tu.stage_kb) * 1024;
       if (!no_stage && in_row_bytes > 0) {
         int k = m.split;
         while (k < 8 && (in_row_bytes + k - 1) / k > stage_budget) k *= 2;
@@ -680,7 +627,7 @@ void select_mapping(Plan& p) {
     for (int i = 0; i < static_cast<int>(g.nodes.size()); ++i)
       if (p.info[i].live && !p.info[i].post && g.nodes[i].kind == ASTITCH_COLVEC) ++ncv;
     m.hoist_colvec = (ncv * m.chunks_per_lane * E) <= 48;
-    if (const char* fh = getenv("ASTITCH_HOIST")) m.hoist_colvec = atoi(fh) == 1;  // tuning knob
+    if (tu.hoist >= 0) m.hoist_colvec = tu.hoist == 1;
   }
 
   // a7: assume-relax-apply.  Assume the 32-register bound (full occupancy),
@@ -711,10 +658,7 @@ void select_mapping(Plan& p) {
   int by_threads = std::max(1, max_threads_sm / m.threads);
   int by_smem = m.smem_bytes > 0 ? (228 * 1024) / (m.smem_bytes + 1024) : 32;
   m.blocks_per_sm = std::max(1, std::min({32, by_threads, by_smem}));
-  if (const char* fb = getenv("ASTITCH_FORCE_BPS")) {  // tuning knob: fixed occupancy target
-    int b = atoi(fb);
-    if (b >= 1 && b <= 32) m.blocks_per_sm = b;
-  }
+  if (tu.bps >= 1 && tu.bps <= 32) m.blocks_per_sm = tu.bps;
   m.reg_cap = std::min(255, (65536 / (m.blocks_per_sm * m.threads)) & ~7);
 
   m.reason = why.str();
@@ -736,33 +680,19 @@ void retune_grid(Plan& p) {
     int64_t clusters = std::max<int64_t>(1, std::min(work_units, wave / m.split));
     m.grid = clusters * m.split;
     m.vertical_trips = (work_units + clusters - 1) / clusters;
-  } else if (m.tmpl == Template::RowTeam && getenv("ASTITCH_NONPERSISTENT") && atoi(getenv("ASTITCH_NONPERSISTENT")) == 1) {
-    // experiments: one row group per CTA, the hardware scheduler streams CTAs
-    m.grid = std::max<int64_t>(1, work_units);
-    m.vertical_trips = 1;
   } else {
     m.grid = std::max<int64_t>(1, std::min(work_units, wave));
     m.vertical_trips = (work_units + m.grid - 1) / m.grid;
   }
-  // Dynamic row tiles: a persistent row team that sweeps several row steps
-  // takes its next tile (RPB x U rows) from a workspace counter, so CTAs
-  // stream through the rows in address order instead of drifting apart on
-  // static strides (measured on B200, 2 reads : 1 write bf16 stream: static
-  // grid-stride 6.4 TB/s, tiles in counter order 7.0 TB/s).  Rows are
-  // independent, so results do not depend on which CTA takes a tile.
-  m.dyn_tiles = m.tmpl == Template::RowTeam && m.prefetch && m.vertical_trips > 1 && p.g.segments_node < 0 &&
-                getenv("ASTITCH_DYN_TILES") && atoi(getenv("ASTITCH_DYN_TILES")) == 1;
   // Global sweep of one column-reduction level on one GPU: counter-ordered
   // tiles of 128 rows, each with its own column partial (tile-ordered final
   // combine: deterministic, independent of which CTA took which tile)
   m.dyn_colred_rows = 0;
   if (m.tmpl == Template::GlobalSweep && p.max_level == 1 && p.desc.shard_world <= 1 &&
-      (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0 && !p.colreds.empty() &&
-      getenv("ASTITCH_DYN_COLRED") && atoi(getenv("ASTITCH_DYN_COLRED")) == 1) {
+      (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0 && !p.colreds.empty() && p.tune.dyn_colred_rows > 0 &&
+      R < (1LL << 30)) {
     const int step = m.rows_per_block * m.row_unroll;
-    int tr = 128;
-    if (const char* e = getenv("ASTITCH_DYN_COLRED_ROWS")) tr = std::max(1, atoi(e));
-    tr = std::max(step, (tr / step) * step);
+    int tr = std::max(step, (p.tune.dyn_colred_rows / step) * step);
     if ((R + tr - 1) / tr > m.grid) m.dyn_colred_rows = tr;  // more tiles than CTAs
   }
   plan_workspace(p);
@@ -774,10 +704,6 @@ void plan_workspace(Plan& p) {
   size_t off = 0;
   auto align = [](size_t x) { return (x + 255) & ~static_cast<size_t>(255); };
   const int64_t C = p.desc.cols, R = p.desc.rows;
-  if (p.map.tmpl == Template::RowTeam && p.map.dyn_tiles) {
-    w.barrier = off;               // [0] next tile, [1] CTAs done (self-resetting)
-    off = align(off + 256);
-  }
   if (p.map.tmpl == Template::GlobalSweep) {
     w.barrier = off;
     off = align(off + 256);
@@ -881,7 +807,7 @@ std::string describe_json(const Plan& p) {
   };
   o << "{\"rows\":" << p.desc.rows << ",\"cols\":" << p.desc.cols << ",\"device\":" << p.desc.device
     << ",\"shard_rank\":" << p.desc.shard_rank << ",\"shard_world\":" << p.desc.shard_world
-    << ",\"sm_count\":" << p.sm_count;
+    << ",\"sm_count\":" << p.sm_count << ",\"flags\":" << p.desc.flags << ",\"tuning\":\"" << esc(p.tune.text) << "\"";
   o << ",\"ops\":[";
   for (size_t i = 0; i < g.nodes.size(); ++i) {
     const Node& nd = g.nodes[i];
@@ -911,7 +837,7 @@ std::string describe_json(const Plan& p) {
     << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
     << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads
     << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
-    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"dyn_tiles\":" << (m.dyn_tiles ? "true" : "false") << ",\"dyn_colred_rows\":" << m.dyn_colred_rows
+    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"dyn_colred_rows\":" << m.dyn_colred_rows
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
     << ",\"grid\":" << m.grid

@@ -86,7 +86,10 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
   // assume-relax-apply as a bisection on blocks per SM: the largest occupancy
   // whose register bound (65536 / (bps * threads)) compiles without spills
   int good = 0, bad = 0;  // best spill-free / smallest spilling bps seen
-  for (int attempt = 0; attempt < 10; ++attempt) {
+  // generate + compile for the current p.map (called again after the loop if
+  // its attempts run out, so the kernel always matches the final mapping and
+  // workspace layout)
+  auto gen_compile = [&]() -> astitch_status {
     std::string base = std::string("astitch_") + template_name(p.map.tmpl) + role_suffix(role);
     k.name = base;
     k.source = generate_kernel(p, role, base);
@@ -107,8 +110,11 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
                            (p.map.tmpl == Template::SplitRow || p.map.tmpl == Template::RowStream) && p.map.split > 1;
     k.cluster = clustered ? p.map.split : 1;
     if (!compile) return ASTITCH_OK;
-    astitch_status st = compile_and_inspect(p, k, load);
-    if (st != ASTITCH_OK) return st;
+    return compile_and_inspect(p, k, load);
+  };
+  for (int attempt = 0; attempt < 10; ++attempt) {
+    astitch_status st = gen_compile();
+    if (st != ASTITCH_OK || !compile) return st;
     // non-portable clusters (9-16 CTAs): keep them only if every row's
     // cluster is co-resident in one wave; else fall back to portable 8
     if (k.cluster > 8 && load && k.max_clusters >= 0 && k.max_clusters * k.cluster < k.grid && !p.portable_clusters) {
@@ -117,12 +123,11 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
       good = bad = 0;
       continue;
     }
-    if (!may_relax || getenv("ASTITCH_FORCE_BPS")) return ASTITCH_OK;
+    if (!may_relax || p.tune.bps > 0) return ASTITCH_OK;
     const int cur = p.map.blocks_per_sm;
     // (measured on B200, fp32 softmax rows of 4096 x C: a 116-byte spill
     // (C=30000) costs less than streaming, 448+ bytes (C >= 60000) more)
-    if (k.spill_bytes >= 256 && cur == 1 && !p.stream_fallback &&
-        !(getenv("ASTITCH_NO_STREAM") && atoi(getenv("ASTITCH_NO_STREAM")) == 1) &&
+    if (k.spill_bytes >= 256 && cur == 1 && !p.stream_fallback && p.tune.stream != 0 &&
         (p.map.tmpl == Template::RowTeam || p.map.tmpl == Template::SplitRow) && p.g.lengths_node < 0 &&
         p.g.segments_node < 0 && p.global_fulls.empty()) {
       // the row does not fit the team's registers even at one block per SM:
@@ -157,10 +162,49 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
     p.map.reg_cap = std::min(255, (65536 / (p.map.blocks_per_sm * p.map.threads)) & ~7);
     retune_grid(p);
   }
-  return ASTITCH_OK;
+  // attempts exhausted after a retune: the last compiled kernel may not match
+  // p.map / p.ws any more -- compile the final mapping once more
+  return gen_compile();
 }
 
 }  // namespace
+
+namespace astitch {
+// "key=value,key=value" -> Tuning (integers only; unknown keys are errors)
+bool parse_tuning(const char* s, Tuning& t, std::string& err) {
+  t = Tuning();
+  if (!s) return true;
+  t.text = s;
+  std::string str(s);
+  size_t pos = 0;
+  while (pos < str.size()) {
+    size_t end = str.find(',', pos);
+    if (end == std::string::npos) end = str.size();
+    std::string item = str.substr(pos, end - pos);
+    pos = end + 1;
+    if (item.empty()) continue;
+    size_t eq = item.find('=');
+    if (eq == std::string::npos) { err = "tuning item without '=': " + item; return false; }
+    std::string key = item.substr(0, eq), val = item.substr(eq + 1);
+    char* ep = nullptr;
+    long v = strtol(val.c_str(), &ep, 10);
+    if (val.empty() || *ep != '\0') { err = "tuning value is not an integer: " + item; return false; }
+    const int iv = static_cast<int>(v);
+    struct { const char* k; int* f; } keys[] = {
+        {"threads", &t.threads}, {"unroll", &t.unroll}, {"team", &t.team}, {"bps", &t.bps},
+        {"vec_bytes", &t.vec_bytes}, {"hoist", &t.hoist}, {"tile_stages", &t.tile_stages},
+        {"tile_rows", &t.tile_rows}, {"tile_threads", &t.tile_threads}, {"split", &t.split},
+        {"split_threads", &t.split_threads}, {"stream", &t.stream}, {"stage", &t.stage},
+        {"stage_kb", &t.stage_kb}, {"portable_clusters", &t.portable_clusters},
+        {"dyn_colred_rows", &t.dyn_colred_rows}};
+    bool found = false;
+    for (auto& kv : keys)
+      if (key == kv.k) { *kv.f = iv; found = true; }
+    if (!found) { err = "unknown tuning key: " + key; return false; }
+  }
+  return true;
+}
+}  // namespace astitch
 
 namespace astitch {
 // (comm.cpp) build one more kernel of a plan, e.g. the fused sharded role
@@ -170,6 +214,11 @@ astitch_status build_plan_kernel(Plan& p, int role, Kernel& k) { return build_ke
 extern "C" {
 
 astitch_status astitch_plan(astitch_graph_t gr, const astitch_plan_desc* desc, astitch_plan_t* out) {
+  return astitch_plan_ex(gr, desc, nullptr, out);
+}
+
+astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc, const char* tuning,
+                               astitch_plan_t* out) {
   if (!gr || !desc || !out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL graph, desc or out");
   *out = nullptr;
   if (desc->rows < 0) return fail(ASTITCH_ERR_SHAPE, "rows < 0");
@@ -185,6 +234,10 @@ astitch_status astitch_plan(astitch_graph_t gr, const astitch_plan_desc* desc, a
     Plan& p = *plan;
     p.g = gr->g;
     p.desc = *desc;
+    {
+      std::string terr;
+      if (!parse_tuning(tuning, p.tune, terr)) return fail(ASTITCH_ERR_INVALID_ARGUMENT, terr);
+    }
     if (p.desc.shard_world == 0) p.desc.shard_world = 1;
     p.device = desc->device;
     p.sm_count = desc->sm_count > 0 ? desc->sm_count : 148;

@@ -82,13 +82,13 @@ def device_inputs(spec: dict, inputs: dict, device="cuda"):
     return [to_torch(inputs[n], d, device) for n, _, d in spec["inputs"]]
 
 
-def run_gpu(spec: dict, inputs: dict, flags: int = 0, plan=None, return_plan=False):
+def run_gpu(spec: dict, inputs: dict, flags: int = 0, plan=None, return_plan=False, tune=None):
     """Plan (unless given) and run `spec` on cuda:0; returns {output: np.float64}."""
     import torch
     import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
     if plan is None:
         g = A.Graph.from_spec(spec)
-        plan = A.Plan(g, spec["rows"], spec["cols"], device=torch.cuda.current_device(), flags=flags)
+        plan = A.Plan(g, spec["rows"], spec["cols"], device=torch.cuda.current_device(), flags=flags, tune=tune)
     ins = device_inputs(spec, inputs)
     outs = plan.alloc_outputs()
     if spec.get("segments"):  # packed rows: elements past a row's 16-byte chunks are never written

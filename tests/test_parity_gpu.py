@@ -239,17 +239,6 @@ def test_virtual_shards(cfg, rows, cols, world):
             check_close(got, ref[name], dt, spec_tol(spec), f"{cfg}:{name} sharded")
 
 
-@pytest.mark.parametrize("cfg,rows", [("C2", 4500), ("remote", 5000), ("C1", 9000)])
-def test_team_tiles_optin(cfg, rows, monkeypatch):
-    """TMA-staged team tiles (opt-in template) stay correct."""
-    monkeypatch.setenv("ASTITCH_TEAM_TILES", "1")
-    spec = specs.get(cfg, rows=rows)
-    x = gen.generate(cfg, spec)
-    got, plan = run_gpu(spec, x, return_plan=True)
-    assert plan.describe()["mapping"]["template"] == "packed_tile"
-    _compare(spec, got, evaluate(spec, x))
-
-
 def test_full_c1_c2():
     for cfg in ("C1", "C2"):
         spec = specs.get(cfg)
@@ -358,17 +347,14 @@ def test_one_kernel_no_memset_per_run(cfg):
                                                  ("lmsoftmax", 64, None, False), ("C1", 37, 600_000, False),
                                                  ("lmsoftmax", 64, None, "stage"), ("C2", 40, 100_000, "stage"),
                                                  ("C4", 300, 60_000, "stage")])
-def test_parity_row_stream(cfg, rows, cols, force, monkeypatch):
+def test_parity_row_stream(cfg, rows, cols, force):
     """Rows longer than a team's registers: streamed column tiles, one pass per
     row-reduction level (forced on small shapes; chosen by the planner for
     multi-MB rows; "stage": inputs kept in the cluster's shared memory)."""
-    if force is True:
-        monkeypatch.setenv("ASTITCH_FORCE_STREAM", "1")
-    if force == "stage":
-        monkeypatch.setenv("ASTITCH_STAGE", "1")
+    tune = {"stream": 1} if force is True else ({"stage": 1} if force == "stage" else None)
     spec = specs.get(cfg, rows=rows, cols=cols)
     x = gen.generate(cfg, spec)
-    got, plan = run_gpu(spec, x, return_plan=True)
+    got, plan = run_gpu(spec, x, return_plan=True, tune=tune)
     d = plan.describe()
     assert d["mapping"]["template"] == "row_stream" and d["kernel_count"] == 1
     assert d["kernels"][0]["spill_bytes"] == 0
