@@ -107,7 +107,8 @@ int astitch_abi_version(void);
  * a FULL value; broadcast ROW takes a ROWVEC, broadcast COL a COLVEC). */
 astitch_status astitch_graph_create(astitch_graph_t* out);
 astitch_status astitch_graph_destroy(astitch_graph_t g);
-/* A tensor input of kind FULL / ROWVEC / COLVEC and storage dtype F32 / BF16 / F16. */
+/* A tensor input of kind FULL / ROWVEC / COLVEC and storage dtype F32 / BF16 / F16
+ * (or kind LENGTHS with dtype I32: a mask bound later by astitch_graph_set_mask). */
 astitch_status astitch_graph_input(astitch_graph_t g, astitch_kind kind, astitch_dtype dtype,
                                    astitch_value_t* out);
 /* A SCALAR constant (applied in fp32 on the device, fp64 in the oracle). */
@@ -127,6 +128,14 @@ astitch_status astitch_graph_broadcast(astitch_graph_t g, astitch_axis axis, ast
  * RMAX) and written as 0 in FULL outputs.  At most one mask per graph. */
 astitch_status astitch_graph_lengths(astitch_graph_t g, int64_t rows_per_segment,
                                      astitch_value_t* out);
+/* The same mask in two steps (SURVEY 8(b)'s form): `lengths` is an existing
+ * input created by astitch_graph_input(g, ASTITCH_LENGTHS, ASTITCH_I32, &v);
+ * this call binds it as the graph's key-padding mask with rows_per_segment.
+ * Errors: ERR_INVALID_ARGUMENT (NULL g, bad value, rows_per_segment < 1),
+ * ERR_INVALID_GRAPH (not a LENGTHS input, or the graph already has a mask /
+ * segments).  astitch_plan fails with ERR_INVALID_GRAPH if a LENGTHS input
+ * was never bound. */
+astitch_status astitch_graph_set_mask(astitch_graph_t g, astitch_value_t lengths, int64_t rows_per_segment);
 /* Packed variable-length rows ("varlen" layout: irregular shapes without
  * padding, Sec. 3.3 Challenge II).  Adds an
  * int32 SEGMENTS input (next in input order) of nseg entries of 4 int32
@@ -166,7 +175,8 @@ enum {
   ASTITCH_FLAG_FORCE_GLOBAL = 1u << 1,  /* ablation: demote regional -> global (Table 4)*/
   ASTITCH_FLAG_NO_PACK = 1u << 2,       /* ablation: no horizontal packing (team = warp)*/
   ASTITCH_FLAG_NO_SPLIT = 1u << 3,      /* ablation: never split long rows             */
-  ASTITCH_FLAG_STRICT_SINGLE_KERNEL = 1u << 4, /* fail with ERR_RESOURCE rather than 2 kernels */
+  ASTITCH_FLAG_STRICT_SINGLE_KERNEL = 1u << 4, /* ERR_RESOURCE if the planned one-wave grid is
+                                           not co-resident (instead of shrinking it) */
   ASTITCH_FLAG_NO_TMA = 1u << 5,        /* do not use the TMA-staged packed template   */
   ASTITCH_FLAG_NO_PREFETCH = 1u << 6,   /* no software prefetch of the next row        */
   ASTITCH_FLAG_LAUNCH_CHECK = 1u << 7,  /* synchronise + check after every launch (debug)*/
@@ -192,7 +202,12 @@ typedef struct {
  * kernel and compile it for sm_100a with NVRTC (unless FLAG_NO_COMPILE) and
  * load it on desc.device (unless device == -1).
  * Errors: ERR_SHAPE (rows < 0, cols < 1, overflow), ERR_UNSUPPORTED,
- * ERR_RESOURCE (STRICT flag and no one-kernel plan), ERR_CUDA (NVRTC / load). */
+ * ERR_RESOURCE (STRICT flag and the planned grid is not co-resident), ERR_CUDA
+ * (NVRTC / load).  Every plan is ONE kernel: when a staged buffer would exceed
+ * the shared memory of a block, the planner demotes the mapping (fewer
+ * pipeline stages / tile rows / teams per block, or a register row team
+ * instead of a staged tile: the paper's "until the memory usage is under the
+ * limit"); describe()["demotions"] lists what it changed. */
 astitch_status astitch_plan(astitch_graph_t g, const astitch_plan_desc* desc, astitch_plan_t* out);
 /* astitch_plan with explicit overrides of the planner's choices, for
  * experiments and tests: `tuning` is NULL or "key=value,..." with integer
@@ -298,7 +313,7 @@ astitch_status astitch_plan_colpart(astitch_plan_t p, size_t* byte_offset, size_
  * identical on every rank.  Every rank must make the same sequence of
  * astitch_run_fused calls; the ranks' kernels must be able to run at the same
  * time (separate GPUs, or grids that fit together).  A rank that does not
- * arrive within ~2 s makes the waiting kernels give up (no hang): their
+ * arrive within 5 s makes the waiting kernels give up (no hang): their
  * outputs are then invalid and astitch_peer_status reports timed_out = 1.
  * Errors: ERR_INVALID_ARGUMENT (mismatched plan / peer, peer not mapped),
  * ERR_UNSUPPORTED (> 64 ranks), ERR_CUDA (allocation, IPC, launch). */

@@ -72,6 +72,7 @@ _sig = {
     "astitch_graph_reduce": (ct.c_int, [_vp, ct.c_int, ct.c_int, ct.c_int32, _i32p]),
     "astitch_graph_broadcast": (ct.c_int, [_vp, ct.c_int, ct.c_int32, _i32p]),
     "astitch_graph_lengths": (ct.c_int, [_vp, ct.c_int64, _i32p]),
+    "astitch_graph_set_mask": (ct.c_int, [_vp, ct.c_int32, ct.c_int64]),
     "astitch_graph_segments": (ct.c_int, [_vp, ct.c_int32, ct.c_int64, _i32p]),
     "astitch_segments_layout": (ct.c_int, [ct.c_int32, ct.POINTER(ct.c_int64), _i32p, _i32p,
                                            ct.POINTER(ct.c_int64), ct.POINTER(ct.c_int64)]),

@@ -59,6 +59,11 @@ class Graph:
         check(lib.astitch_graph_lengths(self._h, int(rows_per_segment), ct.byref(v)), "astitch_graph_lengths")
         return v.value
 
+    def set_mask(self, lengths: int, rows_per_segment: int) -> None:
+        """astitch_graph_set_mask: bind an existing LENGTHS input (created with
+        input("LENGTHS", "I32")) as the key-padding mask."""
+        check(lib.astitch_graph_set_mask(self._h, int(lengths), int(rows_per_segment)), "astitch_graph_set_mask")
+
     def segments(self, nseg: int, elems: int) -> int:
         """Packed varlen rows (astitch_graph_segments): adds the int32 [nseg, 4]
         segment-table input; FULL tensors then hold `elems` packed elements."""

@@ -246,6 +246,10 @@ struct Gen {
     return I(u).level;
   }
 
+  // byte offset of the lo parts of post-barrier COLVEC values (R7c)
+  long long colvals_lo() const {
+    return static_cast<long long>(p.ws.colvals + (p.post_colvecs.size() + p.colreds.size()) * C * 4);
+  }
   // COLVEC values finalised after earlier barriers (loaded from ws)
   void emit_post_colvec_loads() {
     for (size_t q = 0; q < p.post_colvecs.size(); ++q) {
@@ -256,6 +260,13 @@ struct Gen {
       o << "#pragma unroll\n  for (int j = 0; j < V; ++j)\n#pragma unroll\n  for (int e = 0; e < E; ++e) {\n";
       o << "    const long long col = " << col_expr("j", "e") << ";\n";
       o << "    cp" << i << "[j * E + e] = (col < C) ? as::ld_cg(cv + col) : 0.f;\n  }}\n";
+      if (pc(i)) {  // lo part (R7c)
+        o << "  float cp" << i << "lo[NE];\n";
+        o << "  { const float* cv = (const float*)((char*)p.ws + " << colvals_lo() << "LL) + " << q << "LL * C;\n";
+        o << "#pragma unroll\n  for (int j = 0; j < V; ++j)\n#pragma unroll\n  for (int e = 0; e < E; ++e) {\n";
+        o << "    const long long col = " << col_expr("j", "e") << ";\n";
+        o << "    cp" << i << "lo[j * E + e] = (col < C) ? as::ld_cg(cv + col) : 0.f;\n  }}\n";
+      }
     }
   }
 
@@ -532,6 +543,13 @@ struct Gen {
       std::string id = std::to_string(i);
       if (nd.type == NodeType::Reduce && nd.axis == ASTITCH_AXIS_COL) {
         bool mx = nd.sub == ASTITCH_RMAX;
+        if (pc(i)) {  // fp64 accumulation of a cancellation-prone column sum (R7c)
+          std::string okc = act;
+          if (check && !absorb) okc += " && " + col_expr("(k / E)", "(k % E)") + " < " + lim;
+          o << "#pragma unroll\n    for (int k = 0; k < NE; ++k) acc" << id << "[k] += (" << okc << ") ? (double)"
+            << ref(nd.a, "k", sfx) << " : 0.0;\n";
+          continue;
+        }
         if (!mx && (E % 2) == 0 && !(check && !absorb)) {
           // paired accumulation (FADD2); inactive rows contribute zeros
           o << "#pragma unroll\n    for (int k = 0; k < NE; k += 2) {\n";
@@ -832,6 +850,11 @@ struct Gen {
     if (row_div(i)) return "as::mul2(" + ref2(nd.a, sfx) + ", as::bc2(rq" + std::to_string(i) + sfx + "))";
     std::string a = ref2(nd.a, sfx), b = ref2(nd.b, sfx);
     auto lo = [&](int v) { return "as::bc2(s" + std::to_string(N(v).a) + sfx + "lo)"; };
+    auto clo = [&](int v) { return "as::f2{" + col_lo(v, "k") + ", " + col_lo(v, "k + 1") + "}"; };
+    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.b)) return "as::sub2(as::sub2(" + a + ", " + b + "), " + clo(nd.b) + ")";
+    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.a)) return "as::add2(as::sub2(" + a + ", " + b + "), " + clo(nd.a) + ")";
+    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.b)) return "as::add2(as::add2(" + a + ", " + b + "), " + clo(nd.b) + ")";
+    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.a)) return "as::add2(as::add2(" + a + ", " + b + "), " + clo(nd.a) + ")";
     if (nd.sub == ASTITCH_SUB && precise_bcast(nd.b)) return "as::sub2(as::sub2(" + a + ", " + b + "), " + lo(nd.b) + ")";
     if (nd.sub == ASTITCH_SUB && precise_bcast(nd.a)) return "as::add2(as::sub2(" + a + ", " + b + "), " + lo(nd.a) + ")";
     if (nd.sub == ASTITCH_ADD && precise_bcast(nd.b)) return "as::add2(as::add2(" + a + ", " + b + "), " + lo(nd.b) + ")";
@@ -888,8 +911,35 @@ struct Gen {
     const Node& nd = N(v);
     return nd.type == NodeType::Bcast && nd.axis == ASTITCH_AXIS_ROW && precise[nd.a];
   }
+  // ---- cancellation-prone column values (reading R7c): fp64 column sums,
+  // fp64 per-column chain, applied to FULL add/sub as an fp32 hi + lo pair.
+  // Unsharded stitched kernel only (the sharded / chunked roles combine fp32
+  // totals across launches and keep the plain fp32 path).
+  bool pc(int i) const { return role == ROLE_MAIN && I(i).precise_col; }
+  int nslots() const { return static_cast<int>(p.colreds.size()) + p.n_precise_colreds; }
+  int lo_slot(int q) const {  // partial slot of the lo part of precise column sum q
+    int k = static_cast<int>(p.colreds.size());
+    for (int j = 0; j < q; ++j)
+      if (I(p.colreds[j]).precise_col) ++k;
+    return k;
+  }
+  bool any_pc() const {
+    for (int id : p.colreds)
+      if (pc(id)) return true;
+    return false;
+  }
+  // FULL operand v = bcast_col(c) of a precise post-barrier column value
+  bool precise_bcast_col(int v) const {
+    const Node& nd = N(v);
+    return nd.type == NodeType::Bcast && nd.axis == ASTITCH_AXIS_COL && pc(nd.a) && I(nd.a).post;
+  }
+  std::string col_lo(int v, const std::string& k) const { return "cp" + std::to_string(N(v).a) + "lo[" + k + "]"; }
   std::string full_binop(const Node& nd, const std::string& sfx) const {
     std::string a = ref(nd.a, "k", sfx), b = ref(nd.b, "k", sfx);
+    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.b)) return "((" + a + " - " + b + ") - " + col_lo(nd.b, "k") + ")";
+    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.a)) return "((" + a + " - " + b + ") + " + col_lo(nd.a, "k") + ")";
+    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.b)) return "((" + a + " + " + b + ") + " + col_lo(nd.b, "k") + ")";
+    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.a)) return "((" + a + " + " + b + ") + " + col_lo(nd.a, "k") + ")";
     if (nd.sub == ASTITCH_SUB && precise_bcast(nd.b))
       return "((" + a + " - " + b + ") - " + b + "lo)";
     if (nd.sub == ASTITCH_SUB && precise_bcast(nd.a))
@@ -1220,6 +1270,10 @@ struct Gen {
     for (int id : p.colreds) {
       if (phase_of(id) != cur_level) continue;
       bool mx = N(id).sub == ASTITCH_RMAX;
+      if (pc(id)) {  // fp64 per-lane column sums (R7c)
+        o << "  double acc" << id << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) acc" << id << "[k] = 0.0;\n";
+        continue;
+      }
       o << "  float acc" << id << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) acc" << id
         << "[k] = " << (mx ? "-AS_INF" : "0.f") << ";\n";
     }
@@ -1229,8 +1283,11 @@ struct Gen {
   std::string part_idx = "blockIdx.x";
   bool dyn_colred = false;  // counter-ordered tiles in the level-0 sweep (m.dyn_colred_rows)
   // block partial of every column reduction -> ws partial row blockIdx.x
+  // (precise sums, R7c: the block's fp64 sum stored as fp32 hi in slot q and
+  // lo in slot lo_slot(q); hi + lo keeps ~48 bits)
   void emit_block_partials() {
     const int ncr = static_cast<int>(p.colreds.size());
+    const int NS = nslots();
     o << "  {\n    float* part = (float*)((char*)p.ws + " << p.ws.partials << "LL);\n";
     if (RPB == 1) {
       for (int q = 0; q < ncr; ++q) {
@@ -1238,7 +1295,14 @@ struct Gen {
         if (phase_of(id) != cur_level) continue;
         o << "#pragma unroll\n    for (int k = 0; k < NE; ++k) {\n      const long long col = "
           << col_expr("(k / E)", "(k % E)") << ";\n";
-        o << "      if (col < C) part[((long long)" << part_idx << " * " << ncr << " + " << q << ") * C + col] = acc" << id
+        if (pc(id)) {
+          o << "      const float h_ = (float)acc" << id << "[k];\n";
+          o << "      if (col < C) { part[((long long)" << part_idx << " * " << NS << " + " << q << ") * C + col] = h_;\n";
+          o << "        part[((long long)" << part_idx << " * " << NS << " + " << lo_slot(q) << ") * C + col] = (float)(acc"
+            << id << "[k] - (double)h_); }\n    }\n";
+          continue;
+        }
+        o << "      if (col < C) part[((long long)" << part_idx << " * " << NS << " + " << q << ") * C + col] = acc" << id
           << "[k];\n    }\n";
       }
     } else {
@@ -1249,13 +1313,26 @@ struct Gen {
         if (phase_of(id) != cur_level) continue;
         bool mx = N(id).sub == ASTITCH_RMAX;
         o << "    __syncthreads();\n";
+        if (pc(id)) {
+          o << "#pragma unroll\n    for (int k = 0; k < NE; ++k) {\n      const long long c_ = " << col_expr("(k / E)", "(k % E)")
+            << ";\n      const float h_ = (float)acc" << id << "[k];\n      cp_smem[team * CC + c_] = h_;\n"
+            << "      cp_smem[(RPB + team) * CC + c_] = (float)(acc" << id << "[k] - (double)h_);\n    }\n";
+          o << "    __syncthreads();\n";
+          o << "    for (long long col = threadIdx.x; col < C; col += blockDim.x) {\n";
+          o << "      double a_ = 0.0;\n";
+          o << "      for (int t = 0; t < RPB; ++t) a_ += (double)cp_smem[t * CC + col] + (double)cp_smem[(RPB + t) * CC + col];\n";
+          o << "      const float h_ = (float)a_;\n";
+          o << "      part[((long long)" << part_idx << " * " << NS << " + " << q << ") * C + col] = h_;\n";
+          o << "      part[((long long)" << part_idx << " * " << NS << " + " << lo_slot(q) << ") * C + col] = (float)(a_ - (double)h_);\n    }\n";
+          continue;
+        }
         o << "#pragma unroll\n    for (int k = 0; k < NE; ++k) cp_smem[team * CC + " << col_expr("(k / E)", "(k % E)")
           << "] = acc" << id << "[k];\n";
         o << "    __syncthreads();\n";
         o << "    for (long long col = threadIdx.x; col < C; col += blockDim.x) {\n";
         o << "      float a_ = cp_smem[col];\n";
         o << "      for (int t = 1; t < RPB; ++t) a_ = " << (mx ? "as::nmax(a_, cp_smem[t * CC + col])" : "a_ + cp_smem[t * CC + col]") << ";\n";
-        o << "      part[((long long)" << part_idx << " * " << ncr << " + " << q << ") * C + col] = a_;\n    }\n";
+        o << "      part[((long long)" << part_idx << " * " << NS << " + " << q << ") * C + col] = a_;\n    }\n";
       }
     }
     o << "  }\n";
@@ -1274,18 +1351,31 @@ struct Gen {
     if (dyn_colred) o << "    const int NPART = NT_;\n";
     o << "    const long long c1 = min(C, c0 + W);\n";
     o << "    __shared__ float fin_smem[" << m.threads << "];\n";
+    if (any_pc()) o << "    __shared__ double fin_smem_d[" << m.threads << "];\n";
     o << "    int P = 1; while (P * 2 * W <= blockDim.x && P * 2 <= 256) P *= 2;\n";
     o << "    for (long long cb = c0; cb < c1; cb += blockDim.x / P) {\n";
     o << "      const int wi = threadIdx.x / P, pi = threadIdx.x % P;\n";
     o << "      const long long col = cb + wi;\n";
     o << "      const bool own = (wi < (int)(blockDim.x / P)) && col < c1;\n";
+    const int NS = nslots();
     for (int q = 0; q < ncr; ++q) {
       int id = p.colreds[q];
       if (phase_of(id) != cur_level) continue;
       bool mx = N(id).sub == ASTITCH_RMAX;
       std::string ident = mx ? "-AS_INF" : "0.f";
+      if (pc(id)) {  // fp64 combine of the hi + lo partials (R7c)
+        o << "      double t" << id << "d = 0.0;\n";
+        o << "      if (own) for (int r = pi; r < " << (dyn_colred ? "NPART" : "G") << "; r += P) t" << id
+          << "d += (double)as::ld_cg(part + ((long long)r * " << NS << " + " << q << ") * C + col) + (double)as::ld_cg(part + ((long long)r * "
+          << NS << " + " << lo_slot(q) << ") * C + col);\n";
+        o << "      fin_smem_d[threadIdx.x] = t" << id << "d;\n      __syncthreads();\n";
+        o << "      for (int s = P / 2; s > 0; s /= 2) { if (pi < s) fin_smem_d[threadIdx.x] += fin_smem_d[threadIdx.x + s]; __syncthreads(); }\n";
+        o << "      t" << id << "d = fin_smem_d[threadIdx.x - pi];\n      __syncthreads();\n";
+        o << "      const float t" << id << " = (float)t" << id << "d; (void)t" << id << ";\n";
+        continue;
+      }
       o << "      float t" << id << " = " << ident << ";\n";
-      o << "      if (own) for (int r = pi; r < " << (dyn_colred ? "NPART" : "G") << "; r += P) { const float x_ = as::ld_cg(part + ((long long)r * " << ncr
+      o << "      if (own) for (int r = pi; r < " << (dyn_colred ? "NPART" : "G") << "; r += P) { const float x_ = as::ld_cg(part + ((long long)r * " << NS
         << " + " << q << ") * C + col); t" << id << " = " << (mx ? "as::nmax(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_") << "; }\n";
       o << "      fin_smem[threadIdx.x] = t" << id << ";\n      __syncthreads();\n";
       o << "      for (int s = P / 2; s > 0; s /= 2) { if (pi < s) fin_smem[threadIdx.x] = "
@@ -1327,7 +1417,9 @@ struct Gen {
     o << "    const float* colpart = (const float*)((const char*)p.ws + " << colpart << "LL);\n";
     o << "    const int G = gridDim.x;\n    const long long W = (C + G - 1) / G;\n";
     o << "    const long long c0 = (long long)blockIdx.x * W, c1 = min(C, c0 + W);\n";
-    o << "    const int par = (int)(p.gen & 1u);\n";
+    // every block read xgen before the grid barrier above: publish it
+    o << "    if (blockIdx.x == 0 && threadIdx.x == 0) *(volatile unsigned int*)(X + " << kXGen << ") = xgen;\n";
+    o << "    const int par = (int)(xgen & 1u);\n";
     o << "    for (int q = 0; q < XW; ++q) {\n";
     o << "      float* dst = (float*)(__ldcg((const unsigned long long*)X + q) + " << kXSlots
       << "ULL) + ((long long)(par * XW + XR) * NCR) * C;\n";
@@ -1338,8 +1430,8 @@ struct Gen {
     o << "    as::grid_barrier(bar);\n";
     o << "    if (blockIdx.x == 0 && threadIdx.x < XW)\n";
     o << "      as::st_release_sys((unsigned int*)(__ldcg((const unsigned long long*)X + threadIdx.x) + " << kXFlags
-      << "ULL) + XR, p.gen);\n";
-    o << "    if (threadIdx.x == 0) as::wait_flags((const unsigned int*)(X + " << kXFlags << "), XW, p.gen, (unsigned int*)(X + "
+      << "ULL) + XR, xgen);\n";
+    o << "    if (threadIdx.x == 0) as::wait_flags((const unsigned int*)(X + " << kXFlags << "), XW, xgen, (unsigned int*)(X + "
       << kXErr << "));\n";
     o << "    __syncthreads();\n";
     o << "    const float* slots = (const float*)(X + " << kXSlots << ") + (long long)par * XW * NCR * C;\n";
@@ -1375,6 +1467,17 @@ struct Gen {
       if (I(i).level >= 1 && I(i).level < lv) {
         o << "        const float x" << id << " = as::ld_cg((const float*)((const char*)p.ws + " << p.ws.colvals
           << "LL) + " << post_index(i) << "LL * C + col);\n";
+        if (pc(i))  // R7c: the fp64 value = hi + lo
+          o << "        const double x" << id << "d = (double)x" << id << " + (double)as::ld_cg((const float*)((const char*)p.ws + "
+            << colvals_lo() << "LL) + " << post_index(i) << "LL * C + col);\n";
+      } else if (pc(i)) {  // R7c: the per-column chain of a precise value in fp64
+        if (nd.type == NodeType::Reduce)
+          o << "        const double x" << id << "d = " << tpref << id << "d;\n";
+        else if (nd.type == NodeType::Unary)
+          o << "        const double x" << id << "d = " << (nd.sub == ASTITCH_NEG ? "-" : "fabs") << "(" << xdref(nd.a) << ");\n";
+        else
+          o << "        const double x" << id << "d = " << xdbinop(nd.sub, nd.a, nd.b) << ";\n";
+        o << "        const float x" << id << " = (float)x" << id << "d;\n";
       } else if (nd.type == NodeType::Reduce) {
         o << "        const float x" << id << " = " << tpref << id << ";\n";
       } else if (nd.type == NodeType::Input) {
@@ -1393,9 +1496,54 @@ struct Gen {
     }
     for (size_t q = 0; q < p.post_colvecs.size(); ++q) {
       int id = p.post_colvecs[q];
-      if (I(id).level != lv) continue;
+      if (I(id).level != lv || !read_later(id)) continue;
       o << "        ((float*)((char*)p.ws + " << p.ws.colvals << "LL))[" << q << "LL * C + col] = x" << id << ";\n";
+      if (pc(id))
+        o << "        ((float*)((char*)p.ws + " << colvals_lo() << "LL))[" << q << "LL * C + col] = (float)(x" << id
+          << "d - (double)x" << id << ");\n";
     }
+  }
+  // is post-barrier COLVEC value id read by a later sweep or a later level's
+  // column chain?  (only then is it published to the workspace)
+  bool read_later(int id) const {
+    const int lv = I(id).level;
+    for (int u : I(id).consumers) {
+      if (!I(u).live) continue;
+      const Node& un = N(u);
+      if (un.type == NodeType::Bcast) {
+        for (int w : I(u).consumers)
+          if (I(w).live && phase_of(w) >= lv) return true;
+        continue;
+      }
+      if (un.kind == ASTITCH_COLVEC) {
+        if (I(u).level > lv) return true;       // a later level's column chain reads it back
+        if (read_later(u)) return true;         // same level: computed from it, recursively
+        continue;
+      }
+      if (phase_of(u) >= lv) return true;       // FULL / ROWVEC consumer in a later sweep
+    }
+    return false;
+  }
+  std::string xdref(int i) const {
+    if (N(i).type == NodeType::Const) {
+      char buf[64];
+      snprintf(buf, sizeof(buf), "%a", N(i).cval);
+      return std::string("(") + buf + ")";
+    }
+    if (pc(i)) return "x" + std::to_string(i) + "d";
+    return "(double)x" + std::to_string(i);
+  }
+  std::string xdbinop(int op, int a, int b) const {
+    std::string x = xdref(a), y = xdref(b);
+    switch (op) {
+      case ASTITCH_ADD: return "(" + x + " + " + y + ")";
+      case ASTITCH_SUB: return "(" + x + " - " + y + ")";
+      case ASTITCH_MUL: return "(" + x + " * " + y + ")";
+      case ASTITCH_DIV: return "(" + x + " / " + y + ")";
+      case ASTITCH_MAX: return "as::dmaxn(" + x + ", " + y + ")";
+      case ASTITCH_MIN: return "as::dminn(" + x + ", " + y + ")";
+    }
+    return x;
   }
   std::string xref(int i) const {
     if (N(i).type == NodeType::Const) return "k" + std::to_string(i);
@@ -1878,9 +2026,15 @@ struct Gen {
       o << "  unsigned int* bar = (unsigned int*)((char*)p.ws + " << p.ws.barrier << "LL);\n  (void)bar;\n";
       if (dyn_colred) o << "  const int R_all_ = R;\n";
     }
-    if (role == ROLE_FUSED)  // this run's wait status (set only after the grid barriers below)
+    if (role == ROLE_FUSED) {
+      // this run's generation: read by every block BEFORE the first grid
+      // barrier, bumped in the buffer by block 0 after it (emit_fused_exchange),
+      // so eager runs and CUDA-graph replays alike get a fresh generation; and
+      // this run's wait status (set only after the grid barriers below)
+      o << "  const unsigned int xgen = *(volatile unsigned int*)((unsigned char*)p.xbuf + " << kXGen << ") + 1u;\n";
       o << "  if (blockIdx.x == 0 && threadIdx.x == 0) *(volatile unsigned int*)((unsigned char*)p.xbuf + " << kXErr
         << ") = 0u;\n";
+    }
     if (role == ROLE_SHARD_SWEEP2) {  // sharded plans have one barrier level
       cur_level = 1;
       emit_colvecs(false);
@@ -1901,16 +2055,27 @@ struct Gen {
     // level 1 -> barrier -> sweep level 1 -> ...]: one grid barrier pair per
     // level of dependent column reductions
     const int D = p.max_level;
+    auto colred_at = [&](int lv) {
+      for (int id : p.colreds)
+        if (phase_of(id) == lv) return true;
+      return false;
+    };
+    auto sweep_at = [&](int lv) {
+      if (lv == 0) return true;
+      for (size_t i = 0; i < g.nodes.size(); ++i)
+        if (I(i).live && I(i).level == lv && (N(i).kind == ASTITCH_FULL || N(i).kind == ASTITCH_ROWVEC)) return true;
+      return false;
+    };
+    // a grid barrier after a level's column finalise only when a later level
+    // reads what it published (a last level ends the kernel with no barrier)
+    auto later_work = [&](int lv) {
+      for (int l = lv + 1; l <= D; ++l)
+        if (sweep_at(l) || colred_at(l)) return true;
+      return false;
+    };
     for (int lv = 0; lv <= D; ++lv) {
       cur_level = lv;
-      bool colred_here = false, sweep_here = (lv == 0);
-      for (int id : p.colreds)
-        if (phase_of(id) == lv) colred_here = true;
-      for (size_t i = 0; i < g.nodes.size(); ++i) {
-        const Node& nd = N(i);
-        if (!I(i).live || I(i).level != lv || lv == 0) continue;
-        if (nd.kind == ASTITCH_FULL || nd.kind == ASTITCH_ROWVEC) sweep_here = true;
-      }
+      const bool colred_here = colred_at(lv), sweep_here = sweep_at(lv);
       if (!sweep_here && !colred_here) continue;
       o << "  {  // ---- level " << lv << "\n";
       if (lv > 0) emit_post_colvec_loads();
@@ -1939,7 +2104,7 @@ struct Gen {
         o << "  as::grid_barrier(bar);\n";
         o << "  if (blockIdx.x == 0 && threadIdx.x == 0) tctr_[0] = 0u;  // every CTA is past its last grab\n";
         emit_column_finalize(true);
-        if (lv < D) o << "  as::grid_barrier(bar);\n";
+        if (later_work(lv)) o << "  as::grid_barrier(bar);\n";
         o << "  }\n";
         continue;
       }
@@ -1953,12 +2118,12 @@ struct Gen {
         } else if (role == ROLE_FUSED) {
           emit_column_finalize(false);
           emit_fused_exchange();
-          if (lv < D) o << "  as::grid_barrier(bar);\n";
+          if (later_work(lv)) o << "  as::grid_barrier(bar);\n";
         } else {
           emit_column_finalize(true);
-          if (lv < D) o << "  as::grid_barrier(bar);\n";
+          if (later_work(lv)) o << "  as::grid_barrier(bar);\n";
         }
-      } else if (lv < D) {
+      } else if (later_work(lv)) {
         // FORCE_GLOBAL: row-reduction results of this level are in HBM
         o << "  as::grid_barrier(bar);\n";
       }

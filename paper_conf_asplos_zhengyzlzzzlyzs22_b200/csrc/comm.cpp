@@ -83,7 +83,6 @@ struct astitch_peer_s {
   std::vector<void*> ptrs;                // every rank's buffer as addressed from this process
   std::vector<bool> opened;               // ptrs[q] came from cuIpcOpenMemHandle (close on destroy)
   bool table_dirty = true;
-  unsigned int gen = 0;
 };
 
 namespace astitch {
@@ -296,8 +295,6 @@ astitch_status astitch_run_fused(astitch_plan_t h, astitch_peer_t x, const void*
   }
   KernelParams kp = make_params(p, inputs, outputs, ws);
   kp.xbuf = x->local;
-  kp.gen = ++x->gen;
-  if (kp.gen == 0) kp.gen = ++x->gen;  // 0 is the initial flag value
   return launch(p, p.fused_kernels[0], kp, stream);
 }
 

@@ -174,7 +174,7 @@ bool drv_load(Plan& p, Kernel& k, std::string& err) {
   CUfunction fn;
   r = d->ModuleGetFunction(&fn, mod, k.name.c_str());
   if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuModuleGetFunction"); d->ModuleUnload(mod); return false; }
-  if (k.smem > 48 * 1024) {
+  if (k.smem > 0) {  // dynamic + static may exceed the 48 KB default even when dynamic alone does not
     r = d->FuncSetAttribute(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, k.smem);
     if (r != CUDA_SUCCESS) { err = cu_err(d, r, "cuFuncSetAttribute(smem)"); d->ModuleUnload(mod); return false; }
   }

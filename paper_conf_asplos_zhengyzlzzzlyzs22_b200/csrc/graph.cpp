@@ -121,10 +121,11 @@ astitch_status astitch_graph_destroy(astitch_graph_t g) {
 astitch_status astitch_graph_input(astitch_graph_t g, astitch_kind kind, astitch_dtype dtype,
                                    astitch_value_t* out) {
   if (!g || !out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL graph or out");
-  if (kind != ASTITCH_FULL && kind != ASTITCH_ROWVEC && kind != ASTITCH_COLVEC)
-    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "input kind must be FULL, ROWVEC or COLVEC");
-  if (dtype != ASTITCH_F32 && dtype != ASTITCH_BF16 && dtype != ASTITCH_F16)
-    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "input dtype must be F32, BF16 or F16");
+  if (kind != ASTITCH_FULL && kind != ASTITCH_ROWVEC && kind != ASTITCH_COLVEC && kind != ASTITCH_LENGTHS)
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "input kind must be FULL, ROWVEC, COLVEC or LENGTHS");
+  if (kind == ASTITCH_LENGTHS ? dtype != ASTITCH_I32
+                              : (dtype != ASTITCH_F32 && dtype != ASTITCH_BF16 && dtype != ASTITCH_F16))
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "input dtype must be F32, BF16 or F16 (I32 for LENGTHS)");
   if (g->g.inputs.size() >= static_cast<size_t>(kMaxIO))
     return fail(ASTITCH_ERR_UNSUPPORTED, "too many inputs (max 16)");
   Node n;
@@ -157,6 +158,21 @@ astitch_status astitch_graph_lengths(astitch_graph_t g, int64_t rows_per_segment
     g->g.rows_per_segment = rows_per_segment;
   }
   return s;
+}
+
+astitch_status astitch_graph_set_mask(astitch_graph_t g, astitch_value_t lengths, int64_t rows_per_segment) {
+  if (!g) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL graph");
+  if (rows_per_segment < 1) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "rows_per_segment < 1");
+  if (lengths < 0 || lengths >= static_cast<astitch_value_t>(g->g.nodes.size()))
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad value");
+  const Node& n = g->g.nodes[lengths];
+  if (n.type != NodeType::Input || n.kind != ASTITCH_LENGTHS)
+    return fail(ASTITCH_ERR_INVALID_GRAPH, "the mask must be a LENGTHS input (astitch_graph_input)");
+  if (g->g.lengths_node >= 0 || g->g.segments_node >= 0)
+    return fail(ASTITCH_ERR_INVALID_GRAPH, "graph already has a mask or segments");
+  g->g.lengths_node = lengths;
+  g->g.rows_per_segment = rows_per_segment;
+  return ASTITCH_OK;
 }
 
 astitch_status astitch_graph_segments(astitch_graph_t g, int32_t nseg, int64_t elems,

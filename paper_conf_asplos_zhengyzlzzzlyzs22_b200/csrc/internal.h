@@ -78,6 +78,7 @@ struct NodeInfo {
   int group = -1;              // op group id
   Scheme scheme = Scheme::Local;
   bool global_full = false;    // FULL value buffered in HBM across the barrier
+  bool precise_col = false;    // cancellation-prone column value: fp64 sum, applied as hi+lo (R7c)
   std::vector<int> consumers;
 };
 
@@ -173,11 +174,14 @@ struct Plan {
   astitch_plan_desc desc{};
   Tuning tune;
   int sm_count = 148;
+  int smem_optin = 232448;       // max dynamic+static smem per block (B200: 227 KB; device query)
+  std::vector<std::string> demotions;  // resource-driven mapping changes (a6), in order (describe())
   std::vector<NodeInfo> info;
   std::vector<std::vector<int>> groups;
   Mapping map;
   std::vector<int> colreds;      // column reduce node ids (in order)
   std::vector<int> post_colvecs; // COLVEC values computed after the barrier (incl. colreds)
+  int n_precise_colreds = 0;     // column sums with an extra lo partial slot (reading R7c)
   std::vector<int> global_fulls; // FULL / ROWVEC values buffered in HBM across a barrier
   std::vector<size_t> gbuf_off;  // byte offset of each one's buffer within ws.globals (a6 reuse)
   int gbuf_slots = 0;            // distinct buffers after liveness-based reuse
@@ -218,6 +222,7 @@ enum KernelRole { ROLE_MAIN = 0, ROLE_SHARD_MAIN = 1, ROLE_SHARD_FINAL = 2, ROLE
 // kXSlots: 2 (generation parity) x world x ncolred x cols fp32 slots.
 constexpr size_t kXFlags = 8 * 64;           // up to 64 ranks
 constexpr size_t kXErr = kXFlags + 4 * 64;
+constexpr size_t kXGen = kXErr + 4;          // u32: generation of the last fused run (bumped in-kernel)
 constexpr size_t kXSlots = 1024;
 inline size_t xbuf_bytes(int world, size_t ncolred, int64_t cols) {
   return kXSlots + 2 * static_cast<size_t>(world) * ncolred * static_cast<size_t>(cols) * 4;
@@ -264,7 +269,7 @@ struct KernelParams {
   long long row_offset;   // global row index of row 0 (chunked runs; mask segments)
   int flags;              // bit 0: accumulate column totals onto earlier chunks
   void* xbuf;             // fused sharded run: this rank's peer exchange buffer
-  unsigned int gen;       // fused sharded run: generation of this run (flags)
+  unsigned int gen;       // unused (the fused run's generation lives in the exchange buffer)
 };
 
 }  // namespace astitch

@@ -515,7 +515,9 @@ __device__ __forceinline__ void wait_flags(const unsigned int* flags, int world,
                                            unsigned int* err) {
   const unsigned long long t0 = globaltimer_ns();
   for (int q = 0; q < world; ++q) {
-    while (ld_acquire_sys(flags + q) != gen) {
+    // wrap-safe "published at or past this generation": a fast peer may
+    // already have moved on to gen + 1 (never to gen + 2: that needs our flag)
+    while (static_cast<int>(ld_acquire_sys(flags + q) - gen) < 0) {
       if (globaltimer_ns() - t0 > 5000000000ULL) { atomicOr(err, 1u); return; }
       __nanosleep(200);
     }

@@ -286,6 +286,41 @@ void analyse(Plan& p) {
     if (info[i].post && (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC))
       p.needs_sweep2 = true;
   }
+
+  // Reading R7c (the column analogue of R7b): a column SUM whose value, through
+  // light per-column ops, is broadcast into a FULL add / sub (a column mean
+  // that is subtracted: BatchNorm) must keep the column's spread.  It is
+  // accumulated in fp64 (per lane, per block, per column), its per-column
+  // chain is evaluated in fp64, and the value is applied as an fp32 hi + lo pair.
+  std::vector<bool> need(n, false);
+  for (int b = 0; b < n; ++b) {
+    const Node& bn = g.nodes[b];
+    if (!info[b].live || bn.type != NodeType::Bcast || bn.axis != ASTITCH_AXIS_COL) continue;
+    for (int u : info[b].consumers) {
+      const Node& un = g.nodes[u];
+      if (info[u].live && un.type == NodeType::Binary && un.kind == ASTITCH_FULL &&
+          (un.sub == ASTITCH_ADD || un.sub == ASTITCH_SUB))
+        need[bn.a] = true;
+    }
+  }
+  p.n_precise_colreds = 0;
+  for (int i = n - 1; i >= 0; --i) {
+    if (!need[i] || !info[i].post) continue;
+    const Node& nd = g.nodes[i];
+    if (nd.kind != ASTITCH_COLVEC) continue;
+    if (nd.type == NodeType::Reduce && nd.sub == ASTITCH_SUM && nd.axis == ASTITCH_AXIS_COL) {
+      info[i].precise_col = true;
+      continue;
+    }
+    const bool light = (nd.type == NodeType::Binary && nd.sub != ASTITCH_POW) ||
+                       (nd.type == NodeType::Unary && (nd.sub == ASTITCH_NEG || nd.sub == ASTITCH_ABS));
+    if (!light) continue;
+    info[i].precise_col = true;
+    for (int a : {nd.a, nd.b})
+      if (a >= 0 && g.nodes[a].kind == ASTITCH_COLVEC && info[a].post) need[a] = true;
+  }
+  for (int id : p.colreds)
+    if (info[id].precise_col) ++p.n_precise_colreds;
 }
 
 // ------------------------------------------------------------------------ a3/a4/a6/a7
@@ -312,6 +347,7 @@ int lds128_conflict_ways(int stride) {
 void select_mapping(Plan& p) {
   const Graph& g = p.g;
   Mapping m;
+  p.demotions.clear();
   const int64_t R = p.desc.rows, C = p.desc.cols;
   const int sms = p.sm_count;
   std::ostringstream why;
@@ -422,9 +458,24 @@ void select_mapping(Plan& p) {
     m.row_unroll = std::max(1, std::min(4, 64 / std::max(1, ne * nfull_in)));
     if (tu.unroll >= 1 && tu.unroll <= 8) m.row_unroll = tu.unroll;
     // a6: block-level combine of the teams' column partials in smem
+    // (rows_per_block teams x the team's columns, fp32; hi + lo for precise
+    // sums).  Over the budget: fewer teams per block (demotion), down to one
+    // team per block, whose partials go straight to the workspace (no smem).
     if (m.rows_per_block > 1 && has_colred) {
-      int64_t cb = static_cast<int64_t>(m.rows_per_block) * m.team * m.chunks_per_lane * E * 4;
-      if (cb <= 96 * 1024) m.smem_bytes = static_cast<int>(cb);
+      auto cbytes = [&]() {
+        int64_t cb = static_cast<int64_t>(m.rows_per_block) * m.team * m.chunks_per_lane * E * 4;
+        return p.n_precise_colreds > 0 ? 2 * cb : cb;  // hi and lo parts of fp64 column partials (R7c)
+      };
+      const int64_t budget = std::min<int64_t>(96 * 1024, p.smem_optin - 16 * 1024);
+      const int rpb0 = m.rows_per_block;
+      while (m.rows_per_block > 1 && (m.rows_per_block / 2) * m.team >= 32 && cbytes() > budget) {
+        m.rows_per_block /= 2;
+        m.threads = m.rows_per_block * m.team;
+      }
+      if (m.rows_per_block != rpb0)
+        p.demotions.push_back("global sweep block combine: " + std::to_string(rpb0) + " -> " +
+                              std::to_string(m.rows_per_block) + " teams per block (smem)");
+      if (m.rows_per_block > 1) m.smem_bytes = static_cast<int>(cbytes());
     }
     why << (has_colred ? "column reduce -> global sweep (vertical packing, grid barrier); "
                        : "FORCE_GLOBAL: row reductions demoted to global (HBM + grid barrier); ");
@@ -475,25 +526,17 @@ void select_mapping(Plan& p) {
     const bool force_split = (p.desc.flags & ASTITCH_FLAG_FORCE_SPLIT) != 0;
     bool split_rule = !no_split && !ragged && R < blocks_per_wave_1024 && C > 1024 &&
                       (force_split || C * es_max >= 256 * 1024);
-    if (packed_ok) {
-      m.tmpl = Template::PackedTile;
-      m.team = 1;
-      m.chunks_per_lane = chunks;
-      m.lane_util = 1.0;
-      m.threads = 128;
-      m.tile_rows = 128;
-      m.stages = 4;  // prefetch distance 2 tiles + 2 tiles draining (bulk stores)
-      if (tu.tile_stages >= 3 && tu.tile_stages <= 8) m.stages = tu.tile_stages;
-      if (tu.tile_threads >= 32 && tu.tile_threads <= 1024 && tu.tile_threads % 32 == 0) m.threads = tu.tile_threads;
-      if (tu.tile_rows >= 1 && tu.tile_rows % m.threads == 0) m.tile_rows = tu.tile_rows;
-      m.rows_per_block = m.threads / m.team;
-      // stage bytes: input tiles + output tiles that cannot be written in
-      // place over an input tile of the same element size (mirrors codegen)
-      int in_bytes = 0, out_bytes = 0;
+    // packed-tile stage bytes per row: input tiles + output tiles that cannot
+    // be written in place over an input tile of the same element size
+    // (mirrors codegen)
+    int64_t pk_in_bytes = 0, pk_out_bytes = 0;
+    {
+      int64_t& in_bytes = pk_in_bytes;
+      int64_t& out_bytes = pk_out_bytes;
       std::vector<int> in_sizes;
       for (int id : g.inputs)
         if (g.nodes[id].kind == ASTITCH_FULL && p.info[id].live) {
-          in_bytes += static_cast<int>(C) * dtype_size(g.nodes[id].dtype);
+          in_bytes += C * dtype_size(g.nodes[id].dtype);
           in_sizes.push_back(dtype_size(g.nodes[id].dtype));
         }
       for (size_t k = 0; k < g.outputs.size(); ++k)
@@ -501,13 +544,51 @@ void select_mapping(Plan& p) {
           int es = dtype_size(g.output_dtypes[k]);
           auto it = std::find(in_sizes.begin(), in_sizes.end(), es);
           if (it != in_sizes.end()) in_sizes.erase(it);
-          else out_bytes += static_cast<int>(C) * es;
+          else out_bytes += C * es;
         }
-      m.smem_bytes = m.stages * m.tile_rows * (in_bytes + out_bytes) + 64 * m.stages;
-      while (m.smem_bytes > 200 * 1024 && m.stages > 2) {
-        m.stages--;
-        m.smem_bytes = m.stages * m.tile_rows * (in_bytes + out_bytes) + 64 * m.stages;
+    }
+    // a6 shared-memory plan with demotion ("demote ... one by one
+    // until the memory usage is under the limit"): the staged tile ring of
+    // S stages x TR rows must fit HALF the SM's shared memory (>= 2 blocks per
+    // SM, so the producer warp of one block overlaps the other's compute).
+    // Demote in order of cost: 3 stages (prefetch distance 1), 64-row tiles;
+    // if it still does not fit, the staged tile is abandoned for a register
+    // row team (no smem staging at all) -- one warp of 32-row tiles per SM
+    // would starve HBM.
+    int pk_stages = 4, pk_threads = 128;  // prefetch distance 2 tiles + 2 tiles draining (bulk stores)
+    if (tu.tile_stages >= 2 && tu.tile_stages <= 8) pk_stages = tu.tile_stages;
+    if (tu.tile_threads >= 32 && tu.tile_threads <= 1024 && tu.tile_threads % 32 == 0) pk_threads = tu.tile_threads;
+    int pk_rows = (tu.tile_rows >= 1 && tu.tile_rows % pk_threads == 0) ? tu.tile_rows : pk_threads;
+    const int64_t smem_budget = std::min<int64_t>(100 * 1024, p.smem_optin / 2 - 4096);
+    auto pk_smem = [&]() {
+      return static_cast<int64_t>(pk_stages) * pk_rows * (pk_in_bytes + pk_out_bytes) + 64 * pk_stages;
+    };
+    if (packed_ok) {
+      while (pk_smem() > smem_budget) {
+        if (pk_stages > 3) --pk_stages;
+        else if (pk_threads > 64) { pk_threads /= 2; pk_rows = pk_threads; }
+        else break;
       }
+      if (pk_smem() > smem_budget) {
+        packed_ok = false;
+        p.demotions.push_back("packed_tile needs " + std::to_string(pk_smem()) + " B of smem at " +
+                              std::to_string(pk_stages) + " stages x " + std::to_string(pk_rows) + " rows > " +
+                              std::to_string(smem_budget) + " -> row team (no staging)");
+      } else if (pk_stages != 4 || pk_threads != 128) {
+        p.demotions.push_back("packed_tile smem: " + std::to_string(pk_stages) + " stages x " + std::to_string(pk_rows) +
+                              " rows (" + std::to_string(pk_smem()) + " B <= " + std::to_string(smem_budget) + ")");
+      }
+    }
+    if (packed_ok) {
+      m.tmpl = Template::PackedTile;
+      m.team = 1;
+      m.chunks_per_lane = chunks;
+      m.lane_util = 1.0;
+      m.threads = pk_threads;
+      m.tile_rows = pk_rows;
+      m.stages = pk_stages;
+      m.rows_per_block = m.threads / m.team;
+      m.smem_bytes = static_cast<int>(pk_smem());
       m.bank_conflict_ways = lds128_conflict_ways(static_cast<int>(C) * es_min);
       why << "row of " << chunks << " x " << (E * es_min)
           << "B chunks does not tile a power-of-two team -> TMA-staged packed tiles, thread per row; ";
@@ -710,9 +791,13 @@ void plan_workspace(Plan& p) {
     w.partials = off;
     const int64_t nparts = p.map.dyn_colred_rows > 0 ? (R + p.map.dyn_colred_rows - 1) / p.map.dyn_colred_rows
                                                      : p.map.grid;
-    off = align(off + static_cast<size_t>(nparts) * p.colreds.size() * C * 4);
+    // partial slots: one per column reduction + a lo slot per precise sum (R7c)
+    const size_t nslots = p.colreds.size() + static_cast<size_t>(p.n_precise_colreds);
+    off = align(off + static_cast<size_t>(nparts) * nslots * C * 4);
     w.colvals = off;
-    off = align(off + std::max<size_t>(p.post_colvecs.size(), 1) * C * 4 + C * 4 * p.colreds.size());
+    // [post COLVEC hi][rank-local column totals][post COLVEC lo (R7c)]
+    off = align(off + std::max<size_t>(p.post_colvecs.size(), 1) * C * 4 + C * 4 * p.colreds.size() +
+                (p.n_precise_colreds ? p.post_colvecs.size() * C * 4 : 0));
     w.globals = off;
     // a6 memory reuse: a global buffer is live from the sweep that
     // writes it to the last sweep that reads it; a later value of the same
@@ -851,6 +936,9 @@ std::string describe_json(const Plan& p) {
   o << ",\"global_fulls\":[";
   for (size_t k = 0; k < p.global_fulls.size(); ++k) o << (k ? "," : "") << p.global_fulls[k];
   o << "],\"global_buffers\":" << p.gbuf_slots;
+  o << ",\"demotions\":[";
+  for (size_t k = 0; k < p.demotions.size(); ++k) o << (k ? "," : "") << "\"" << esc(p.demotions[k]) << "\"";
+  o << "]";
   o << ",\"needs_sweep2\":" << (p.needs_sweep2 ? "true" : "false");
   if (g.segments_node >= 0)
     o << ",\"ragged\":{\"nseg\":" << g.nseg << ",\"elems\":" << g.seg_elems << "}";

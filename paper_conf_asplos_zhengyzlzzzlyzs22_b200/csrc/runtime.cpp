@@ -229,6 +229,9 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
   if (desc->shard_world < 0 || (desc->shard_world > 0 && (desc->shard_rank < 0 || desc->shard_rank >= desc->shard_world)))
     return fail(ASTITCH_ERR_INVALID_ARGUMENT, "bad shard_rank / shard_world");
   if (gr->g.outputs.empty()) return fail(ASTITCH_ERR_INVALID_GRAPH, "graph has no outputs");
+  for (int id : gr->g.inputs)
+    if (gr->g.nodes[id].kind == ASTITCH_LENGTHS && id != gr->g.lengths_node)
+      return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS input not bound by astitch_graph_set_mask");
   try {
     auto plan = std::make_unique<Plan>();
     Plan& p = *plan;
@@ -246,6 +249,7 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
       int sms = 0, smem_optin = 0;
       if (!drv_device_info(p.device, sms, smem_optin, err)) return fail(ASTITCH_ERR_CUDA, err);
       if (desc->sm_count <= 0) p.sm_count = sms;
+      if (smem_optin > 0) p.smem_optin = smem_optin;
     }
     analyse(p);
     if (p.desc.shard_world > 1 && (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL))
@@ -280,7 +284,16 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
           int64_t max_grid = static_cast<int64_t>(k.occupancy) * p.sm_count;
           if (max_grid < 1)
             return fail(ASTITCH_ERR_RESOURCE, "kernel " + k.name + " cannot be resident (occupancy 0)");
-          if (k.grid > max_grid) k.grid = max_grid;
+          if (k.grid > max_grid) {
+            // the planned one-wave grid is not co-resident (the register /
+            // smem estimate was optimistic): STRICT refuses, otherwise the
+            // persistent grid shrinks to what is resident (still one kernel)
+            if (p.desc.flags & ASTITCH_FLAG_STRICT_SINGLE_KERNEL)
+              return fail(ASTITCH_ERR_RESOURCE, "kernel " + k.name + ": planned grid " + std::to_string(k.grid) +
+                                                    " > resident " + std::to_string(max_grid) + " (STRICT_SINGLE_KERNEL)");
+            p.demotions.push_back("grid " + std::to_string(k.grid) + " -> " + std::to_string(max_grid) + " (residency)");
+            k.grid = max_grid;
+          }
         }
         return ASTITCH_OK;
       };

@@ -151,3 +151,61 @@ def test_binding_checks_tensors_against_the_plan():
         p.check_io(ins[:2], outs, device=False)
     with pytest.raises(ValueError, match="CUDA"):
         p.check_io(ins, outs)
+
+
+def test_set_mask_binds_an_existing_lengths_input():
+    """SURVEY 8(b)'s two-step mask: astitch_graph_input(LENGTHS, I32) then
+    astitch_graph_set_mask; an unbound LENGTHS input is rejected at plan time."""
+    def graph(bind):
+        g = A.Graph()
+        x = g.input("FULL", "BF16")
+        L = g.input("LENGTHS", "I32")
+        if bind:
+            g.set_mask(L, 8)
+        m = g.reduce("RMAX", "ROW", x)
+        g.output(g.binary("SUB", x, g.broadcast("ROW", m)), "BF16")
+        return g, L
+    g, L = graph(True)
+    p = A.Plan(g, 64, 128, device=-1, flags=A.FLAG_NO_COMPILE)
+    assert p.inputs == [("FULL", "BF16"), ("LENGTHS", "I32")]
+    with pytest.raises(A.AstitchError) as e:
+        g.set_mask(L, 8)                                   # already has a mask
+    assert e.value.status == 2
+    g2, _ = graph(False)
+    with pytest.raises(A.AstitchError) as e:
+        A.Plan(g2, 64, 128, device=-1, flags=A.FLAG_NO_COMPILE)
+    assert e.value.status == 2 and "set_mask" in _lib.lib.astitch_last_error().decode()
+    g3 = A.Graph()
+    x = g3.input("FULL", "F32")
+    with pytest.raises(A.AstitchError) as e:
+        g3.set_mask(x, 8)                                  # not a LENGTHS input
+    assert e.value.status == 2
+    with pytest.raises(A.AstitchError):
+        g3.input("LENGTHS", "F32")                         # LENGTHS are int32
+
+
+def test_tuning_string_overrides_and_errors():
+    """astitch_plan_ex: explicit planner overrides (the library reads no
+    environment variables); unknown keys / non-integers are argument errors."""
+    spec = specs.get("C2", rows=4096)
+    base = A.Plan(A.Graph.from_spec(spec), 4096, 768, device=-1, flags=A.FLAG_NO_COMPILE).describe()
+    t = A.Plan(A.Graph.from_spec(spec), 4096, 768, device=-1, flags=A.FLAG_NO_COMPILE,
+               tune={"threads": 256, "unroll": 2}).describe()
+    assert base["tuning"] == "" and t["tuning"] == "threads=256,unroll=2"
+    assert t["mapping"]["threads"] == 256 and t["mapping"]["row_unroll"] == 2
+    assert base["mapping"]["threads"] != 256 or base["mapping"]["row_unroll"] != 2
+    for bad in ("nope=1", "threads=abc", "threads"):
+        with pytest.raises(A.AstitchError) as e:
+            A.Plan(A.Graph.from_spec(spec), 4096, 768, device=-1, flags=A.FLAG_NO_COMPILE, tune=bad)
+        assert e.value.status == 1
+    s = A.Plan(A.Graph.from_spec(specs.get("C1", rows=4, cols=512)), 4, 512, device=-1,
+               flags=A.FLAG_NO_COMPILE, tune="stream=1").describe()
+    assert s["mapping"]["template"] == "row_stream"
+
+
+def test_library_reads_no_planning_environment_variables():
+    """A plan is a pure function of (graph, desc, tuning): no getenv in the
+    planner or code generator (only the dlopen paths of libnccl / libnvrtc)."""
+    src = os.path.join(ROOT, "paper_conf_asplos_zhengyzlzzzlyzs22_b200", "csrc")
+    for f in ("planner.cpp", "codegen.cpp", "runtime.cpp", "graph.cpp"):
+        assert "getenv" not in open(os.path.join(src, f)).read(), f

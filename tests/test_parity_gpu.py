@@ -507,13 +507,205 @@ def test_parity_random_shapes(seed):
         _compare(spec, got, evaluate(spec, x))
 
 
-@pytest.mark.xfail(strict=False, reason="cancellation-prone column means are plain fp32 column sums "
-                                        "(column analogue of reading R7b: DESIGN.md NEXT)")
 def test_parity_batchnorm_two_rows_column_mean_cancellation():
-    """Known limitation found by scripts/fuzz_shapes.py (seed 244): BatchNorm
-    over 2 rows x 4513 fp32 columns; columns with |x1 - x2| << |x| lose
-    ~5e-5 relative accuracy in x - mean."""
+    """Found by scripts/fuzz_shapes.py in round 1 (seed 244): BatchNorm over
+    2 rows x 4513 fp32 columns, where columns with |x1 - x2| << |x| lose
+    ~5e-5 relative accuracy in x - mean unless the subtracted column mean
+    keeps the column's spread (reading R7c: fp64 column sums, hi + lo)."""
     spec = specs.get("bn", rows=2, cols=4513)
     x = gen.generate("bn", spec)
     got = run_gpu(spec, x)
     _compare(spec, got, evaluate(spec, x))
+
+
+@pytest.mark.parametrize("rows,cols", [(2, 4513), (3, 1000), (777, 64), (20000, 96), (5, 4096)])
+@pytest.mark.parametrize("mean", [0.0, 1000.0, -3.0e4])
+def test_parity_batchnorm_column_mean_far_from_spread(rows, cols, mean):
+    """Column means far from the spread (|mean| up to 3e6 x the spread),
+    fp32 I/O at the 1e-5 rule (reading R7c)."""
+    spec = specs.get("bn", rows=rows, cols=cols)
+    x = gen.generate("bn", spec)
+    x["x"] = (mean + 0.01 * x["x"].astype(np.float64)).astype(np.float32)
+    _compare(spec, run_gpu(spec, x), evaluate(spec, x))
+
+
+# Reading R12: RMAX (row and column) and binary MAX / MIN propagate NaN, as
+# the oracle's numpy max / maximum do (the kernels use max.NaN.f32).
+NAN_ROW = {
+    "name": "nan_row", "rows": 300, "cols": 256,
+    "inputs": [("x", "FULL", "F32"), ("w", "COLVEC", "F32")], "mask": None,
+    "ops": [("rm", "reduce", "RMAX", "ROW", "x"), ("wb", "broadcast", "COL", "w"),
+            ("mx", "binary", "MAX", "x", "wb"), ("mn", "binary", "MIN", "x", "wb")],
+    "outputs": [("rm", "F32"), ("mx", "F32"), ("mn", "F32")],
+}
+NAN_COL = dict(NAN_ROW, name="nan_col", ops=NAN_ROW["ops"] + [("cm", "reduce", "RMAX", "COL", "x")],
+               outputs=NAN_ROW["outputs"] + [("cm", "F32")])
+
+
+@pytest.mark.parametrize("spec,template", [(NAN_ROW, "row_team"), (NAN_COL, "global_sweep")])
+def test_nan_propagation_r12(spec, template):
+    rng = np.random.default_rng(12)
+    x = {"x": rng.standard_normal((300, 256)).astype(np.float32),
+         "w": rng.standard_normal(256).astype(np.float32)}
+    x["x"][7, 100] = np.nan
+    x["x"][299, 0] = np.nan
+    x["x"][150, 255] = np.nan
+    x["w"][33] = np.nan
+    got, plan = run_gpu(spec, x, return_plan=True)
+    assert plan.describe()["mapping"]["template"] == template
+    ref = evaluate(spec, x)
+    assert np.isnan(ref["rm"][[7, 150, 299]]).all() and np.isnan(ref["mx"][:, 33]).all()
+    _compare(spec, got, ref)        # non-finite reference values must be reproduced exactly
+
+
+def _virtual_ranks(spec, x, world):
+    """world ShardedPlans on one GPU (each sized for 148/world SMs), linked
+    peer exchanges, per-rank inputs / outputs / workspace / stream."""
+    import torch
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import PeerExchange, ShardedPlan
+    from tests.harness import device_inputs
+    rows, cols = spec["rows"], spec["cols"]
+    g = A.Graph.from_spec(spec)
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    ranks = []
+    for r in range(world):
+        sp = ShardedPlan(g, rows, cols, world, r, 0, sm_count=sms // world)
+        b, n = sp.row_begin, sp.row_count
+        xs = {k: (v[b:b + n] if getattr(v, "ndim", 0) == 2 else v) for k, v in x.items()}
+        ranks.append([sp, device_inputs(dict(spec, rows=n), xs), sp.plan.alloc_outputs(),
+                      sp.plan.alloc_workspace(), torch.cuda.Stream()])
+    for sp, *_ in ranks:
+        sp.peer = PeerExchange(sp.plan)
+    for sp, *_ in ranks:
+        for other, *_ in ranks:
+            if other is not sp:
+                sp.peer.link(other.rank, other.peer)
+    return ranks
+
+
+@pytest.mark.parametrize("K", [1, 3, 4])
+def test_fused_exchange_cuda_graph_replay(K):
+    """The fused exchange keeps its run generation in the exchange buffer
+    (bumped in-kernel), so a CUDA graph of K fused steps per rank can be
+    replayed: every replay is a fresh generation (odd K included), waits are
+    wrap-safe (flag - gen >= 0), and results match eager runs bitwise."""
+    import torch
+    from tests.harness import from_torch
+    world = 2
+    spec = specs.get("C5", rows=4099, cols=256)
+    x = gen.generate("C5", spec)
+    ranks = _virtual_ranks(spec, x, world)
+
+    def snapshot():
+        return [[from_torch(o).copy() for o in rk[2]] for rk in ranks]
+
+    torch.cuda.synchronize()
+    for sp, ins, outs, ws, st in ranks:         # eager warm-up: builds the fused kernel + peer table
+        sp.run(ins, outs, ws=ws, stream=st)
+    torch.cuda.synchronize()
+    eager = snapshot()
+    for rk in ranks:
+        for o in rk[2]:
+            o.zero_()
+    cap = torch.cuda.Stream()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph, stream=cap):
+        fork = torch.cuda.Event()
+        fork.record(cap)
+        joins = []
+        for sp, ins, outs, ws, st in ranks:
+            st.wait_event(fork)
+            for _ in range(K):
+                sp.run(ins, outs, ws=ws, stream=st)
+            e = torch.cuda.Event()
+            e.record(st)
+            joins.append(e)
+        for e in joins:
+            cap.wait_event(e)
+    for rep in range(3):
+        for rk in ranks:
+            for o in rk[2]:
+                o.zero_()
+        torch.cuda.synchronize()
+        graph.replay()
+        torch.cuda.synchronize()
+        for sp, *_ in ranks:
+            assert not sp.peer.timed_out(), f"replay {rep}: a rank timed out"
+        got = snapshot()
+        for r in range(world):
+            for a, b in zip(eager[r], got[r]):
+                assert np.array_equal(a, b), f"replay {rep} rank {r} differs from the eager run"
+    # eager runs interleaved with replays keep working (same generation counter)
+    for sp, ins, outs, ws, st in ranks:
+        sp.run(ins, outs, ws=ws, stream=st)
+    torch.cuda.synchronize()
+    for sp, *_ in ranks:
+        assert not sp.peer.timed_out()
+    got = snapshot()
+    for r in range(world):
+        for a, b in zip(eager[r], got[r]):
+            assert np.array_equal(a, b)
+
+
+
+def test_set_mask_matches_lengths_bitwise():
+    """astitch_graph_set_mask builds the same kernel as
+    astitch_graph_lengths: C3's masked softmax, bitwise equal outputs."""
+    import torch
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from tests.harness import device_inputs, from_torch
+    spec = specs.get("C3", rows=4 * 256)
+    spec["mask"]["rows_per_segment"] = 256
+    x = gen.generate("C3", spec)
+    ref = evaluate(spec, x)
+    g = A.Graph()
+    s_ = g.input("FULL", "BF16")
+    L = g.input("LENGTHS", "I32")
+    g.set_mask(L, 256)
+    n = {"s": s_}
+    for op in spec["ops"]:
+        if op[1] == "const":
+            n[op[0]] = g.const(op[2])
+        elif op[1] == "unary":
+            n[op[0]] = g.unary(op[2], n[op[3]])
+        elif op[1] == "binary":
+            n[op[0]] = g.binary(op[2], n[op[3]], n[op[4]])
+        elif op[1] == "reduce":
+            n[op[0]] = g.reduce(op[2], op[3], n[op[4]])
+        else:
+            n[op[0]] = g.broadcast(op[2], n[op[3]])
+    for name, dt in spec["outputs"]:
+        g.output(n[name], dt)
+    p = A.Plan(g, spec["rows"], spec["cols"], device=0)
+    outs = p.alloc_outputs()
+    p.run(device_inputs(spec, x), outs)
+    torch.cuda.synchronize()
+    got = run_gpu(spec, x)
+    assert np.array_equal(from_torch(outs[0]), got["p"])
+    _compare(spec, got, ref)
+
+
+@pytest.mark.parametrize("n,cols", [(3, 36), (7, 36), (12, 100), (16, 120), (2, 100)])
+def test_parity_smem_demoted_plans(n, cols):
+    """Graphs whose staged tiles would overflow shared memory (7-16 short-row
+    FULL inputs) plan a demoted mapping and stay within the oracle's tolerance."""
+    from tests.test_planner import _many_inputs_spec
+    spec = _many_inputs_spec(n, cols, rows=20_011)
+    x = gen.generate("fig6a", spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    assert plan.describe()["mapping"]["smem_bytes"] <= 227 * 1024
+    _compare(spec, got, evaluate(spec, x))
+
+
+def test_strict_single_kernel_flag():
+    """STRICT_SINGLE_KERNEL: a plan whose one-wave grid is resident is
+    unaffected (every benchmark graph); the flag only refuses to shrink a
+    non-resident planned grid."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    for cfg in ("C1", "C4", "C5"):
+        spec = specs.get(cfg, rows=4096 if cfg != "C1" else None)
+        x = gen.generate(cfg, spec)
+        got, plan = run_gpu(spec, x, return_plan=True, flags=A.FLAG_STRICT_SINGLE_KERNEL)
+        assert plan.kernel_count() == 1 and plan.describe()["demotions"] == []
+        _compare(spec, got, evaluate(spec, x))

@@ -269,3 +269,46 @@ def test_cluster_size_fills_one_wave():
         m = d["mapping"]
         assert m["template"] == "row_stream" and m["split"] == k, (rows, m["split"])
         assert rows * m["split"] <= 148 or m["split"] == 1
+
+
+def _many_inputs_spec(n, cols, rows=100_000, dt="F32"):
+    """n short-row FULL inputs summed, then a row-centred output (row reduce)."""
+    ins = [(f"x{i}", "FULL", dt) for i in range(n)]
+    ops, prev = [], "x0"
+    for i in range(1, n):
+        ops.append((f"a{i}", "binary", "ADD", prev, f"x{i}"))
+        prev = f"a{i}"
+    ops += [("s", "reduce", "SUM", "ROW", prev), ("sb", "broadcast", "ROW", "s"), ("y", "binary", "SUB", prev, "sb")]
+    return {"name": f"many{n}", "rows": rows, "cols": cols, "inputs": ins, "mask": None, "ops": ops,
+            "outputs": [("y", dt)]}
+
+
+@pytest.mark.parametrize("n", [2, 3, 7, 12, 16])
+@pytest.mark.parametrize("cols", [36, 100, 120])
+def test_smem_overflow_demotion(n, cols):
+    """a6 / P:L288: no plan ever asks for more shared memory than a B200 block
+    can have (227 KB opt-in); a staged tile that would overflow is demoted
+    (fewer stages / rows) or abandoned for a register row team, and the plan
+    says so in describe()["demotions"].  Round 1 planned 442-1475 KB here."""
+    s = _many_inputs_spec(n, cols)
+    d = A.Plan(A.Graph.from_spec(s), s["rows"], cols, device=-1, flags=A.FLAG_NO_COMPILE).describe()
+    m = d["mapping"]
+    assert m["smem_bytes"] <= 227 * 1024
+    if m["template"] == "packed_tile":
+        assert m["smem_bytes"] <= 100 * 1024           # >= 2 blocks per SM
+    if n >= 7:
+        assert m["template"] == "row_team" and m["smem_bytes"] == 0
+        assert any("row team" in x for x in d["demotions"])
+    assert d["kernel_count"] == 1
+
+
+def test_global_sweep_block_combine_fits_smem():
+    """The global sweep's block combine (teams x columns x 4 B, x2 for fp64
+    hi/lo partials) is demoted to fewer teams per block instead of
+    overflowing shared memory."""
+    for name, rows, cols in (("C5", 4096, 1024), ("bn", 3000, 4096), ("bn", 3000, 8192), ("C5", 4096, 16384)):
+        s = specs.get(name, rows=rows, cols=cols)
+        d = A.Plan(A.Graph.from_spec(s), rows, cols, device=-1, flags=A.FLAG_NO_COMPILE).describe()
+        m = d["mapping"]
+        assert m["smem_bytes"] <= 96 * 1024, (name, cols, m)
+        assert m["rows_per_block"] == 1 or m["smem_bytes"] > 0
