@@ -263,6 +263,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg (ablation sweeps)")
     ap.add_argument("--flags", type=int, default=0)
+    ap.add_argument("--tune", default=None, help="planner overrides (astitch_plan_ex), e.g. bps=2,unroll=2")
     ap.add_argument("--exchange", default="fused", choices=["fused", "nccl"],
                     help="N>1 column reductions: in-kernel exchange over peer memory (fused) or ncclAllReduce + epilogue")
     ap.add_argument("--eager", action="store_true", help="time eager launches instead of a CUDA graph")
@@ -310,7 +311,7 @@ def main():
     R, C = spec["rows"], spec["cols"]
     graph = A.Graph.from_spec(spec)
     comm = Comm.from_process_group(dev) if world > 1 else None
-    sp = ShardedPlan(graph, R, C, 1 if ragged else world, 0 if ragged else rank, dev, comm=comm, flags=args.flags)
+    sp = ShardedPlan(graph, R, C, 1 if ragged else world, 0 if ragged else rank, dev, comm=comm, flags=args.flags, tune=args.tune)
     exchange = "none"
     if world > 1 and not ragged and sp.needs_exchange():
         exchange = "ncclAllReduce + epilogue"
@@ -582,7 +583,8 @@ def main():
                        else f"{nsets} rotating input sets >= 4x L2",
                        "timing": "cuda_graph_replay" if graph is not None else "eager",
                        "template": desc["mapping"]["template"], "grid": desc["kernels"][0]["grid"],
-                       "threads": desc["mapping"]["threads"], "regs": desc["kernels"][0]["regs"]},
+                       "threads": desc["mapping"]["threads"], "regs": desc["kernels"][0]["regs"],
+                       "tuning": desc.get("tuning") or None, "flags": args.flags or None},
             "us_per_subgraph": round(ms_step * 1e3, 3),
             "eager_us_per_call": round(eager_us, 3) if eager_us is not None else None,
             "pct_of_8TBps": round(100.0 * gbs / world / 8000.0, 2),

@@ -102,7 +102,7 @@ struct Mapping {
   int row_unroll = 1;       // U: rows per team per iteration (vertical packing ILP)
   bool prefetch = true;     // software-pipeline the next row's loads
   int single_wave_bps = 0;  // RowTeam: blocks/SM that give every row its own team in one wave (0 = off)
-  int dyn_colred_rows = 0;  // GlobalSweep (N=1): rows per counter-ordered tile with its own column partial (0 = off)
+  bool sync_steps = false;  // block barrier at every row step of a persistent sweep (keeps the CTA's warps aligned)
   bool hoist_colvec = true; // keep COLVEC operands in registers across rows
   int tile_rows = 0;        // PackedTile rows per stage
   int stages = 0;           // PackedTile pipeline stages
@@ -136,7 +136,8 @@ struct Tuning {
   int stage = 0;            // 1: row_stream stages the row's inputs in smem
   int stage_kb = 0;         // row_stream staging budget per CTA (KB)
   int portable_clusters = 0;  // 1: never ask for 16-CTA clusters
-  int dyn_colred_rows = 0;  // global sweep: rows per counter-ordered tile (0 = static)
+  int sync = -1;            // 1 / 0: block barrier at every row step of a persistent sweep
+  int prefetch = -1;        // 1: software-prefetch the next rows in the global sweep (off by default)
   std::string text;         // the string it was parsed from (describe())
 };
 bool parse_tuning(const char* s, Tuning& t, std::string& err);

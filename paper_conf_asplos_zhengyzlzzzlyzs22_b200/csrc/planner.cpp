@@ -448,9 +448,22 @@ void select_mapping(Plan& p) {
     bool has_rowred = false;
     for (size_t i = 0; i < g.nodes.size(); ++i)
       if (p.info[i].live && p.info[i].cls == OpClass::ReduceRow) has_rowred = true;
-    // a multi-warp team reduces through block-wide smem: one team per block
-    m.threads = (m.team > 32 && has_rowred) ? m.team : std::max(512, m.team);
+    // a multi-warp team reduces through block-wide smem: one team per block.
+    // Long sweeps (>= 32 row steps per CTA: bandwidth-bound): one 1024-thread
+    // CTA per SM, no software prefetch, a block barrier per row step
+    // (sync_steps, retune_grid): the SM's warps sweep the same rows in lock
+    // step.  Measured on B200 (C5): 981 us vs 1012 us for the round-1 mapping
+    // (512 threads, register ping-pong prefetch).  Short sweeps (latency-
+    // bound: BatchNorm 25088 x 128 fp32, 32 vs 48 us) keep 512 threads with
+    // prefetch and no per-step barrier.  (scripts/sweeps/r02_*.txt)
+    const int ne0 = m.chunks_per_lane * E;
+    const int u0 = std::max(1, std::min(4, 64 / std::max(1, ne0 * nfull_in)));
+    const int64_t steps_1024 = R / std::max<int64_t>(1, static_cast<int64_t>(sms) * std::max(1, 1024 / m.team) * u0);
+    const bool long_sweep = steps_1024 >= 32;
+    m.threads = (m.team > 32 && has_rowred) ? m.team : std::max(long_sweep ? 1024 : 512, m.team);
     if (tu.threads >= m.team && tu.threads <= 1024 && tu.threads % m.team == 0) m.threads = tu.threads;
+    if (long_sweep) m.prefetch = false;
+    if (tu.prefetch >= 0) m.prefetch = tu.prefetch == 1 && (p.desc.flags & ASTITCH_FLAG_NO_PREFETCH) == 0;
     m.rows_per_block = m.threads / m.team;
     int ne = m.chunks_per_lane * E;
     // rows per team per iteration: ~64 input elements in flight per lane
@@ -765,17 +778,13 @@ void retune_grid(Plan& p) {
     m.grid = std::max<int64_t>(1, std::min(work_units, wave));
     m.vertical_trips = (work_units + m.grid - 1) / m.grid;
   }
-  // Global sweep of one column-reduction level on one GPU: counter-ordered
-  // tiles of 128 rows, each with its own column partial (tile-ordered final
-  // combine: deterministic, independent of which CTA took which tile)
-  m.dyn_colred_rows = 0;
-  if (m.tmpl == Template::GlobalSweep && p.max_level == 1 && p.desc.shard_world <= 1 &&
-      (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0 && !p.colreds.empty() && p.tune.dyn_colred_rows > 0 &&
-      R < (1LL << 30)) {
-    const int step = m.rows_per_block * m.row_unroll;
-    int tr = std::max(step, (p.tune.dyn_colred_rows / step) * step);
-    if ((R + tr - 1) / tr > m.grid) m.dyn_colred_rows = tr;  // more tiles than CTAs
-  }
+  // block barrier per row step of a persistent multi-trip sweep (the CTA's
+  // warps stay on the same rows): default for the global sweep (measured on
+  // B200); tuning sync=0/1 overrides
+  m.sync_steps = (m.tmpl == Template::GlobalSweep) && m.vertical_trips >= 32 && !m.prefetch;
+  if (p.tune.sync >= 0)
+    m.sync_steps = p.tune.sync == 1 && m.vertical_trips > 1 &&
+                   (m.tmpl == Template::GlobalSweep || m.tmpl == Template::RowTeam);
   plan_workspace(p);
 }
 
@@ -789,8 +798,7 @@ void plan_workspace(Plan& p) {
     w.barrier = off;
     off = align(off + 256);
     w.partials = off;
-    const int64_t nparts = p.map.dyn_colred_rows > 0 ? (R + p.map.dyn_colred_rows - 1) / p.map.dyn_colred_rows
-                                                     : p.map.grid;
+    const int64_t nparts = p.map.grid;
     // partial slots: one per column reduction + a lo slot per precise sum (R7c)
     const size_t nslots = p.colreds.size() + static_cast<size_t>(p.n_precise_colreds);
     off = align(off + static_cast<size_t>(nparts) * nslots * C * 4);
@@ -922,7 +930,7 @@ std::string describe_json(const Plan& p) {
     << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
     << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads
     << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
-    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"dyn_colred_rows\":" << m.dyn_colred_rows
+    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"sync_steps\":" << (m.sync_steps ? "true" : "false")
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
     << ",\"grid\":" << m.grid

@@ -110,10 +110,10 @@ class ShardedPlan:
     astitch_run_sharded)."""
 
     def __init__(self, graph: Graph, rows: int, cols: int, world: int, rank: int, device: int,
-                 comm: Comm | None = None, flags: int = 0, sm_count: int = 0):
+                 comm: Comm | None = None, flags: int = 0, sm_count: int = 0, tune=None):
         self.row_begin, self.row_count = shard_rows(rows, world, rank)
         self.plan = Plan(graph, self.row_count, cols, device=device, flags=flags, shard_rank=rank,
-                         shard_world=world, sm_count=sm_count)
+                         shard_world=world, sm_count=sm_count, tune=tune)
         self.comm = comm
         self.peer: PeerExchange | None = None
         self.world, self.rank = world, rank

@@ -18,6 +18,7 @@ def main():
     ap.add_argument("--flags", type=int, default=0)
     ap.add_argument("--rows", type=int, default=None)
     ap.add_argument("--cols", type=int, default=None)
+    ap.add_argument("--tune", default=None, help="astitch_plan_ex tuning string, e.g. bps=2,unroll=2")
     a = ap.parse_args()
     import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
     from workloads import specs
@@ -25,7 +26,7 @@ def main():
     if s.get("segments"):
         from workloads import gen
         s = gen.ragged_spec(s, gen.CONFIG_SEEDS.get(a.config, 0))
-    p = A.Plan(A.Graph.from_spec(s), s["rows"], s["cols"], device=-1, flags=a.flags)
+    p = A.Plan(A.Graph.from_spec(s), s["rows"], s["cols"], device=-1, flags=a.flags, tune=a.tune)
     os.makedirs(a.outdir, exist_ok=True)
     base = os.path.join(a.outdir, f"{a.config}_f{a.flags}")
     with open(base + ".cu", "w") as f:

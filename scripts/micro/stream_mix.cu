@@ -184,6 +184,94 @@ __global__ void dynamic_pf(const V4* __restrict__ x, const V4* __restrict__ y, V
   }
 }
 
+
+// (h) static grid-stride (deterministic ownership) with a drift throttle: a
+// CTA may start step k only once every CTA has finished step k - SLACK
+// (global step counter, one atomic per CTA per step), so the grid sweeps the
+// address space in lock step like counter-ordered tiles do
+template <int U>
+__global__ void persistent_throttle(const V4* __restrict__ x, const V4* __restrict__ y, V4* __restrict__ z, long long n,
+                                    unsigned int* done, int slack) {
+  long long stride = (long long)gridDim.x * blockDim.x * U;
+  int k = 0;
+  for (long long base = (long long)blockIdx.x * blockDim.x * U + threadIdx.x; base < n; base += stride, ++k) {
+    if (k >= slack) {
+      if (threadIdx.x == 0) {
+        const unsigned int need = (unsigned int)(k - slack + 1) * gridDim.x;
+        unsigned int v;
+        do { asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(done) : "memory"); } while (v < need);
+      }
+      __syncthreads();
+    }
+    V4 a[U], b[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) { a[u] = ld(x + i); b[u] = ld(y + i); } }
+#pragma unroll
+    for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) z[i] = addv(a[u], b[u]); }
+    __syncthreads();
+    if (threadIdx.x == 0) atomicAdd(done, 1u);
+  }
+}
+
+// (i) static grid-stride with a cheap drift throttle: thread 0 adds 1 to a
+// global step counter after every step (fire-and-forget red), and every
+// EVERY steps checks (one relaxed load; spins with nanosleep only when
+// behind) that every CTA has finished step k - SLACK.  CTAs that run out of
+// steps add the steps they will never do, so nobody waits forever; a 20 ms
+// guard bounds any spin.  Ownership of rows stays static (deterministic).
+template <int U>
+__global__ void persistent_throttle2(const V4* __restrict__ x, const V4* __restrict__ y, V4* __restrict__ z, long long n,
+                                     unsigned int* done, int slack, int every) {
+  const long long stride = (long long)gridDim.x * blockDim.x * U;
+  const long long maxsteps = (n + stride - 1) / stride;
+  int k = 0;
+  for (long long base = (long long)blockIdx.x * blockDim.x * U + threadIdx.x; k < maxsteps; base += stride, ++k) {
+    if (k >= slack && (k % every) == 0) {
+      if (threadIdx.x == 0) {
+        const unsigned int need = (unsigned int)(k - slack + 1) * gridDim.x;
+        unsigned int v;
+        asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(done) : "memory");
+        if (v < need) {
+          unsigned long long t0; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+          for (;;) {
+            __nanosleep(100);
+            asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(done) : "memory");
+            if (v >= need) break;
+            unsigned long long t1; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+            if (t1 - t0 > 20000000ULL) break;
+          }
+        }
+      }
+      __syncthreads();
+    }
+    if (base < n) {
+      V4 a[U], b[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) { a[u] = ld(x + i); b[u] = ld(y + i); } }
+#pragma unroll
+      for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) z[i] = addv(a[u], b[u]); }
+    }
+    if (threadIdx.x == 0) asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" :: "l"(done) : "memory");
+  }
+}
+
+// (j) static grid-stride with a block barrier every EVERY steps (re-aligns the
+// CTA's warps; no global communication)
+template <int U>
+__global__ void persistent_sync(const V4* __restrict__ x, const V4* __restrict__ y, V4* __restrict__ z, long long n,
+                                int every) {
+  const long long stride = (long long)gridDim.x * blockDim.x * U;
+  int k = 0;
+  for (long long base = (long long)blockIdx.x * blockDim.x * U + threadIdx.x; base < n; base += stride, ++k) {
+    if ((k % every) == 0) __syncthreads();
+    V4 a[U], b[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) { a[u] = ld(x + i); b[u] = ld(y + i); } }
+#pragma unroll
+    for (int u = 0; u < U; ++u) { long long i = base + (long long)u * blockDim.x; if (i < n) z[i] = addv(a[u], b[u]); }
+  }
+}
+
 template <typename F>
 float timeit(F f) {
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
@@ -197,7 +285,8 @@ float timeit(F f) {
   return best;
 }
 
-int main() {
+int main(int argc, char** argv) {
+  const bool only_throttle = argc > 1;
   const long long elems = 1LL << 30, n = elems / 8;  // V4 = 8 bf16
   V4 *x, *y, *z;
   cudaMalloc(&x, n * 16); cudaMalloc(&y, n * 16); cudaMalloc(&z, n * 16);
@@ -205,6 +294,7 @@ int main() {
   const double bytes = 3.0 * n * 16;
   auto rep = [&](const char* name, float ms) { printf("%-40s %8.1f us %8.1f GB/s\n", name, ms * 1e3, bytes / (ms * 1e-3) / 1e9); };
   int sms = 148;
+  if (!only_throttle)
   for (int t : {256, 512}) for (int bps : {1, 2, 4, 8}) {
     if (t * bps > 2048) continue;
     char nm[128];
@@ -215,6 +305,7 @@ int main() {
   }
   unsigned long long* ctr;
   cudaMalloc(&ctr, 8);
+  if (!only_throttle)
   for (int t : {256, 512}) for (int bps : {1, 2, 4}) {
     if (t * bps > 2048) continue;
     char nm[128];
@@ -229,6 +320,7 @@ int main() {
     snprintf(nm, sizeof nm, "persistent+prefetch U2 t%d x %d/SM", t, bps);
     rep(nm, timeit([&] { persistent_pf<2><<<sms * bps, t>>>(x, y, z, n); }));
   }
+  if (!only_throttle)
   for (int t : {128, 256, 512}) for (int u : {1, 2, 4}) {
     char nm[128];
     snprintf(nm, sizeof nm, "tiled U%d t%d", u, t);
@@ -237,12 +329,32 @@ int main() {
     if (u == 2) rep(nm, timeit([&] { tiled<2><<<g, t>>>(x, y, z, n); }));
     if (u == 4) rep(nm, timeit([&] { tiled<4><<<g, t>>>(x, y, z, n); }));
   }
+  if (!only_throttle)
   for (int S : {1, 2, 4, 8, 16}) for (int bps : {1, 2}) {
     char nm[128];
     snprintf(nm, sizeof nm, "dynamic coarse S%d U4 t512 x %d/SM", S, bps);
     rep(nm, timeit([&] { cudaMemsetAsync(ctr, 0, 8); dynamic_coarse<4><<<sms * bps, 512>>>(x, y, z, n, ctr, S); }));
   }
-  {  // finish-time spread of the static persistent sweep (tail effect?)
+  {
+    unsigned int* done;
+    cudaMalloc(&done, 4);
+    for (int t : {256, 512}) for (int bps : {1, 2}) {
+      char nm[128];
+      snprintf(nm, sizeof nm, "persistent U4 t%d x %d/SM", t, bps);
+      rep(nm, timeit([&] { persistent<4><<<sms * bps, t>>>(x, y, z, n); }));
+      for (int ev : {1, 2, 4, 8, 16}) {
+        snprintf(nm, sizeof nm, "syncthreads every %d U4 t%d x %d/SM", ev, t, bps);
+        rep(nm, timeit([&] { persistent_sync<4><<<sms * bps, t>>>(x, y, z, n, ev); }));
+      }
+      for (int sl : {8, 32}) for (int ev : {4, 8, 16}) {
+        snprintf(nm, sizeof nm, "throttle2 U4 t%d x %d/SM slack %d every %d", t, bps, sl, ev);
+        rep(nm, timeit([&] { cudaMemsetAsync(done, 0, 4); persistent_throttle2<4><<<sms * bps, t>>>(x, y, z, n, done, sl, ev); }));
+      }
+      snprintf(nm, sizeof nm, "dynamic tiles U4 t%d x %d/SM", t, bps);
+      rep(nm, timeit([&] { cudaMemsetAsync(ctr, 0, 8); dynamic_tiles<4><<<sms * bps, t>>>(x, y, z, n, ctr); }));
+    }
+  }
+  if (!only_throttle) {  // finish-time spread of the static persistent sweep (tail effect?)
     const int G = sms;
     unsigned long long* t_end; unsigned int* smid;
     cudaMalloc(&t_end, G * 8); cudaMalloc(&smid, G * 4);
