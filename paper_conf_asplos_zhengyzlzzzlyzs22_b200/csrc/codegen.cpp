@@ -587,7 +587,7 @@ struct Gen {
         } else {
           o << "#pragma unroll\n      for (int k = 0; k < NE; ++k) t_[k] = " << ref(nd.a, "k", sfx) << " - x0_;\n";
         }
-        o << "      float r_ = as::Tree<NE, false>::reduce(t_);\n";
+        o << "      float r_ = as::TreeSum<NE>::reduce(t_);\n";
         if (T > 1) o << "      r_ = as::team_sum<T>(r_);\n";
         o << "      d" << id << sfx << " = fma((double)x0_, (double)C, (double)r_);\n    }\n";
         emit_split(id, sfx);
@@ -642,7 +642,8 @@ struct Gen {
                        << " : " << ident << ";\n";
           else o << ref(src, "k", sfx) << ";\n";
         }
-        o << "      float r_ = as::Tree<" << nev() << ", " << (mx ? "true" : "false") << ">::reduce(t_);\n";
+        if (mx) o << "      float r_ = as::Tree<" << nev() << ", true>::reduce(t_);\n";
+        else o << "      float r_ = as::TreeSum<" << nev() << ">::reduce(t_);\n";
         if (T <= 32) o << "      r_ = as::team_" << (mx ? "max" : "sum") << "<T>(r_);\n";
         else if (split)
           o << "      r_ = as::cluster_team_reduce<" << m.threads << ", " << m.split << ", " << (mx ? "true" : "false")
@@ -1945,7 +1946,7 @@ struct Gen {
         else o << ref(N(r).a, "k", "") << ";\n";
         if (precise[r]) o << "        ad" << r << " += as::TreeD<NE>::reduce(t_);\n";
         else if (mx) o << "        a" << r << " = as::nmax(a" << r << ", as::Tree<NE, true>::reduce(t_));\n";
-        else o << "        a" << r << " += as::Tree<NE, false>::reduce(t_);\n";
+        else o << "        a" << r << " += as::TreeSum<NE>::reduce(t_);\n";
         o << "      }\n";
       }
       // FULL outputs of this level

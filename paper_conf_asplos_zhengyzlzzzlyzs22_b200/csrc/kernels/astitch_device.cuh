@@ -492,6 +492,30 @@ template <int N, bool MAX> struct Tree {
   }
 };
 
+// pairwise tree over f32x2 pairs: (a[0],a[1]), (a[2],a[3]), ... reduced with
+// paired FADD2 (half the issue slots of the scalar tree), then x + y.  A fixed
+// order, so deterministic (a different order from Tree<N,false>).
+template <int M> struct Tree2 {
+  __device__ static __forceinline__ f2 reduce(const float* a) {
+    if constexpr (M == 1) {
+      return f2{a[0], a[1]};
+    } else {
+      constexpr int H = M / 2;
+      return add2(Tree2<H>::reduce(a), Tree2<M - H>::reduce(a + 2 * H));
+    }
+  }
+};
+template <int N> struct TreeSum {
+  __device__ static __forceinline__ float reduce(const float* a) {
+    if constexpr (N >= 4 && (N % 2) == 0) {
+      const f2 r = Tree2<N / 2>::reduce(a);
+      return r.x + r.y;
+    } else {
+      return Tree<N, false>::reduce(a);
+    }
+  }
+};
+
 // ------------------------------------------------------------------ fused sharded exchange
 // System-scope release / acquire on flags that other GPUs write over NVLink
 // (peer memory); the data they guard is published with a system fence.

@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--flags", type=int, default=0)
     ap.add_argument("--rows", type=int, default=None)
     ap.add_argument("--cols", type=int, default=None)
+    ap.add_argument("--tune", default=None)
     args = ap.parse_args()
 
     import torch
@@ -50,7 +51,7 @@ def main():
         shape = {"FULL": (spec["segments"]["elems"],) if spec.get("segments") else (R, C),
                  "ROWVEC": (R,), "COLVEC": (C,)}[kind]
         ins.append(torch.randn(shape, generator=g, device="cuda", dtype=torch.float32).to(tdt[dt]))
-    plan = A.Plan(A.Graph.from_spec(spec), R, C, device=0, flags=args.flags)
+    plan = A.Plan(A.Graph.from_spec(spec), R, C, device=0, flags=args.flags, tune=args.tune)
     outs = plan.alloc_outputs()
     ws = plan.alloc_workspace()
     for _ in range(args.iters):
