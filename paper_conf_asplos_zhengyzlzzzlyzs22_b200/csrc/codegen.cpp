@@ -48,12 +48,19 @@ struct Gen {
     C = p.desc.cols;
     ragged = g.segments_node >= 0;
     masked = g.lengths_node >= 0 || ragged;  // varlen rows: masks of the row's own length
-    exact = (static_cast<long long>(T) * V * E == C);
+    slab = m.tmpl == Template::GlobalSweep && m.nslab > 1 && role != ROLE_SHARD_FINAL;
+    exact = slab ? (C % (static_cast<long long>(T) * V * E) == 0) : (static_cast<long long>(T) * V * E == C);
+    if (slab) tile_off = "SLABOFF";
     split = (m.tmpl == Template::SplitRow) || (m.tmpl == Template::RowStream && m.split > 1);
     compute_precise();
     compute_absorb();
   }
   bool split = false;
+  bool slab = false;  // column slabs (wide rows): every column index is offset by the CTA's slab
+  // chunk index of chunk j of this lane within its row (slab-relative columns + slab offset)
+  std::string chx(const std::string& j) const {
+    return slab ? "(" + j + " * T + lane + SLABCH)" : "(" + j + " * T + lane)";
+  }
   // chunk-count specialisation of masked rows: inside a `switch` on the
   // row's number of fully valid team chunks KF (a compile-time constant in
   // each case), chunk predicates fold at compile time, chunks past the
@@ -178,6 +185,14 @@ struct Gen {
         if (I(i).live && I(i).cls == OpClass::ReduceRow) ++nred;
       o << "  __shared__ float cl_slot[" << std::max(1, nred) << "];\n";
       o << "  __shared__ double cl_slot_d[" << std::max(1, nred) << "];\n";
+    } else if (slab) {
+      o << "  const int lane = threadIdx.x % T;\n";
+      o << "  const int team = threadIdx.x / T;\n";
+      o << "  constexpr int NSLAB = " << m.nslab << ";\n  constexpr long long SLABW = (long long)T * V * E;\n";
+      o << "  const int SLAB = (int)(blockIdx.x % NSLAB);  // column slab of this CTA\n";
+      o << "  const long long SLABOFF = (long long)SLAB * SLABW, SLABCH = (long long)SLAB * T * V;\n";
+      o << "  (void)SLABOFF; (void)SLABCH;\n";
+      o << "  const long long UNIT = blockIdx.x / NSLAB, NUNITS = gridDim.x / NSLAB;\n";
     } else {
       o << "  const int lane = threadIdx.x % T;\n";
       o << "  const int team = threadIdx.x / T;\n";
@@ -324,12 +339,12 @@ struct Gen {
       const Stream& st = streams[s];
       if (declare) o << "    " << raw_t(st) << " r" << s << sfx << "[V];\n";
       o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n";
-      o << "      const int c0 = (j * T + lane) * E;\n";
+      o << "      const long long c0 = " << chx("j") << " * E;\n";
       std::string cond = act;
       if (!exact || masked) cond += " && c0 < " + lim;
       o << "      if (" << cond << ") r" << s << sfx << "[j] = "
         << (st.ws_buf ? "as::ldg_cg(" : "as::ldg(") << "gs" << s << " + " << rowbase(row, lim)
-        << " + (j * T + lane));\n";
+        << " + " << chx("j") << ");\n";
       // chunks that are not loaded need no defined bits when the mask is
       // absorbed: the unpack step overwrites every invalid element with S
       if (!(absorb && !st.ws_buf)) o << "      else r" << s << sfx << "[j] = " << raw_t(st) << "{};\n";
@@ -983,16 +998,16 @@ struct Gen {
         o << "    if (" << act << ") {\n      " << rt << "* __restrict__ op_ = (" << rt << "*)p.out[" << k
           << "] + " << rowbase(row, lim) << ";\n";
         std::string val = ref(id, "(j * E + e)", sfx);
-        const std::string cguard = exact ? "" : "        if ((long long)(j * T + lane) < CH)\n";
+        const std::string cguard = exact ? "" : "        if ((long long)" + chx("j") + " < CH)\n";
         if (store_absorbed(id) && !ragged) {
           // every invalid element already holds 0 (absorbed mask): no
           // per-element selects; fully-masked rows (the only ones whose row
           // scalars may be non-finite) store zeros on a team-uniform branch
           o << "      if (" << lim << " > 0) {\n#pragma unroll\n      for (int j = 0; j < V; ++j) {\n        float t_[E];\n"
             << "#pragma unroll\n        for (int e = 0; e < E; ++e) t_[e] = " << val << ";\n"
-            << cguard << "        as::stg(op_ + (j * T + lane), as::Conv<" << dt_code(dt) << ", E>::pack(t_));\n"
+            << cguard << "        as::stg(op_ + " << chx("j") << ", as::Conv<" << dt_code(dt) << ", E>::pack(t_));\n"
             << "      }\n      } else {\n#pragma unroll\n      for (int j = 0; j < V; ++j) {\n"
-            << cguard << "        as::stg(op_ + (j * T + lane), " << rt << "{});\n      }\n      }\n    }\n";
+            << cguard << "        as::stg(op_ + " << chx("j") << ", " << rt << "{});\n      }\n      }\n    }\n";
           continue;
         }
         o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
@@ -1009,8 +1024,8 @@ struct Gen {
           o << "#pragma unroll\n        for (int e = 0; e < E; ++e) t_[e] = " << val << ";\n";
         }
         if (ragged) o << "        if (" << live_pred(lim) << " && (j * T + lane) * E < " << lim << ")  // chunks of the row only (packed)\n";
-        else if (!exact) o << "        if ((long long)(j * T + lane) < CH)\n";
-        o << "        as::stg(op_ + (j * T + lane), as::Conv<" << dt_code(dt) << ", E>::pack(t_));\n";
+        else if (!exact) o << "        if ((long long)" << chx("j") << " < CH)\n";
+        o << "        as::stg(op_ + " << chx("j") << ", as::Conv<" << dt_code(dt) << ", E>::pack(t_));\n";
         o << "      }\n    }\n";
       } else if (nd.kind == ASTITCH_ROWVEC) {
         o << "    if ((" << act << ") && lane == 0) as::st_scalar<" << dt_code(dt) << ">(p.out[" << k << "], " << row
@@ -1029,8 +1044,8 @@ struct Gen {
           o << "    if (" << act << ") {\n      " << rt << "* gb_ = (" << rt << "*)((char*)p.ws + " << off
             << "LL) + (" << row << ") * CH;\n";
           o << "#pragma unroll\n      for (int j = 0; j < V; ++j) {\n";
-          if (!exact) o << "        if ((long long)(j * T + lane) < CH)\n";
-          o << "        as::stg(gb_ + (j * T + lane), as::Conv<0, E>::pack(v" << id << sfx << " + j * E));\n";
+          if (!exact) o << "        if ((long long)" << chx("j") << " < CH)\n";
+          o << "        as::stg(gb_ + " << chx("j") << ", as::Conv<0, E>::pack(v" << id << sfx << " + j * E));\n";
           o << "      }\n    }\n";
         } else if (N(id).kind == ASTITCH_ROWVEC) {
           o << "    if ((" << act << ") && lane == 0) ((float*)((char*)p.ws + " << off << "LL))[" << row << "] = s"
@@ -1343,6 +1358,10 @@ struct Gen {
     o << "  }\n";
   }
 
+  // partial rows of column `col` combined by the finalise: every CTA's, or
+  // (column slabs) the CTAs of col's slab, r = slab + k * NSLAB, in k order
+  std::string fin_r0() const { return slab ? "(int)(col / SLABW) + pi * NSLAB" : "pi"; }
+  std::string fin_rs() const { return slab ? "P * NSLAB" : "P"; }
   // after the barrier: fixed-order combine of the grid partials per column
   // (deterministic), then the COLVEC consumers (global stage) for that column.
   // final == false (sharded): write the rank-local totals to ws colpart only.
@@ -1369,7 +1388,7 @@ struct Gen {
       std::string ident = mx ? "-AS_INF" : "0.f";
       if (pc(id)) {  // fp64 combine of the hi + lo partials (R7c)
         o << "      double t" << id << "d = 0.0;\n";
-        o << "      if (own) for (int r = pi; r < " << "G" << "; r += P) t" << id
+        o << "      if (own) for (int r = " << fin_r0() << "; r < G; r += " << fin_rs() << ") t" << id
           << "d += (double)as::ld_cg(part + ((long long)r * " << NS << " + " << q << ") * C + col) + (double)as::ld_cg(part + ((long long)r * "
           << NS << " + " << lo_slot(q) << ") * C + col);\n";
         o << "      fin_smem_d[threadIdx.x] = t" << id << "d;\n      __syncthreads();\n";
@@ -1379,7 +1398,7 @@ struct Gen {
         continue;
       }
       o << "      float t" << id << " = " << ident << ";\n";
-      o << "      if (own) for (int r = pi; r < " << "G" << "; r += P) { const float x_ = as::ld_cg(part + ((long long)r * " << NS
+      o << "      if (own) for (int r = " << fin_r0() << "; r < G; r += " << fin_rs() << ") { const float x_ = as::ld_cg(part + ((long long)r * " << NS
         << " + " << q << ") * C + col); t" << id << " = " << (mx ? "as::nmax(t" + std::to_string(id) + ", x_)" : "t" + std::to_string(id) + " + x_") << "; }\n";
       o << "      fin_smem[threadIdx.x] = t" << id << ";\n      __syncthreads();\n";
       o << "      for (int s = P / 2; s > 0; s /= 2) { if (pi < s) fin_smem[threadIdx.x] = "

@@ -195,7 +195,8 @@ astitch_status astitch_peer_create(astitch_plan_t h, astitch_peer_t* out, uint8_
       return s;
     }
     Kernel& k = pm.fused_kernels[0];
-    k.grid = std::min<int64_t>(k.grid, static_cast<int64_t>(k.occupancy) * pm.sm_count);
+    k.grid = resident_grid(pm, k);
+    if (k.grid < 1) return fail(ASTITCH_ERR_RESOURCE, "kernel cannot be resident");
   }
   auto* x = new astitch_peer_s();
   x->world = p.desc.shard_world;
@@ -285,7 +286,8 @@ astitch_status astitch_run_fused(astitch_plan_t h, astitch_peer_t x, const void*
     }
     Kernel& k = p.fused_kernels[0];
     if (!k.module && !drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
-    k.grid = std::min<int64_t>(k.grid, static_cast<int64_t>(k.occupancy) * p.sm_count);
+    k.grid = resident_grid(p, k);
+    if (k.grid < 1) return fail(ASTITCH_ERR_RESOURCE, "kernel cannot be resident");
   }
   if (x->table_dirty) {  // device addresses of every rank's buffer, read by the kernel
     std::vector<uint64_t> t(x->world);

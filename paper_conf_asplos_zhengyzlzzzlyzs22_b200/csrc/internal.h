@@ -7,6 +7,7 @@
 //   Plan     — everything astitch_run needs: kernels, launch config, workspace.
 #pragma once
 
+#include <algorithm>
 #include <cstdint>
 #include <memory>
 #include <string>
@@ -103,6 +104,7 @@ struct Mapping {
   bool prefetch = true;     // software-pipeline the next row's loads
   int single_wave_bps = 0;  // RowTeam: blocks/SM that give every row its own team in one wave (0 = off)
   bool sync_steps = false;  // block barrier at every row step of a persistent sweep (keeps the CTA's warps aligned)
+  int nslab = 1;            // GlobalSweep: column slabs of T x V x E columns (wide rows); CTA b owns slab b % nslab
   bool hoist_colvec = true; // keep COLVEC operands in registers across rows
   int tile_rows = 0;        // PackedTile rows per stage
   int stages = 0;           // PackedTile pipeline stages
@@ -204,6 +206,14 @@ struct Plan {
   int device = -1;
   std::string describe;
 };
+
+// a cooperative kernel's grid clamped to what is co-resident (whole row groups
+// of column slabs); 0 if not even one row group fits
+inline int64_t resident_grid(const Plan& p, const Kernel& k) {
+  int64_t g = std::min<int64_t>(k.grid, static_cast<int64_t>(k.occupancy) * p.sm_count);
+  if (p.map.nslab > 1) g = (g / p.map.nslab) * p.map.nslab;
+  return g;
+}
 
 // planner.cpp
 void analyse(Plan& p);                 // a1, a2, a5: classes, dominants, groups, schemes

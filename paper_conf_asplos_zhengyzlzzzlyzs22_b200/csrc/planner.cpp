@@ -445,9 +445,39 @@ void select_mapping(Plan& p) {
     m.tmpl = Template::GlobalSweep;
     choose_team(1024, 8, 16);
     if (no_pack && m.team < 32) { m.team = 32; m.chunks_per_lane = (chunks + 31) / 32; }
-    bool has_rowred = false;
-    for (size_t i = 0; i < g.nodes.size(); ++i)
+    bool has_rowred = false, has_rowvec = false;
+    for (size_t i = 0; i < g.nodes.size(); ++i) {
       if (p.info[i].live && p.info[i].cls == OpClass::ReduceRow) has_rowred = true;
+      if (p.info[i].live && g.nodes[i].kind == ASTITCH_ROWVEC) has_rowvec = true;
+    }
+    // Wide rows (a vocabulary-sized bias gradient, P:L103-L109 K3): a team
+    // keeps its row's columns in registers, so past ~16 values per lane it
+    // would spill.  Column slabs instead: the columns are cut into slabs of
+    // T x V x E (V*E ~ 8 values per lane) and CTA b sweeps slab b % nslab over
+    // its row group (b / nslab); each CTA's column partials cover its slab
+    // only, and the finalise sums the row groups of each column's slab in
+    // order (deterministic).  Element-wise + column-reduction graphs only (a
+    // row reduction needs the whole row in one team).
+    m.nslab = 1;
+    if (m.chunks_per_lane * E > 16 && !has_rowred && !has_rowvec && !has_mask && !ragged &&
+        (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0) {
+      const int T = 512;
+      const int64_t wave = 2LL * sms;                      // 2 x 512-thread CTAs per SM
+      int V = std::max(1, 8 / E);
+      int64_t ns = (chunks + static_cast<int64_t>(T) * V - 1) / (static_cast<int64_t>(T) * V);
+      while (ns > wave / 4 && V * E < 32) {               // keep >= 4 row groups per slab
+        V *= 2;
+        ns = (chunks + static_cast<int64_t>(T) * V - 1) / (static_cast<int64_t>(T) * V);
+      }
+      if (ns <= wave / 4) {
+        m.team = T;
+        m.chunks_per_lane = V;
+        m.nslab = static_cast<int>(ns);
+        m.lane_util = static_cast<double>(chunks) / (static_cast<double>(ns) * T * V);
+        why << "wide rows: " << ns << " column slabs of " << (T * V * E) << " columns (team " << T << " x " << V
+            << " chunks), CTA b -> slab b % " << ns << "; ";
+      }
+    }
     // a multi-warp team reduces through block-wide smem: one team per block.
     // Long sweeps (>= 32 row steps per CTA: bandwidth-bound): one 1024-thread
     // CTA per SM, no software prefetch, a block barrier per row step
@@ -462,6 +492,7 @@ void select_mapping(Plan& p) {
     const bool long_sweep = steps_1024 >= 32;
     m.threads = (m.team > 32 && has_rowred) ? m.team : std::max(long_sweep ? 1024 : 512, m.team);
     if (tu.threads >= m.team && tu.threads <= 1024 && tu.threads % m.team == 0) m.threads = tu.threads;
+    if (m.nslab > 1) m.threads = m.team;  // one 512-lane team per CTA (2 CTAs per SM)
     if (long_sweep) m.prefetch = false;
     if (tu.prefetch >= 0) m.prefetch = tu.prefetch == 1 && (p.desc.flags & ASTITCH_FLAG_NO_PREFETCH) == 0;
     m.rows_per_block = m.threads / m.team;
@@ -469,6 +500,7 @@ void select_mapping(Plan& p) {
     // rows per team per iteration: ~64 input elements in flight per lane
     // (measured on B200 for C5: U=4 reaches 98% of the copy roofline, U=2 94%)
     m.row_unroll = std::max(1, std::min(4, 64 / std::max(1, ne * nfull_in)));
+    if (m.nslab > 1) m.row_unroll = std::min(m.row_unroll, 2);  // 2 x 512-thread CTAs per SM at <= 64 registers
     if (tu.unroll >= 1 && tu.unroll <= 8) m.row_unroll = tu.unroll;
     // a6: block-level combine of the teams' column partials in smem
     // (rows_per_block teams x the team's columns, fp32; hi + lo for precise
@@ -774,6 +806,11 @@ void retune_grid(Plan& p) {
     int64_t clusters = std::max<int64_t>(1, std::min(work_units, wave / m.split));
     m.grid = clusters * m.split;
     m.vertical_trips = (work_units + clusters - 1) / clusters;
+  } else if (m.tmpl == Template::GlobalSweep && m.nslab > 1) {
+    // column slabs: nslab CTAs per row group, grid a multiple of nslab
+    const int64_t groups = std::max<int64_t>(1, std::min(work_units, wave / m.nslab));
+    m.grid = groups * m.nslab;
+    m.vertical_trips = (work_units + groups - 1) / groups;
   } else {
     m.grid = std::max<int64_t>(1, std::min(work_units, wave));
     m.vertical_trips = (work_units + m.grid - 1) / m.grid;
@@ -930,7 +967,7 @@ std::string describe_json(const Plan& p) {
     << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
     << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads
     << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
-    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"sync_steps\":" << (m.sync_steps ? "true" : "false")
+    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"sync_steps\":" << (m.sync_steps ? "true" : "false") << ",\"nslab\":" << m.nslab
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
     << ",\"grid\":" << m.grid

@@ -284,6 +284,9 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
           int64_t max_grid = static_cast<int64_t>(k.occupancy) * p.sm_count;
           if (max_grid < 1)
             return fail(ASTITCH_ERR_RESOURCE, "kernel " + k.name + " cannot be resident (occupancy 0)");
+          if (p.map.nslab > 1) max_grid = (max_grid / p.map.nslab) * p.map.nslab;  // whole row groups
+          if (max_grid < 1)
+            return fail(ASTITCH_ERR_RESOURCE, "kernel " + k.name + ": fewer resident CTAs than column slabs");
           if (k.grid > max_grid) {
             // the planned one-wave grid is not co-resident (the register /
             // smem estimate was optimistic): STRICT refuses, otherwise the
@@ -524,7 +527,10 @@ astitch_status astitch_run_host_pipelined(astitch_plan_t h, const void* const* h
     if ((s = build_kernel(p, ROLE_SHARD_FINAL, p.chunk_kernels[1])) != ASTITCH_OK) return s;
     for (Kernel& k : p.chunk_kernels) {
       if (!k.module && !drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
-      if (k.cooperative) k.grid = std::min<int64_t>(k.grid, static_cast<int64_t>(k.occupancy) * p.sm_count);
+      if (k.cooperative) {
+        k.grid = resident_grid(p, k);
+        if (k.grid < 1) return fail(ASTITCH_ERR_RESOURCE, "chunk kernel cannot be resident");
+      }
     }
   }
   for (int i = 0; i < 3; ++i)

@@ -709,3 +709,39 @@ def test_strict_single_kernel_flag():
         got, plan = run_gpu(spec, x, return_plan=True, flags=A.FLAG_STRICT_SINGLE_KERNEL)
         assert plan.kernel_count() == 1 and plan.describe()["demotions"] == []
         _compare(spec, got, evaluate(spec, x))
+
+
+@pytest.mark.parametrize("rows,cols", [(300, 40000), (37, 131072), (1000, 50001), (2049, 32768)])
+def test_parity_wide_column_slabs(rows, cols):
+    """Wide rows (K3 column reduce, a vocabulary-sized bias gradient): the
+    global sweep cuts the columns into slabs (CTA b -> slab b % nslab) so no
+    lane holds more than ~8 columns: no register spill, oracle parity,
+    bitwise run-to-run determinism."""
+    spec = specs.get("C5", rows=rows, cols=cols)
+    x = gen.generate("C5", spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    d = plan.describe()
+    assert d["mapping"]["nslab"] > 1 and d["kernels"][0]["spill_bytes"] == 0
+    _compare(spec, got, evaluate(spec, x))
+    again = run_gpu(spec, x, plan=plan)
+    for k in got:
+        assert np.array_equal(got[k], again[k])
+
+
+@pytest.mark.slow
+def test_wide_bias_grad_4096x131072_sampled():
+    """bf16 [4096, 131072] bias gradient (SURVEY 8(f) wide rows): sampled
+    columns against the oracle (column ops only: the sub-problem on those
+    columns is exact), sampled rows of dz, b_new bitwise from the GPU's db."""
+    spec = specs.get("C5", rows=4096, cols=131072)
+    x = gen.generate("C5", spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    assert plan.describe()["kernels"][0]["spill_bytes"] == 0
+    rng = np.random.default_rng(7)
+    cols = np.unique(np.concatenate([rng.integers(0, 131072, 40), [0, 4095, 4096, 131071]]))
+    refc = evaluate_columns(spec, x, cols)
+    check_close(got["db"][cols], refc["db"], "F32", 2e-3, "wide db")
+    check_close(got["dz"][:, cols], refc["dz"], "BF16", 2e-3, "wide dz")
+    b = x["b"].astype(np.float32)
+    exp = (b - np.float32(0.0078125) * got["db"].astype(np.float32)).astype(np.float32)
+    np.testing.assert_array_equal(got["b_new"].astype(np.float32), exp)
