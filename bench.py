@@ -190,28 +190,182 @@ def _out_kind(spec, name):
     return kinds[name]
 
 
+# ---------------------------------------------------------------------- oracle on the host cores
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def _shard_problem(cfg, spec, x, r0, n):
+    """The same graph on rows [r0, r0 + n) of a dense spec (masked specs: r0 a
+    multiple of rows_per_segment, lengths re-sliced)."""
+    from workloads import specs
+    sspec = specs.resized(spec, rows=n)
+    sx = {}
+    for name, kind, _ in spec["inputs"]:
+        v = x[name]
+        sx[name] = v[r0:r0 + n] if kind in ("FULL", "ROWVEC") else v
+    m = spec.get("mask")
+    if m is not None:
+        rps = m["rows_per_segment"]
+        assert r0 % rps == 0
+        sspec["mask"] = dict(m, rows_per_segment=min(rps, n))
+        sx[m["lengths"]] = x[m["lengths"]][r0 // rps: -(-(r0 + n) // rps)]
+        if n < rps:  # one partial segment: its single length
+            sx[m["lengths"]] = x[m["lengths"]][r0 // rps: r0 // rps + 1]
+    return sspec, sx
+
+
+def oracle_on_host_cores(cfg, spec, x, target_s=15.0, reps=1, rows_cap=None, skip=0, min_shard_rows=256,
+                         full_rows=None):
+    """The fp64 oracle as it stands (oracle.evaluate, unmodified) on every
+    host core: the rows (the method's independent units) are cut into W
+    contiguous shards, W = the cores this process may run on, and each shard
+    is evaluated by its own forked process (numpy pinned to one thread), the
+    same data-parallel split as the GPU path's row shards.  The sample is the
+    whole problem when it fits ~target_s of wall time at the pilot-measured
+    rate, else its first rows (a bounded sample, stated in the result).  Wall
+    time = last shard end - first shard start, median over `reps`.
+    Packed varlen specs shard whole segments."""
+    import multiprocessing as mp
+    import statistics
+    from oracle import evaluate
+    cores = len(os.sched_getaffinity(0))
+    ragged = bool(spec.get("segments"))
+    R = spec["rows"]
+    # pilot: one small slice in this process (rows/s of one core)
+    if ragged:
+        from workloads import gen
+        nseg = len(spec["segments"]["seg_rows"])
+        psub = gen.ragged_subset(spec, [0])
+        px = gen.generate(cfg, psub)
+        t0 = time.perf_counter()
+        evaluate(psub, px)
+        rate = psub["segments"]["elems"] / max(time.perf_counter() - t0, 1e-6)   # elements / s
+        total = spec["segments"]["elems"]
+    else:
+        unit = spec["mask"]["rows_per_segment"] if spec.get("mask") else 1
+        pr = min(R, max(unit, 256 if unit == 1 else unit))
+        psp, pxx = _shard_problem(cfg, spec, x, 0, pr)
+        t0 = time.perf_counter()
+        evaluate(psp, pxx, row_chunk=2048)
+        rate = pr / max(time.perf_counter() - t0, 1e-6)                          # rows / s
+        total = R
+    budget = rate * cores * target_s
+    W = cores
+    if ragged:
+        # whole segments, in order, until the element budget is reached
+        segs, acc = [], 0
+        for i, (r, c) in enumerate(zip(spec["segments"]["seg_rows"], spec["segments"]["seg_cols"])):
+            if segs and acc + r * c > budget:
+                break
+            segs.append(i)
+            acc += r * c
+        W = min(W, len(segs))
+        parts = [segs[k::W] for k in range(W)]
+        sample = f"segments 0-{segs[-1]} of {nseg} ({acc} valid elements)"
+    else:
+        rows = int(min(R, max(unit, budget), rows_cap or R))
+        rows = max(unit, rows // unit * unit) if unit > 1 else max(1, rows)
+        W = max(1, min(W, rows // max(unit, min_shard_rows)))
+        per = -(-rows // W)
+        if unit > 1:
+            per = -(-per // unit) * unit
+        bounds = [(r0, min(per, rows - r0)) for r0 in range(0, rows, per)]
+        W = len(bounds)
+        FR = full_rows or R
+        sample = f"rows 0-{rows - 1} of {FR}" + (" (whole problem)" if rows == FR else "") + f", {W} row shards"
+
+    def work(k, bar, q):
+        try:
+            from threadpoolctl import threadpool_limits
+            threadpool_limits(1)
+        except Exception:
+            pass
+        if ragged:
+            from workloads import gen
+            sspec = gen.ragged_subset(spec, parts[k])
+            sx = gen.generate(cfg, sspec, threads=1)
+        else:
+            sspec, sx = _shard_problem(cfg, spec, x, *bounds[k])
+        nb = compulsory_bytes(sspec, sx)
+        for _ in range(total_reps):
+            bar.wait()
+            a = time.time()
+            evaluate(sspec, sx, row_chunk=2048) if not ragged else evaluate(sspec, sx)
+            q.put((k, a, time.time(), nb))
+        bar.wait()
+
+    total_reps = reps + skip
+    ctx = mp.get_context("fork")
+    bar = ctx.Barrier(W)
+    q = ctx.Queue()
+    procs = [ctx.Process(target=work, args=(k, bar, q)) for k in range(W)]
+    for pr_ in procs:
+        pr_.start()
+    reps += skip
+    res = [q.get() for _ in range(W * reps)]
+    for pr_ in procs:
+        pr_.join()
+    walls, nbytes = [], 0
+    for r in range(skip, reps):
+        chunk = res[r * W:(r + 1) * W]
+        walls.append(max(c[2] for c in chunk) - min(c[1] for c in chunk))
+    nbytes = sum(c[3] for c in res[:W])
+    wall = statistics.median(walls)
+    return {"value": round(nbytes / wall / 1e9, 4), "unit": "GB/s", "cores": W, "kind": "oracle",
+            "sample": f"{sample}; unmodified numpy fp64 oracle, one process per core; "
+                      f"{wall:.2f} s wall (median of {reps - skip})",
+            "cpu_model": _cpu_model(), "host_cores": cores, "bytes": int(nbytes), "wall_s": round(wall, 3)}
+
+
 # ---------------------------------------------------------------------- reference arm
 def run_reference(args, rank, world):
-    """--impl reference: the fp64 oracle as it stands, on the host cores, on a
-    bounded row sample of the same workload (each step one sample)."""
+    """--impl reference: the fp64 oracle as it stands, on the host cores (one
+    process per core over row shards), each step a bounded sample of the same
+    workload (~2 s of wall time), median over the timed steps."""
     if rank != 0:
         return None
-    import numpy as np  # noqa: F401
-    from oracle import evaluate
-    from workloads import specs
     cfg = args.config
-    spec_full = _full_spec(cfg)
-    if spec_full.get("segments"):  # packed varlen: a bounded subset of whole segments
-        from workloads import gen
-        spec = gen.ragged_subset(spec_full, list(range(4)))
-        x = make_inputs(cfg, spec)
-        return _reference_line(args, world, cfg, spec, spec_full, x)
-    sample_rows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 200_000, "C5": 16384}.get(cfg, 4096)
-    spec = specs.get(cfg, rows=min(sample_rows, spec_full["rows"]))
-    if spec.get("mask"):
-        spec["mask"]["rows_per_segment"] = min(spec["mask"]["rows_per_segment"], spec["rows"])
-    x = make_inputs(cfg, spec)
-    return _reference_line(args, world, cfg, spec, spec_full, x)
+    spec = _full_spec(cfg, rows=args.rows, cols=args.cols)
+    if spec.get("segments"):
+        x = None
+    else:
+        # the rows a ~2 s step can cover on this host, generated once
+        from workloads import specs
+        cap = {"C1": 32, "C2": 4096, "C3": 524288, "C4": 2_000_000, "C5": 262144}.get(cfg, 65536)
+        cap = min(cap, spec["rows"])
+        if spec.get("mask"):
+            cap = max(spec["mask"]["rows_per_segment"], cap // spec["mask"]["rows_per_segment"] * spec["mask"]["rows_per_segment"])
+        sub = specs.resized(spec, rows=cap) if cap < spec["rows"] else spec
+        x = make_inputs(cfg, sub)
+    cpu = oracle_on_host_cores(cfg, spec if x is None else _sub_or_full(spec, x), x, target_s=2.0,
+                               reps=args.steps, skip=args.warmup, full_rows=spec["rows"])
+    gbs = cpu["value"]
+    dt = cpu["wall_s"]
+    return {
+        "impl": "reference", "metric": METRIC, "value": gbs, "unit": "GB/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
+        "config": {"workload": f"{cfg}: {WORKLOAD_NAMES.get(cfg, spec_name(cfg))}", "rows": spec["rows"], "cols": spec["cols"],
+                   "parallelism": f"host oracle, {cpu['cores']} processes (rank 0)"},
+        "cpu_baseline": cpu,
+        "e2e": {"value": gbs, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+
+
+def _sub_or_full(spec, x):
+    """The spec restricted to the rows present in x (the generated prefix)."""
+    from workloads import specs
+    n = len(next(v for k, v in x.items() if getattr(v, "ndim", 0) == 2))
+    return spec if n == spec["rows"] else specs.resized(spec, rows=n)
 
 
 def _full_spec(cfg, rows=None, cols=None):
@@ -221,32 +375,6 @@ def _full_spec(cfg, rows=None, cols=None):
     if spec.get("segments"):
         spec = gen.ragged_spec(spec, gen.CONFIG_SEEDS.get(cfg, 0))
     return spec
-
-
-def _reference_line(args, world, cfg, spec, spec_full, x):
-    from oracle import evaluate
-    nbytes = compulsory_bytes(spec, x)
-    for _ in range(args.warmup):
-        evaluate(spec, x)
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        evaluate(spec, x)
-    dt = (time.perf_counter() - t0) / args.steps
-    gbs = nbytes / dt / 1e9
-    sample = f"{spec['rows']} of {spec_full['rows']} rows x {spec['cols']} cols per step"
-    if spec.get("segments"):
-        sample = (f"segments 0-{len(spec['segments']['seg_rows']) - 1} of {len(spec_full['segments']['seg_rows'])} "
-                  f"({spec['rows']} of {spec_full['rows']} packed rows) per step")
-    return {
-        "impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s",
-        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic",
-        "config": {"workload": f"{cfg}: {WORKLOAD_NAMES.get(cfg, spec_name(cfg))}", "rows": spec["rows"], "cols": spec["cols"],
-                   "parallelism": "host oracle (rank 0)"},
-        "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
-        "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-    }
 
 
 # ---------------------------------------------------------------------- main arm
@@ -544,30 +672,11 @@ def main():
                 "bidir_ms": round(bidir_ms, 3), "floor_ms": round(floor, 3),
                 "frac_of_floor": round(floor / e2e_ms, 4)}
 
-    # ---- oracle on the host cores: bounded sample of the same workload (rank 0, N=1)
+    # ---- oracle on the host cores (rank 0, N=1): the whole problem (or a
+    # bounded sample of its rows) over one process per host core
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        from oracle import evaluate
-        if ragged:  # whole segments 0-7 (bit-identical to the full problem's)
-            from workloads import gen
-            sspec = gen.ragged_subset(spec, list(range(min(8, len(spec["segments"]["seg_rows"])))))
-            sx = make_inputs(cfg, sspec)
-        else:
-            srows = {"C1": 32, "C2": 4096, "C3": 8192, "C4": 400_000, "C5": 131_072}.get(cfg, 4096)
-            sspec = specs.get(cfg, rows=min(srows, R))
-            if sspec.get("mask"):
-                sspec["mask"]["rows_per_segment"] = min(sspec["mask"]["rows_per_segment"], sspec["rows"])
-            sx = {k: (v[: sspec["rows"]] if getattr(v, "ndim", 0) == 2 else v) for k, v in x.items()}
-            if sspec.get("mask"):
-                sx[sspec["mask"]["lengths"]] = x[spec["mask"]["lengths"]][: -(-sspec["rows"] // sspec["mask"]["rows_per_segment"])]
-        reps = 3 if cfg in ("C1", "C2") else 1
-        t0 = time.perf_counter()
-        for _ in range(reps):
-            evaluate(sspec, sx)
-        cdt = (time.perf_counter() - t0) / reps
-        cb = compulsory_bytes(sspec, sx)
-        cpu = {"value": round(cb / cdt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-               "sample": f"{sspec['rows']} of {R} rows x {C} cols (numpy fp64, {cdt:.2f} s)"}
+        cpu = oracle_on_host_cores(cfg, spec, x, target_s=15.0, reps=3 if cfg in ("C1", "C2") else 1)
 
     if rank == 0:
         clocks = clk.summary()

@@ -37,3 +37,14 @@ def test_reference_arm_other_ranks_silent():
              {"WORLD_SIZE": "2", "RANK": "1", "LOCAL_RANK": "1"})
     assert r.returncode == 0, r.stderr
     assert r.stdout.strip() == ""
+
+
+def test_reference_arm_uses_host_cores_and_records_cpu():
+    """SURVEY 8(d) oracle timing: one unmodified-oracle process per host core
+    over row shards; the line records the core count and the CPU model."""
+    r = _run(["--impl", "reference", "--config", "C4", "--steps", "2", "--warmup", "3"])
+    assert r.returncode == 0, r.stderr
+    d = json.loads([ln for ln in r.stdout.splitlines() if ln.strip()][-1])
+    cb = d["cpu_baseline"]
+    assert cb["cores"] >= 1 and cb["host_cores"] >= cb["cores"] and cb["cpu_model"]
+    assert "row shards" in cb["sample"] and cb["value"] > 0
