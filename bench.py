@@ -439,7 +439,18 @@ def main():
     R, C = spec["rows"], spec["cols"]
     graph = A.Graph.from_spec(spec)
     comm = Comm.from_process_group(dev) if world > 1 else None
-    sp = ShardedPlan(graph, R, C, 1 if ragged else world, 0 if ragged else rank, dev, comm=comm, flags=args.flags, tune=args.tune)
+    row_range = None
+    if spec.get("mask") and world > 1:
+        # masked batches: whole segments per rank, balanced by compulsory bytes
+        from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import mask_row_ranges
+        from workloads import gen as _gen
+        L = _gen.lengths_for(spec, _gen.CONFIG_SEEDS.get(cfg, 0))
+        es = {"F32": 4, "BF16": 2, "F16": 2}
+        ein = sum(es[d] for _, k, d in spec["inputs"] if k == "FULL")
+        eout = sum(es[d] for n, d in spec["outputs"] if _out_kind(spec, n) == "FULL")
+        row_range = mask_row_ranges(L, spec["mask"]["rows_per_segment"], C, R, world, ein, eout)[rank]
+    sp = ShardedPlan(graph, R, C, 1 if ragged else world, 0 if ragged else rank, dev, comm=comm, flags=args.flags,
+                     tune=args.tune, row_range=row_range)
     exchange = "none"
     if world > 1 and not ragged and sp.needs_exchange():
         exchange = "ncclAllReduce + epilogue"

@@ -182,7 +182,9 @@ enum {
   ASTITCH_FLAG_LAUNCH_CHECK = 1u << 7,  /* synchronise + check after every launch (debug)*/
   ASTITCH_FLAG_FORCE_SPLIT = 1u << 8,   /* ablation: split rows over clusters whenever the
                                            paper's shape rule holds (no B200 size threshold) */
-  ASTITCH_FLAG_NO_PDL = 1u << 9         /* launch without programmatic dependent launch   */
+  ASTITCH_FLAG_NO_PDL = 1u << 9,        /* launch without programmatic dependent launch   */
+  ASTITCH_FLAG_DEBUG_BARRIER = 1u << 10 /* debug: a grid barrier waiting > 5 s prints and
+                                           traps (a launch error) instead of spinning on */
 };
 
 typedef struct {
@@ -224,6 +226,12 @@ astitch_status astitch_plan(astitch_graph_t g, const astitch_plan_desc* desc, as
 astitch_status astitch_plan_ex(astitch_graph_t g, const astitch_plan_desc* desc, const char* tuning,
                                astitch_plan_t* out);
 astitch_status astitch_plan_destroy(astitch_plan_t p);
+/* Directory of the on-disk cubin cache (generated kernels compiled by NVRTC,
+ * one file per source: "<dir>/<64-bit hash>.cubin", written atomically).
+ * NULL or "" disables it.  Default: $XDG_CACHE_HOME/astitch, else
+ * $HOME/.cache/astitch.  A cache hit skips NVRTC; describe()'s plan_time_ms
+ * reports the plan's analysis / codegen / NVRTC / load times and the hits. */
+astitch_status astitch_set_cache_dir(const char* dir);
 /* Bytes of device workspace astitch_run needs (0 if none). */
 astitch_status astitch_plan_workspace_bytes(astitch_plan_t p, size_t* bytes);
 /* JSON description: op classes, dominants, groups, schemes, mapping, grid,

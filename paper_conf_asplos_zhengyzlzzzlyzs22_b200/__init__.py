@@ -12,8 +12,9 @@ Multi-GPU row sharding lives in ``.dist``.
 
 from ._lib import (FLAG_FORCE_GLOBAL, FLAG_LAUNCH_CHECK, FLAG_NO_COMPILE, FLAG_NO_PACK,  # noqa: F401
                    FLAG_FORCE_SPLIT, FLAG_NO_PREFETCH, FLAG_NO_SPLIT, FLAG_NO_TMA,
-                   FLAG_STRICT_SINGLE_KERNEL, LIB_PATH,
+                   FLAG_STRICT_SINGLE_KERNEL, FLAG_NO_PDL, FLAG_DEBUG_BARRIER, LIB_PATH,
                    AstitchError)
-from .api import Graph, Plan, bench_barrier, bench_copy, plan, segments_layout, shard_rows  # noqa: F401
+from .api import (Graph, Plan, bench_barrier, bench_copy, plan, segments_layout, set_cache_dir,  # noqa: F401
+                  shard_rows)
 
-__version__ = "0.1.0"
+__version__ = "0.2.0"

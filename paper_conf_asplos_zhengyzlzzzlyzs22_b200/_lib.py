@@ -36,6 +36,7 @@ FLAG_NO_PREFETCH = 1 << 6
 FLAG_LAUNCH_CHECK = 1 << 7
 FLAG_FORCE_SPLIT = 1 << 8
 FLAG_NO_PDL = 1 << 9
+FLAG_DEBUG_BARRIER = 1 << 10
 
 
 class AstitchError(RuntimeError):
@@ -79,6 +80,7 @@ _sig = {
     "astitch_graph_output": (ct.c_int, [_vp, ct.c_int32, ct.c_int, _i32p]),
     "astitch_plan": (ct.c_int, [_vp, ct.POINTER(PlanDesc), ct.POINTER(_vp)]),
     "astitch_plan_ex": (ct.c_int, [_vp, ct.POINTER(PlanDesc), ct.c_char_p, ct.POINTER(_vp)]),
+    "astitch_set_cache_dir": (ct.c_int, [ct.c_char_p]),
     "astitch_plan_destroy": (ct.c_int, [_vp]),
     "astitch_plan_workspace_bytes": (ct.c_int, [_vp, ct.POINTER(ct.c_size_t)]),
     "astitch_plan_describe": (ct.c_int, [_vp, ct.c_char_p, ct.c_size_t, ct.POINTER(ct.c_size_t)]),

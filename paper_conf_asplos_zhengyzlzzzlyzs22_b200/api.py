@@ -170,7 +170,8 @@ class Plan:
         check(lib.astitch_plan_io_count(h, ct.byref(ni), ct.byref(no)), "astitch_plan_io_count")
         self.inputs = [self._io(0, i) for i in range(ni.value)]
         self.outputs = [self._io(1, i) for i in range(no.value)]
-        self._ws_cache = None
+        self._ws_cache = None   # workspace per stream (concurrent runs need distinct workspaces)
+        self._ws_by_stream = {}
 
     def __del__(self):
         h = getattr(self, "_h", None)
@@ -277,14 +278,34 @@ class Plan:
                     raise ValueError(f"{what} {i} ({kind}): {t.numel()} elements, plan expects {n}")
                 if device and not t.is_cuda:
                     raise ValueError(f"{what} {i} ({kind}): expected a CUDA tensor")
+                if device and t.device.index is not None and t.device.index != self.device:
+                    raise ValueError(f"{what} {i} ({kind}): tensor on cuda:{t.device.index}, plan is for cuda:{self.device}")
+
+    def _stream_ws(self, stream):
+        """The plan's cached workspace for `stream` (one per stream: the grid
+        barrier words of a workspace must not be shared by concurrent runs)."""
+        if self.workspace_bytes() == 0:
+            return None
+        sp = _stream_ptr(stream)
+        ws = self._ws_by_stream.get(sp)
+        if ws is None:
+            ws = self._ws_by_stream[sp] = self.alloc_workspace(stream)
+            if self._ws_cache is None:
+                self._ws_cache = ws
+        return ws
+
+    def _check_stream(self, stream):
+        if stream is not None and not isinstance(stream, int):
+            dev = getattr(stream, "device", None)
+            if dev is not None and getattr(dev, "index", None) is not None and dev.index != self.device:
+                raise ValueError(f"stream is on cuda:{dev.index}, plan is for cuda:{self.device}")
 
     def run(self, inputs, outputs, ws=None, stream=None) -> None:
         """astitch_run on device tensors (in declaration order) on `stream`."""
         self.check_io(inputs, outputs)
-        if ws is None and self._ws_cache is None and self.workspace_bytes() > 0:
-            self._ws_cache = self.alloc_workspace(stream)
+        self._check_stream(stream)
         if ws is None:
-            ws = self._ws_cache
+            ws = self._stream_ws(stream)
         ins = ptr_array([t.data_ptr() for t in inputs])
         outs = ptr_array([t.data_ptr() for t in outputs])
         check(lib.astitch_run(self._h, ins, outs, ct.c_void_p(ws.data_ptr() if ws is not None else 0),
@@ -296,10 +317,9 @@ class Plan:
         call is the C-ABI call (pointer arrays, workspace and stream are
         resolved once here; the tensors are kept alive by the callable)."""
         self.check_io(inputs, outputs)
-        if ws is None and self._ws_cache is None and self.workspace_bytes() > 0:
-            self._ws_cache = self.alloc_workspace(stream)
+        self._check_stream(stream)
         if ws is None:
-            ws = self._ws_cache
+            ws = self._stream_ws(stream)
         ins = ptr_array([t.data_ptr() for t in inputs])
         outs = ptr_array([t.data_ptr() for t in outputs])
         w = ct.c_void_p(ws.data_ptr() if ws is not None else 0)
@@ -321,10 +341,9 @@ class Plan:
         H2D inputs, stitched kernel(s), D2H outputs, asynchronous on `stream`."""
         self.check_io(host_inputs, host_outputs, device=False)
         self.check_io(dev_inputs, dev_outputs)
-        if ws is None and self.workspace_bytes() > 0:
-            if self._ws_cache is None:
-                self._ws_cache = self.alloc_workspace(stream)
-            ws = self._ws_cache
+        self._check_stream(stream)
+        if ws is None:
+            ws = self._stream_ws(stream)
         hi = ptr_array([t.data_ptr() for t in host_inputs])
         ho = ptr_array([t.data_ptr() for t in host_outputs])
         di = ptr_array([t.data_ptr() for t in dev_inputs])
@@ -356,6 +375,11 @@ def segments_layout(seg_rows, seg_cols):
     return [list(t[4 * s: 4 * s + 4]) for s in range(nseg)], rows.value, elems.value
 
 
+def set_cache_dir(path: str | None) -> None:
+    """astitch_set_cache_dir: on-disk cubin cache directory (None / "" = off)."""
+    check(lib.astitch_set_cache_dir(path.encode() if path else None), "astitch_set_cache_dir")
+
+
 def shard_rows(rows: int, world: int, rank: int) -> tuple[int, int]:
     b, c = ct.c_int64(), ct.c_int64()
     check(lib.astitch_shard_rows(int(rows), int(world), int(rank), ct.byref(b), ct.byref(c)), "astitch_shard_rows")
@@ -372,4 +396,4 @@ def bench_copy(device: int, src, dst, nbytes: int, stream=None) -> None:
                                  ct.c_void_p(_stream_ptr(stream))), "astitch_bench_copy")
 
 
-__all__ = ["Graph", "Plan", "plan", "segments_layout", "shard_rows", "bench_barrier", "bench_copy", "AstitchError"]
+__all__ = ["Graph", "Plan", "plan", "segments_layout", "shard_rows", "set_cache_dir", "bench_barrier", "bench_copy", "AstitchError"]

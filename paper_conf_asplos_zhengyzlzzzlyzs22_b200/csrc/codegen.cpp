@@ -159,6 +159,7 @@ struct Gen {
   void header(const std::string& name, bool cooperative_sync) {
     (void)cooperative_sync;
     o << "// generated by astitch codegen: " << template_name(m.tmpl) << " role " << role << "\n";
+    if (p.desc.flags & ASTITCH_FLAG_DEBUG_BARRIER) o << "#define AS_BARRIER_TIMEOUT_NS 5000000000ULL\n";
     o << "#include \"astitch_device.cuh\"\n";
     o << "struct Params { const void* in[16]; void* out[16]; void* ws; long long rows; long long row_offset; int flags; void* xbuf; unsigned int gen; };\n";
     o << "extern \"C\" __global__ void __launch_bounds__(" << m.threads << ", " << m.blocks_per_sm << ") ";

@@ -179,6 +179,10 @@ struct Plan {
   int sm_count = 148;
   int smem_optin = 232448;       // max dynamic+static smem per block (B200: 227 KB; device query)
   std::vector<std::string> demotions;  // resource-driven mapping changes (a6), in order (describe())
+  // plan (JIT) time, milliseconds: analysis + mapping, code generation,
+  // NVRTC (or cubin cache), module load; and the compile / cache counts
+  double ms_analyse = 0, ms_codegen = 0, ms_nvrtc = 0, ms_load = 0, ms_total = 0;
+  int n_compiles = 0, n_mem_hits = 0, n_disk_hits = 0;
   std::vector<NodeInfo> info;
   std::vector<std::vector<int>> groups;
   Mapping map;
@@ -240,9 +244,12 @@ inline size_t xbuf_bytes(int world, size_t ncolred, int64_t cols) {
 }
 
 // jit.cpp
+// cache_state (optional out): 0 = compiled by NVRTC, 1 = in-process cache hit,
+// 2 = on-disk cache hit (astitch_set_cache_dir)
 bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<char>& cubin,
-                   std::string& log, std::string& err);
+                   std::string& log, std::string& err, int* cache_state = nullptr);
 const char* device_header_source();
+void set_cache_dir(const char* dir);  // "" disables the on-disk cubin cache
 
 // driver.cpp — libcuda via dlopen
 struct Driver;

@@ -3,8 +3,14 @@
 // LLVM backend is replaced by NVRTC + ptxas).  libnvrtc is dlopen'ed so the
 // library loads on machines without CUDA libraries on the default path.
 #include <dlfcn.h>
+#include <sys/stat.h>
+#include <unistd.h>
 
+#include <cerrno>
+#include <cstdio>
 #include <cstdlib>
+#include <fstream>
+#include <sstream>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -84,18 +90,112 @@ Nvrtc* load_nvrtc(std::string& err) {
 std::mutex g_cache_mu;
 std::unordered_map<std::string, std::pair<std::vector<char>, std::string>> g_cache;
 
+// ---- on-disk cubin cache (astitch_set_cache_dir): one file per generated
+// source, keyed by a 64-bit FNV-1a of (source, device header, NVRTC options);
+// the file repeats the source length and hash and is written atomically
+// (temp + rename), so concurrent processes and stale files are harmless.
+std::mutex g_dir_mu;
+bool g_dir_set = false;
+std::string g_dir;
+
+uint64_t fnv(const std::string& s, uint64_t h = 1469598103934665603ULL) {
+  for (unsigned char c : s) {
+    h ^= c;
+    h *= 1099511628211ULL;
+  }
+  return h;
+}
+
+std::string cache_dir() {
+  std::lock_guard<std::mutex> lk(g_dir_mu);
+  if (g_dir_set) return g_dir;
+  const char* x = getenv("XDG_CACHE_HOME");
+  const char* h = getenv("HOME");
+  if (x && *x) return std::string(x) + "/astitch";
+  if (h && *h) return std::string(h) + "/.cache/astitch";
+  return "";
+}
+
+bool mkdirs(const std::string& d) {
+  if (d.empty()) return false;
+  std::string cur;
+  std::stringstream ss(d);
+  std::string part;
+  if (d[0] == '/') cur = "/";
+  while (std::getline(ss, part, '/')) {
+    if (part.empty()) continue;
+    cur += part + "/";
+    if (mkdir(cur.c_str(), 0755) != 0 && errno != EEXIST) return false;
+  }
+  return true;
+}
+
+const char* kMagic = "ASTITCH-CUBIN-2";
+
+bool disk_load(const std::string& path, uint64_t key, size_t src_len, std::vector<char>& cubin, std::string& log) {
+  std::ifstream f(path, std::ios::binary);
+  if (!f) return false;
+  std::string magic;
+  uint64_t k = 0;
+  size_t sl = 0, ls = 0, cs = 0;
+  if (!std::getline(f, magic) || magic != kMagic) return false;
+  if (!(f >> k >> sl >> ls >> cs) || k != key || sl != src_len || cs == 0 || cs > (1u << 30)) return false;
+  f.get();  // newline
+  log.assign(ls, '\0');
+  cubin.resize(cs);
+  if (ls && !f.read(&log[0], static_cast<std::streamsize>(ls))) return false;
+  if (!f.read(cubin.data(), static_cast<std::streamsize>(cs))) return false;
+  return true;
+}
+
+void disk_store(const std::string& dir, const std::string& path, uint64_t key, size_t src_len,
+                const std::vector<char>& cubin, const std::string& log) {
+  if (!mkdirs(dir)) return;
+  const std::string tmp = path + ".tmp" + std::to_string(getpid());
+  {
+    std::ofstream f(tmp, std::ios::binary);
+    if (!f) return;
+    f << kMagic << "\n" << key << " " << src_len << " " << log.size() << " " << cubin.size() << "\n";
+    f.write(log.data(), static_cast<std::streamsize>(log.size()));
+    f.write(cubin.data(), static_cast<std::streamsize>(cubin.size()));
+    if (!f) { std::remove(tmp.c_str()); return; }
+  }
+  if (std::rename(tmp.c_str(), path.c_str()) != 0) std::remove(tmp.c_str());
+}
+
 }  // namespace
 
+void set_cache_dir(const char* dir) {
+  std::lock_guard<std::mutex> lk(g_dir_mu);
+  g_dir_set = true;
+  g_dir = dir ? dir : "";
+}
+
 bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<char>& cubin,
-                   std::string& log, std::string& err) {
+                   std::string& log, std::string& err, int* cache_state) {
+  if (cache_state) *cache_state = 0;
   {
     std::lock_guard<std::mutex> lk(g_cache_mu);
     auto it = g_cache.find(src);
     if (it != g_cache.end()) {
       cubin = it->second.first;
       log = it->second.second;
+      if (cache_state) *cache_state = 1;
       return true;
     }
+  }
+  static const char* kOpts = "--gpu-architecture=sm_100a --std=c++17 -default-device --generate-line-info "
+                             "--ptxas-options=-v -DASTITCH_JIT=1 -diag-suppress=177,550";
+  const uint64_t key = fnv(src, fnv(kOpts, fnv(kAstitchDeviceCuh)));
+  const std::string dir = cache_dir();
+  char hex[32];
+  snprintf(hex, sizeof(hex), "%016llx", static_cast<unsigned long long>(key));
+  const std::string path = dir.empty() ? "" : dir + "/" + hex + ".cubin";
+  if (!path.empty() && disk_load(path, key, src.size(), cubin, log)) {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    g_cache[src] = {cubin, log};
+    if (cache_state) *cache_state = 2;
+    return true;
   }
   Nvrtc* n = load_nvrtc(err);
   if (!n) return false;
@@ -126,6 +226,7 @@ bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<
   cubin.resize(cs);
   n->cubin(prog, cubin.data());
   n->destroy(&prog);
+  if (!path.empty()) disk_store(dir, path, key, src.size(), cubin, log);
   std::lock_guard<std::mutex> lk(g_cache_mu);
   g_cache[src] = {cubin, log};
   return true;

@@ -575,7 +575,20 @@ __device__ __forceinline__ void grid_barrier(u32* bar) {
       asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(bar), "r"(0u) : "memory");
       st_release(bar + 1, gen + 1);
     } else {
+#ifdef AS_BARRIER_TIMEOUT_NS
+      // debug build of the barrier (ASTITCH_FLAG_DEBUG_BARRIER): a block that
+      // never arrives (a non-resident grid, a corrupted workspace) makes the
+      // waiters trap after the bound instead of hanging the GPU
+      const unsigned long long t0 = globaltimer_ns();
+      while (ld_acquire(bar + 1) == gen) {
+        if (globaltimer_ns() - t0 > (unsigned long long)(AS_BARRIER_TIMEOUT_NS)) {
+          printf("astitch: grid barrier timeout (block %u of %u arrived count %u)\n", blockIdx.x, nb, ld_acquire(bar));
+          __trap();
+        }
+      }
+#else
       while (ld_acquire(bar + 1) == gen) { }
+#endif
     }
   }
   __syncthreads();

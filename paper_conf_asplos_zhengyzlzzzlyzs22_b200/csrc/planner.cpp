@@ -998,6 +998,10 @@ std::string describe_json(const Plan& p) {
       << ",\"occupancy_blocks_per_sm\":" << kk.occupancy << ",\"cubin_bytes\":" << kk.cubin.size() << "}";
   }
   o << "],\"shard_kernels\":" << p.shard_kernels.size();
+  o << ",\"plan_time_ms\":{\"analyse_map\":" << p.ms_analyse << ",\"codegen\":" << p.ms_codegen
+    << ",\"nvrtc\":" << p.ms_nvrtc << ",\"load\":" << p.ms_load << ",\"total\":" << p.ms_total
+    << ",\"nvrtc_compiles\":" << p.n_compiles << ",\"cache_hits_memory\":" << p.n_mem_hits
+    << ",\"cache_hits_disk\":" << p.n_disk_hits << "}";
   o << ",\"compulsory_bytes\":" << p.compulsory_bytes << "}";
   return o.str();
 }

@@ -1,4 +1,5 @@
 // Plan construction (JIT) and execution entry points of the C ABI.
+#include <chrono>
 #include <cstdio>
 #include <cstring>
 #include <mutex>
@@ -10,6 +11,10 @@
 using namespace astitch;
 
 namespace {
+
+double ms_since(std::chrono::steady_clock::time_point t0) {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
 
 uint64_t fnv1a(const std::string& s) {
   uint64_t h = 1469598103934665603ULL;
@@ -68,12 +73,20 @@ static astitch_status compile_and_inspect(Plan& p, Kernel& k, bool load) {
   if (k.module) drv_unload(k);
   k.regs = -1;
   k.spill_bytes = -1;
-  if (!nvrtc_compile(k.source, k.name, k.cubin, k.log, err)) return fail(ASTITCH_ERR_CUDA, err);
+  auto t0 = std::chrono::steady_clock::now();
+  int cs = 0;
+  if (!nvrtc_compile(k.source, k.name, k.cubin, k.log, err, &cs)) return fail(ASTITCH_ERR_CUDA, err);
+  p.ms_nvrtc += ms_since(t0);
+  if (cs == 0) ++p.n_compiles;
+  else if (cs == 1) ++p.n_mem_hits;
+  else ++p.n_disk_hits;
   parse_ptxas(k);
   if (load) {
     int log_spill = k.spill_bytes;
     k.spill_bytes = -1;
+    auto t1 = std::chrono::steady_clock::now();
     if (!drv_load(p, k, err)) return fail(ASTITCH_ERR_CUDA, err);
+    p.ms_load += ms_since(t1);
     k.spill_bytes = std::max(log_spill, k.spill_bytes);
   }
   return ASTITCH_OK;
@@ -92,7 +105,9 @@ astitch_status build_kernel(Plan& p, int role, Kernel& k) {
   auto gen_compile = [&]() -> astitch_status {
     std::string base = std::string("astitch_") + template_name(p.map.tmpl) + role_suffix(role);
     k.name = base;
+    auto tg = std::chrono::steady_clock::now();
     k.source = generate_kernel(p, role, base);
+    p.ms_codegen += ms_since(tg);
     char hb[32];
     snprintf(hb, sizeof(hb), "_%012llx", static_cast<unsigned long long>(fnv1a(k.source) & 0xffffffffffffULL));
     // give each specialisation a unique, recognisable symbol
@@ -233,6 +248,7 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
     if (gr->g.nodes[id].kind == ASTITCH_LENGTHS && id != gr->g.lengths_node)
       return fail(ASTITCH_ERR_INVALID_GRAPH, "LENGTHS input not bound by astitch_graph_set_mask");
   try {
+    const auto t_start = std::chrono::steady_clock::now();
     auto plan = std::make_unique<Plan>();
     Plan& p = *plan;
     p.g = gr->g;
@@ -260,6 +276,7 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
     select_mapping(p);
     plan_workspace(p);
     p.compulsory_bytes = compulsory_bytes(p);
+    p.ms_analyse = ms_since(t_start);
 
     std::vector<int> roles = {ROLE_MAIN};
     p.kernels.resize(1);
@@ -305,6 +322,7 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
       for (auto& k : p.shard_kernels)
         if ((s = load(k)) != ASTITCH_OK) return s;
     }
+    p.ms_total = ms_since(t_start);
     p.describe = describe_json(p);
     auto* h = new astitch_plan_s();
     h->p = std::move(plan);
@@ -316,6 +334,11 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
   } catch (const std::exception& e) {
     return fail(ASTITCH_ERR_INTERNAL, e.what());
   }
+}
+
+astitch_status astitch_set_cache_dir(const char* dir) {
+  set_cache_dir(dir);
+  return ASTITCH_OK;
 }
 
 astitch_status astitch_plan_destroy(astitch_plan_t h) {

@@ -110,8 +110,14 @@ class ShardedPlan:
     astitch_run_sharded)."""
 
     def __init__(self, graph: Graph, rows: int, cols: int, world: int, rank: int, device: int,
-                 comm: Comm | None = None, flags: int = 0, sm_count: int = 0, tune=None):
-        self.row_begin, self.row_count = shard_rows(rows, world, rank)
+                 comm: Comm | None = None, flags: int = 0, sm_count: int = 0, tune=None, row_range=None):
+        """row_range: (row_begin, row_count) of this rank when the rows are not
+        split evenly (e.g. masked batches balanced by bytes, `mask_row_ranges`);
+        default: astitch_shard_rows' contiguous even split."""
+        if row_range is None:
+            self.row_begin, self.row_count = shard_rows(rows, world, rank)
+        else:
+            self.row_begin, self.row_count = int(row_range[0]), int(row_range[1])
         self.plan = Plan(graph, self.row_count, cols, device=device, flags=flags, shard_rank=rank,
                          shard_world=world, sm_count=sm_count, tune=tune)
         self.comm = comm
@@ -122,12 +128,7 @@ class ShardedPlan:
         return self.world > 1 and self.plan.describe()["shard_kernels"] > 0
 
     def _ws(self, ws, stream):
-        p = self.plan
-        if ws is None and p.workspace_bytes() > 0:
-            if p._ws_cache is None:
-                p._ws_cache = p.alloc_workspace(stream)
-            ws = p._ws_cache
-        return ws
+        return self.plan._stream_ws(stream) if ws is None else ws
 
     def run(self, inputs, outputs, ws=None, stream=None) -> None:
         p = self.plan
@@ -167,19 +168,55 @@ class ShardedPlan:
 
 def partition_by_weight(weights, world: int):
     """Contiguous partition of units (e.g. C3's 64 batches, weighted by their
-    bytes) into `world` ranges with balanced total weight.  Pure host logic."""
-    n = len(weights)
-    total = float(sum(weights))
-    bounds, acc, k = [0], 0.0, 1
-    for i, w in enumerate(weights):
-        acc += w
-        while k < world and acc >= total * k / world and len(bounds) < world:
-            bounds.append(i + 1)
-            k += 1
+    bytes) into `world` ranges minimising the largest range weight (the
+    slowest rank): binary search on that bound, each probe a greedy left-to-
+    right fill.  Pure host logic; returns [(begin, end)] per rank."""
+    w = [float(x) for x in weights]
+    n = len(w)
+    if n == 0:
+        return [(0, 0)] * world
+
+    def fill(cap):
+        bounds, acc = [0], 0.0
+        for i, x in enumerate(w):
+            if acc + x > cap and acc > 0:
+                bounds.append(i)
+                acc = 0.0
+            acc += x
+        return bounds
+
+    lo, hi = max(w), sum(w)
+    for _ in range(100):
+        mid = (lo + hi) / 2
+        if len(fill(mid)) <= world:
+            hi = mid
+        else:
+            lo = mid
+    bounds = fill(hi)
     while len(bounds) < world:
         bounds.append(n)
     bounds.append(n)
     return [(bounds[r], bounds[r + 1]) for r in range(world)]
 
 
-__all__ = ["Comm", "PeerExchange", "ShardedPlan", "partition_by_weight", "_lib"]
+def mask_row_ranges(lengths, rows_per_segment: int, cols: int, rows: int, world: int,
+                    in_bytes: int = 2, out_bytes: int = 2):
+    """Row shards of a key-padding-masked problem: whole
+    mask segments (batches) per rank, contiguous, balanced by each segment's
+    compulsory bytes rows_per_segment x (in_bytes x L_b + out_bytes x cols)
+    (valid-prefix reads + full-row writes).  Returns [(row_begin, row_count)]."""
+    nseg = -(-rows // rows_per_segment)
+    w = []
+    for s_ in range(nseg):
+        nr = min(rows_per_segment, rows - s_ * rows_per_segment)
+        L = min(max(int(lengths[s_]), 0), cols)
+        w.append(nr * (in_bytes * L + out_bytes * cols))
+    out = []
+    for a, b in partition_by_weight(w, world):
+        r0 = a * rows_per_segment
+        r1 = min(rows, b * rows_per_segment)
+        out.append((r0, max(0, r1 - r0)))
+    return out
+
+
+__all__ = ["Comm", "PeerExchange", "ShardedPlan", "partition_by_weight", "mask_row_ranges", "_lib"]

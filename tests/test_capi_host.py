@@ -2,6 +2,7 @@
 symbol include/astitch.h declares, and returns the documented status codes."""
 
 import ctypes as ct
+import json
 import os
 import re
 
@@ -209,3 +210,32 @@ def test_library_reads_no_planning_environment_variables():
     src = os.path.join(ROOT, "paper_conf_asplos_zhengyzlzzzlyzs22_b200", "csrc")
     for f in ("planner.cpp", "codegen.cpp", "runtime.cpp", "graph.cpp"):
         assert "getenv" not in open(os.path.join(src, f)).read(), f
+
+
+def test_disk_cubin_cache_and_plan_time(tmp_path):
+    """The on-disk cubin cache: a fresh process-level miss compiles with NVRTC
+    and stores the cubin; a plan of the same source in a NEW process loads it
+    from disk (no NVRTC); describe() reports the plan (JIT) time split."""
+    import subprocess
+    import sys
+    code = ("import sys, json; sys.path.insert(0, %r)\n"
+            "import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A\n"
+            "from workloads import specs\n"
+            "A.set_cache_dir(%r)\n"
+            "s = specs.get('C4', rows=5000)\n"
+            "d = A.Plan(A.Graph.from_spec(s), 5000, 36, device=-1).describe()\n"
+            "print(json.dumps(d['plan_time_ms']))\n") % (ROOT, str(tmp_path))
+    runs = [json.loads(subprocess.run([sys.executable, "-c", code], capture_output=True, text=True,
+                                      check=True).stdout.strip().splitlines()[-1]) for _ in range(2)]
+    assert runs[0]["nvrtc_compiles"] >= 1 and runs[0]["cache_hits_disk"] == 0
+    assert runs[1]["nvrtc_compiles"] == 0 and runs[1]["cache_hits_disk"] >= 1
+    assert any(f.suffix == ".cubin" for f in tmp_path.iterdir())
+    for k in ("analyse_map", "codegen", "nvrtc", "load", "total"):
+        assert runs[0][k] >= 0
+    assert runs[1]["nvrtc"] < runs[0]["nvrtc"]
+    # a corrupted cache file is ignored (recompiled), never trusted
+    for f in tmp_path.iterdir():
+        f.write_bytes(b"garbage")
+    r3 = json.loads(subprocess.run([sys.executable, "-c", code], capture_output=True, text=True,
+                                   check=True).stdout.strip().splitlines()[-1])
+    assert r3["nvrtc_compiles"] >= 1

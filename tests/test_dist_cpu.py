@@ -122,3 +122,26 @@ def test_sharded_plans_describe_same_mapping(world):
         m = p.describe()["mapping"]
         maps.append((m["template"], m["team"], m["chunks_per_lane"], m["vec_elems"]))
     assert len(set(maps)) == 1
+
+
+def test_mask_row_ranges_balance_c3_bytes():
+    """C3 at N>1 shards whole batches balanced by compulsory bytes (SURVEY
+    8(e)), not equal rows: contiguous, segment-aligned, covering all rows, and
+    better balanced than the even row split."""
+    from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import mask_row_ranges
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from workloads import gen, specs
+    spec = specs.get("C3")
+    L = gen.lengths_for(spec, gen.CONFIG_SEEDS["C3"])
+    R, C, rps = spec["rows"], spec["cols"], spec["mask"]["rows_per_segment"]
+
+    def load(r0, n):
+        return sum(min(rps, R - s * rps) * (2 * int(L[s]) + 2 * C) for s in range(r0 // rps, -(-(r0 + n) // rps)))
+    for world in (2, 4, 8):
+        rr = mask_row_ranges(L, rps, C, R, world)
+        assert rr[0][0] == 0 and sum(n for _, n in rr) == R
+        assert all(a[0] + a[1] == b[0] for a, b in zip(rr, rr[1:]))
+        assert all(r0 % rps == 0 for r0, _ in rr)
+        bal = max(load(*x) for x in rr)
+        even = max(load(*A.shard_rows(R, world, r)) for r in range(world))
+        assert bal <= even
