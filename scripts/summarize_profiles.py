@@ -136,8 +136,10 @@ def main():
         for k, v in by.most_common():
             lines.append(f"* `{k}`: {100.0 * v / tot:.1f}%")
     lines += ["", "## ncu --set full digests (one launch each)", ""]
-    for rep in sorted(glob.glob(os.path.join(OUT, "prof_C*.ncu-rep"))):
-        c = os.path.basename(rep)[5:].split(".")[0]
+    reps = sorted(glob.glob(os.path.join(OUT, f"prof_{rnd}_C*.ncu-rep"))) or \
+        sorted(glob.glob(os.path.join(OUT, "prof_C*.ncu-rep")))
+    for rep in reps:
+        c = os.path.basename(rep).split(".")[0].split("_")[-1]
         d = full_digest(rep)
         if d is None:
             continue
