@@ -678,6 +678,17 @@ void select_mapping(Plan& p) {
       }
       m.rows_per_block = m.threads / m.team;
       m.row_unroll = (tu.unroll >= 1 && tu.unroll <= 8) ? tu.unroll : 1;
+      // Light rows (<= 16 values per lane over all input streams, no mask):
+      // a non-persistent grid, one row group per CTA, so the hardware block
+      // scheduler streams the CTAs through the rows in address order and the
+      // low register count keeps many warps per SM.  Measured on B200
+      // (scripts/sweeps/r02_readmostly.txt): row sums [4M, 32] fp32 87.6 ->
+      // 75.1 us, [1M, 256] 153 -> 144 us; softmax fp32 [1M, 128] 184 -> 157 us.
+      // Heavier rows keep the persistent prefetching sweep (LayerNorm+GELU
+      // [65536, 768] 52.9 vs 54.7 us, masked softmax C3 145 vs 165 us).
+      m.nonpersistent = !has_mask && !ragged && m.single_wave_bps == 0 &&
+                        nfull_in * m.chunks_per_lane * E <= 16;
+      if (tu.persistent >= 0) m.nonpersistent = tu.persistent == 0;
       why << (m.single_wave_bps ? "one wave of teams (one row per team); " : "") << "row team of " << m.team << " lanes x " << m.chunks_per_lane << " chunks ("
           << m.rows_per_block << " rows / block, packing), regional via shuffles" << (m.team > 32 ? "+smem" : "")
           << "; ";
@@ -811,6 +822,11 @@ void retune_grid(Plan& p) {
     const int64_t groups = std::max<int64_t>(1, std::min(work_units, wave / m.nslab));
     m.grid = groups * m.nslab;
     m.vertical_trips = (work_units + groups - 1) / groups;
+  } else if (m.tmpl == Template::RowTeam && m.nonpersistent) {
+    // one row group per CTA: the hardware block scheduler streams the CTAs
+    // through the rows in address order (no software prefetch needed)
+    m.grid = std::max<int64_t>(1, work_units);
+    m.vertical_trips = 1;
   } else {
     m.grid = std::max<int64_t>(1, std::min(work_units, wave));
     m.vertical_trips = (work_units + m.grid - 1) / m.grid;
@@ -967,7 +983,7 @@ std::string describe_json(const Plan& p) {
     << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
     << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads
     << ",\"rows_per_block\":" << m.rows_per_block << ",\"row_unroll\":" << m.row_unroll
-    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"sync_steps\":" << (m.sync_steps ? "true" : "false") << ",\"nslab\":" << m.nslab
+    << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"sync_steps\":" << (m.sync_steps ? "true" : "false") << ",\"nslab\":" << m.nslab << ",\"nonpersistent\":" << (m.nonpersistent ? "true" : "false")
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
     << ",\"grid\":" << m.grid

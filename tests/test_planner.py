@@ -107,7 +107,11 @@ def test_fig6_selector_branches():
     d, _, _ = describe("fig6a")              # <750000,32>: pack many rows per block
     m = d["mapping"]
     assert m["team"] < 32 and m["rows_per_block"] > 32
-    assert m["grid"] <= m["blocks_per_sm"] * 148
+    # light rows: one row group per CTA on a non-persistent grid (the block
+    # scheduler orders the sweep); heavier rows: a persistent one-wave grid
+    assert m["nonpersistent"] and m["grid"] * m["rows_per_block"] >= 750_000 and m["vertical_trips"] == 1
+    d, _, _ = describe("C3")
+    assert not d["mapping"]["nonpersistent"] and d["mapping"]["grid"] <= d["mapping"]["blocks_per_sm"] * 148
     # <64,30000>: the paper's shape rule holds, but 120 KB rows are below the
     # measured B200 threshold (reading R15) -> one block team per row
     d, _, _ = describe("fig6b")
