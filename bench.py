@@ -719,7 +719,7 @@ def main():
             "e2e": None if e2e_gbs is None else {"value": round(e2e_gbs, 3), "unit": "GB/s", "h2d_bytes_per_step": int(h2d),
                     "d2h_bytes_per_step": int(d2h), "ms_per_step": round(e2e_ms, 3),
                     "api": "astitch_run_host_pipelined" if (world == 1 and args.e2e_chunks > 1) else
-                           ("astitch_run_host" if world == 1 else "torch H2D/D2H + astitch_run_sharded"),
+                           ("astitch_run_host" if world == 1 else "astitch_run_sharded_host"),
                     "chunks": args.e2e_chunks if world == 1 else 1, "pcie": link},
             "gpu_launches": int(args.steps * sp.kernels_per_run()),
             "clocks": clocks,
@@ -763,12 +763,9 @@ def check_fused_exchange(sp, inputs, plan, ws, exchange):
 
 
 def _sharded_host(sp, host_in, host_out, dev_in, dev_out, ws):
-    """Sharded e2e step: H2D of this rank's inputs, astitch_run_sharded, D2H."""
-    for h, d in zip(host_in, dev_in):
-        d.copy_(h, non_blocking=True)
-    sp.run(dev_in, dev_out, ws=ws)
-    for h, d in zip(host_out, dev_out):
-        h.copy_(d, non_blocking=True)
+    """Sharded e2e step through the C ABI (astitch_run_sharded_host): H2D of
+    this rank's inputs, the fused / NCCL sharded run, D2H of its outputs."""
+    sp.run_host(host_in, host_out, dev_in, dev_out, ws=ws)
 
 
 if __name__ == "__main__":

@@ -334,6 +334,14 @@ astitch_status astitch_peer_status(astitch_peer_t x, int32_t* timed_out);
 astitch_status astitch_peer_destroy(astitch_peer_t x);
 astitch_status astitch_run_fused(astitch_plan_t p, astitch_peer_t x, const void* const* inputs,
                                  void* const* outputs, void* ws, void* stream);
+/* End-to-end sharded run from HOST buffers (the rank's row slice): async H2D
+ * of every input into dev_inputs, then astitch_run_fused (x != NULL) or
+ * astitch_run_sharded (comm c), then async D2H of every output, all on
+ * `stream`.  Same errors as those calls. */
+astitch_status astitch_run_sharded_host(astitch_plan_t p, astitch_comm_t c, astitch_peer_t x,
+                                        const void* const* host_inputs, void* const* host_outputs,
+                                        const void* const* dev_inputs, void* const* dev_outputs, void* ws,
+                                        void* stream);
 /* Contiguous row partition: rows_k = floor(R/g) (+1 for the first R mod g ranks). */
 astitch_status astitch_shard_rows(int64_t rows, int32_t world, int32_t rank, int64_t* row_begin,
                                   int64_t* row_count);

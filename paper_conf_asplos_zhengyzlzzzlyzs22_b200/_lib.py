@@ -91,6 +91,8 @@ _sig = {
     "astitch_plan_io": (ct.c_int, [_vp, ct.c_int32, ct.c_int32, ct.POINTER(ct.c_int), ct.POINTER(ct.c_int)]),
     "astitch_workspace_init": (ct.c_int, [_vp, _vp, _vp]),
     "astitch_run": (ct.c_int, [_vp, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
+    "astitch_run_sharded_host": (ct.c_int, [_vp, _vp, _vp, ct.POINTER(_vp), ct.POINTER(_vp), ct.POINTER(_vp),
+                                             ct.POINTER(_vp), _vp, _vp]),
     "astitch_run_host": (ct.c_int, [_vp, ct.POINTER(_vp), ct.POINTER(_vp), ct.POINTER(_vp),
                                     ct.POINTER(_vp), _vp, _vp]),
     "astitch_run_host_pipelined": (ct.c_int, [_vp, ct.POINTER(_vp), ct.POINTER(_vp), ct.POINTER(_vp),

@@ -502,8 +502,14 @@ astitch_status astitch_run(astitch_plan_t h, const void* const* inputs, void* co
   return ASTITCH_OK;
 }
 
-astitch_status astitch_run_host(astitch_plan_t h, const void* const* host_inputs, void* const* host_outputs,
-                                const void* const* dev_inputs, void* const* dev_outputs, void* ws, void* stream) {
+}  // extern "C"
+
+namespace astitch {
+// H2D of every input, `run` (the stitched kernel(s) on the device buffers),
+// D2H of every output, all asynchronous on `stream`
+template <typename F>
+astitch_status run_with_host_copies(astitch_plan_t h, const void* const* host_inputs, void* const* host_outputs,
+                                    const void* const* dev_inputs, void* const* dev_outputs, void* stream, F run) {
   if (!h || !host_inputs || !host_outputs || !dev_inputs || !dev_outputs)
     return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
   const Plan& p = *h->p;
@@ -516,7 +522,7 @@ astitch_status astitch_run_host(astitch_plan_t h, const void* const* host_inputs
     if (!drv_memcpy_async(const_cast<void*>(dev_inputs[i]), host_inputs[i], nbytes, 1, stream, err))
       return fail(ASTITCH_ERR_CUDA, err);
   }
-  astitch_status s = astitch_run(h, dev_inputs, dev_outputs, ws, stream);
+  astitch_status s = run();
   if (s != ASTITCH_OK) return s;
   for (size_t i = 0; i < p.g.outputs.size(); ++i) {
     size_t nbytes = io_bytes(p, p.g.outputs[i], p.g.output_dtypes[i]);
@@ -525,6 +531,25 @@ astitch_status astitch_run_host(astitch_plan_t h, const void* const* host_inputs
       return fail(ASTITCH_ERR_CUDA, err);
   }
   return ASTITCH_OK;
+}
+}  // namespace astitch
+
+extern "C" {
+
+astitch_status astitch_run_sharded_host(astitch_plan_t h, astitch_comm_t c, astitch_peer_t x,
+                                        const void* const* host_inputs, void* const* host_outputs,
+                                        const void* const* dev_inputs, void* const* dev_outputs, void* ws,
+                                        void* stream) {
+  return run_with_host_copies(h, host_inputs, host_outputs, dev_inputs, dev_outputs, stream, [&]() {
+    return x ? astitch_run_fused(h, x, dev_inputs, dev_outputs, ws, stream)
+             : astitch_run_sharded(h, c, dev_inputs, dev_outputs, ws, stream);
+  });
+}
+
+astitch_status astitch_run_host(astitch_plan_t h, const void* const* host_inputs, void* const* host_outputs,
+                                const void* const* dev_inputs, void* const* dev_outputs, void* ws, void* stream) {
+  return run_with_host_copies(h, host_inputs, host_outputs, dev_inputs, dev_outputs, stream,
+                              [&]() { return astitch_run(h, dev_inputs, dev_outputs, ws, stream); });
 }
 
 astitch_status astitch_run_host_pipelined(astitch_plan_t h, const void* const* host_inputs,

@@ -144,6 +144,20 @@ class ShardedPlan:
         check(lib.astitch_run_sharded(p.handle, self.comm.handle if self.comm else None, ins, outs, w, s),
               "astitch_run_sharded")
 
+    def run_host(self, host_inputs, host_outputs, dev_inputs, dev_outputs, ws=None, stream=None) -> None:
+        """astitch_run_sharded_host: H2D of this rank's inputs, the sharded
+        (fused or NCCL) run, D2H of its outputs, asynchronous on `stream`."""
+        p = self.plan
+        p.check_io(host_inputs, host_outputs, device=False)
+        p.check_io(dev_inputs, dev_outputs)
+        ws = self._ws(ws, stream)
+        arr = lambda ts: ptr_array([t.data_ptr() for t in ts])  # noqa: E731
+        check(lib.astitch_run_sharded_host(p.handle, self.comm.handle if self.comm else None,
+                                           self.peer.handle if self.peer is not None else None,
+                                           arr(host_inputs), arr(host_outputs), arr(dev_inputs), arr(dev_outputs),
+                                           ct.c_void_p(ws.data_ptr() if ws is not None else 0),
+                                           ct.c_void_p(_stream_ptr(stream))), "astitch_run_sharded_host")
+
     def run_stage(self, stage: int, inputs, outputs, ws, stream=None) -> None:
         """astitch_run_shard_stage: 0 = stitched kernel leaving rank-local column
         totals in ws; 1 = column consumers reading the combined totals."""

@@ -284,9 +284,10 @@ def test_full_c5_sampled():
     refc = evaluate_columns(spec, x, cols)
     check_close(got["db"][cols], refc["db"], "F32", 2e-3, "C5 db")
     check_close(got["b_new"][cols], refc["b_new"], "F32", 2e-3, "C5 b_new")
-    # fp32-quality report for db (reading R4): informational bound 1e-5 relative to RMS
+    # fp32-quality check for db (reading R4): 1e-5 relative to the RMS
+    # (measured 9.7e-7 at full size, profiles/r02_parity_report.json)
     s = np.sqrt(np.mean(refc["db"] ** 2))
-    assert np.max(np.abs(got["db"][cols] - refc["db"])) <= 1e-4 * s
+    assert np.max(np.abs(got["db"][cols] - refc["db"])) <= 1e-5 * s
     rows = np.unique(rng.integers(0, spec["rows"], 3000))
     sub = dict(spec, outputs=[("dz", "BF16")], ops=[o for o in spec["ops"] if o[0] in ("g", "dz")])
     refr = evaluate_rows(sub, x, rows)
@@ -745,3 +746,35 @@ def test_wide_bias_grad_4096x131072_sampled():
     b = x["b"].astype(np.float32)
     exp = (b - np.float32(0.0078125) * got["db"].astype(np.float32)).astype(np.float32)
     np.testing.assert_array_equal(got["b_new"].astype(np.float32), exp)
+
+
+def test_sharded_host_entry_point_virtual_ranks():
+    """astitch_run_sharded_host (the N>1 end-to-end C-ABI call): pinned host
+    inputs -> device -> fused sharded kernel -> pinned host outputs, per
+    virtual rank, bitwise equal to the device-buffer run."""
+    import torch
+    from tests.harness import from_torch
+    spec = specs.get("C5", rows=4099, cols=256)
+    x = gen.generate("C5", spec)
+    ranks = _virtual_ranks(spec, x, 2)
+    torch.cuda.synchronize()
+    for sp, ins, outs, ws, st in ranks:
+        sp.run(ins, outs, ws=ws, stream=st)
+    torch.cuda.synchronize()
+    dev = [[from_torch(o).copy() for o in rk[2]] for rk in ranks]
+    hosts = []
+    for sp, ins, outs, ws, st in ranks:
+        hin = [t.cpu().pin_memory() for t in ins]
+        hout = [torch.empty(o.shape, dtype=o.dtype).pin_memory() for o in outs]
+        for o in outs:
+            o.zero_()
+        hosts.append((hin, hout))
+    torch.cuda.synchronize()
+    for (sp, ins, outs, ws, st), (hin, hout) in zip(ranks, hosts):
+        sp.run_host(hin, hout, ins, outs, ws=ws, stream=st)
+    torch.cuda.synchronize()
+    for sp, *_ in ranks:
+        assert not sp.peer.timed_out()
+    for r, (hin, hout) in enumerate(hosts):
+        for a, b in zip(dev[r], hout):
+            assert np.array_equal(a, from_torch(b)), r
