@@ -979,6 +979,37 @@ std::string describe_json(const Plan& p) {
     for (size_t j = 0; j < p.groups[k].size(); ++j) o << (j ? "," : "") << p.groups[k][j];
     o << "]";
   }
+  // Step 2: each group's schedule = its dominant's.  Every group of
+  // one stitched kernel shares the block and the lane -> (row, columns)
+  // assignment of the template (the team shape is a function of C and the
+  // dtypes only); groups differ in the index space their dominant iterates:
+  o << "],\"group_mappings\":[";
+  for (size_t k = 0; k < p.groups.size(); ++k) {
+    int dom = -1;
+    bool any_full = false, any_row = false, any_col = false;
+    for (int i : p.groups[k]) {
+      if (p.info[i].dominant) dom = i;
+      any_full |= g.nodes[i].kind == ASTITCH_FULL;
+      any_row |= g.nodes[i].kind == ASTITCH_ROWVEC;
+      any_col |= g.nodes[i].kind == ASTITCH_COLVEC;
+    }
+    std::string how;
+    const OpClass dc = dom >= 0 ? p.info[dom].cls : OpClass::LightEW;
+    if (dc == OpClass::ReduceCol)
+      how = "column reduce: each lane accumulates its columns over its rows (vertical packing), block + grid "
+            "partials, then one thread per column after the grid barrier";
+    else if (dc == OpClass::ReduceRow)
+      how = "row reduce: a team of T lanes per row (elements (j*T+lane)*E..), shuffle / smem / DSMEM tree, "
+            "row scalar team-uniform";
+    else if (!any_full && any_col)
+      how = "column values: one thread per column (finalise after the barrier) or per lane chunk (hoisted)";
+    else if (!any_full && any_row)
+      how = "row values: team-uniform scalars";
+    else
+      how = "element-wise only: adopts its producer group's mapping (proactive block locality, P:L282)";
+    o << (k ? "," : "") << "{\"group\":" << k << ",\"dominant\":" << dom << ",\"level\":"
+      << (dom >= 0 ? p.info[dom].level : 0) << ",\"schedule\":\"" << how << "\"}";
+  }
   o << "],\"mapping\":{\"template\":\"" << template_name(m.tmpl) << "\",\"vec_elems\":" << m.vec_elems
     << ",\"chunks\":" << m.chunks << ",\"team\":" << m.team << ",\"chunks_per_lane\":" << m.chunks_per_lane
     << ",\"lane_util\":" << m.lane_util << ",\"threads\":" << m.threads

@@ -316,3 +316,17 @@ def test_global_sweep_block_combine_fits_smem():
         m = d["mapping"]
         assert m["smem_bytes"] <= 96 * 1024, (name, cols, m)
         assert m["rows_per_block"] == 1 or m["smem_bytes"] > 0
+
+
+def test_group_mappings_follow_their_dominants():
+    """Step 2: every group's schedule is its dominant's; Fig. 7(a)
+    has a row-reduce group (level 0) and a column-reduce group (level 1);
+    an element-wise-only group adopts its producer's mapping."""
+    d, _, _ = describe("fig7a")
+    gm = d["group_mappings"]
+    kinds = sorted((x["level"], x["schedule"].split(":")[0]) for x in gm)
+    assert kinds == [(0, "row reduce"), (1, "column reduce")]
+    ew = {"name": "ew", "rows": 100, "cols": 64, "inputs": [("x", "FULL", "F32")], "mask": None,
+          "ops": [("e", "unary", "EXP", "x"), ("n", "unary", "NEG", "e")], "outputs": [("n", "F32")]}
+    p = A.Plan(A.Graph.from_spec(ew), 100, 64, device=-1, flags=A.FLAG_NO_COMPILE)
+    assert all("element-wise only" in x["schedule"] or "dominant" in x for x in p.describe()["group_mappings"])
