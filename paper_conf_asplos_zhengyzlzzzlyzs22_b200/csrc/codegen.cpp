@@ -304,12 +304,23 @@ struct Gen {
     return false;
   }
 
+  // FULL bf16 / f16 input streams whose raw 32-bit words (two elements) are
+  // kept next to their fp32 unpack: an ADD of such an element and an fp32
+  // value is ONE sm_100a mixed-precision add (add.rn.f32.bf16 -> FHADD.BF16,
+  // exact widening + one fp32 rounding: bitwise the same as unpack + FADD)
+  // and the unpack of that element disappears when nothing else reads it.
+  // Unmasked rows only (an absorbed mask rewrites invalid elements).
+  std::vector<bool> rawok;
   void collect_streams(bool /*post*/) {
     streams.clear();
+    rawok.assign(g.nodes.size(), false);
     for (int id : g.inputs) {
       const Node& nd = N(id);
-      if (nd.kind == ASTITCH_FULL && I(id).live && node_used_in_phase(id, false))
+      if (nd.kind == ASTITCH_FULL && I(id).live && node_used_in_phase(id, false)) {
         streams.push_back({id, false, nd.dtype, 0});  // re-read from HBM in later sweeps
+        rawok[id] = !masked && (E % 2) == 0 && (nd.dtype == ASTITCH_BF16 || nd.dtype == ASTITCH_F16) &&
+                    m.tmpl != Template::RowStream;
+      }
     }
     for (size_t q = 0; q < p.global_fulls.size(); ++q) {
       int id = p.global_fulls[q];
@@ -372,6 +383,11 @@ struct Gen {
       o << "    float " << dst << "[NE];\n";
       o << "#pragma unroll\n    for (int j = 0; j < V; ++j) as::Conv<" << dt << ", E>::unpack(r" << s << src
         << "[j], " << dst << " + j * E);\n";
+      if (rawok.size() > static_cast<size_t>(id) && rawok[id]) {
+        o << "    unsigned int w" << id << sfx << "[NE / 2];\n";
+        o << "#pragma unroll\n    for (int j = 0; j < V; ++j)\n#pragma unroll\n    for (int q = 0; q < E / 2; ++q) w" << id << sfx
+          << "[j * (E / 2) + q] = as::word(r" << s << src << "[j], q);\n";
+      }
     }
   }
   void emit_unpack_mask(const std::string& sfx, const std::string& lim) {
@@ -752,9 +768,10 @@ struct Gen {
         if (nd.b >= 0 && N(nd.b).kind == ASTITCH_ROWVEC) need[nd.b] = true;
       }
     }
-    // global-buffered / post values keep the plain fp32 path
+    // row values read after a grid barrier (FORCE_GLOBAL) stay precise: the
+    // ROWVEC buffer carries the lo part next to the value (R floats later)
     for (int i = 0; i < n; ++i)
-      if (I(i).post || I(i).global_full) precise[i] = false;
+      if ((I(i).post || I(i).global_full) && N(i).kind != ASTITCH_ROWVEC) precise[i] = false;
   }
   void emit_split(const std::string& id, const std::string& sfx) {
     o << "    const float s" << id << sfx << " = (float)d" << id << sfx << ";\n";
@@ -865,6 +882,15 @@ struct Gen {
     }
     if (nd.type == NodeType::Unary) return unop2(nd.sub, ref2(nd.a, sfx));
     if (row_div(i)) return "as::mul2(" + ref2(nd.a, sfx) + ", as::bc2(rq" + std::to_string(i) + sfx + "))";
+    if (nd.type == NodeType::Binary && nd.sub == ASTITCH_ADD && !precise_bcast(nd.a) && !precise_bcast(nd.b) &&
+        !precise_bcast_col(nd.a) && !precise_bcast_col(nd.b)) {
+      const std::string hf = N(nd.a).dtype == ASTITCH_F16 ? "f16" : "bf16";
+      if (raw_operand(nd.a))
+        return "as::hadd2_" + hf + "(w" + std::to_string(nd.a) + sfx + "[k / 2], " + ref2(nd.b, sfx) + ")";
+      if (raw_operand(nd.b))
+        return "as::hadd2_" + std::string(N(nd.b).dtype == ASTITCH_F16 ? "f16" : "bf16") + "(w" + std::to_string(nd.b) +
+               sfx + "[k / 2], " + ref2(nd.a, sfx) + ")";
+    }
     std::string a = ref2(nd.a, sfx), b = ref2(nd.b, sfx);
     auto lo = [&](int v) { return "as::bc2(s" + std::to_string(N(v).a) + sfx + "lo)"; };
     auto clo = [&](int v) { return "as::f2{" + col_lo(v, "k") + ", " + col_lo(v, "k + 1") + "}"; };
@@ -879,6 +905,10 @@ struct Gen {
     return binop2(nd.sub, nd.b, a, b);
   }
 
+  bool raw_operand(int v) const {
+    return v >= 0 && static_cast<size_t>(v) < rawok.size() && rawok[v] && N(v).type == NodeType::Input &&
+           N(v).kind == ASTITCH_FULL;
+  }
   // Per-element expression of a FULL op.  Peephole (local stitching lets the
   // whole chain sit in registers, so it can be re-associated once):
   //   exp((k*x) - s)  ->  ex2(fma(x, k*log2e, -s*log2e))   (s: row scalar / const)
@@ -981,6 +1011,11 @@ struct Gen {
         if (N(id).kind != ASTITCH_ROWVEC || I(id).level >= cur_level || !node_used_in_phase(id, true)) continue;
         o << "    const float s" << id << sfx << " = (" << act << ") ? as::ld_cg((const float*)((const char*)p.ws + "
           << (p.ws.globals + gbuf_offset(q)) << "LL) + " << row << ") : 0.f;\n";
+        if (precise[id]) {  // R7b across the barrier: hi + lo
+          o << "    const float s" << id << sfx << "lo = (" << act << ") ? as::ld_cg((const float*)((const char*)p.ws + "
+            << (p.ws.globals + gbuf_offset(q)) << "LL) + " << p.desc.rows << "LL + " << row << ") : 0.f;\n";
+          o << "    const double d" << id << sfx << " = (double)s" << id << sfx << " + (double)s" << id << sfx << "lo;\n";
+        }
       }
     }
   }
@@ -1051,6 +1086,9 @@ struct Gen {
         } else if (N(id).kind == ASTITCH_ROWVEC) {
           o << "    if ((" << act << ") && lane == 0) ((float*)((char*)p.ws + " << off << "LL))[" << row << "] = s"
             << id << sfx << ";\n";
+          if (precise[id])
+            o << "    if ((" << act << ") && lane == 0) ((float*)((char*)p.ws + " << off << "LL))[" << p.desc.rows << "LL + "
+              << row << "] = s" << id << sfx << "lo;\n";
         }
       }
     }

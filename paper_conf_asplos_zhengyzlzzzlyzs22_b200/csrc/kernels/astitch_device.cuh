@@ -31,6 +31,13 @@ template <> struct Raw<4> { u32 x; };
 template <> struct Raw<8> { u32 x, y; };
 template <> struct Raw<16> { u32 x, y, z, w; };
 template <> struct Raw<32> { u32 x, y, z, w, a, b, c, d; };
+// 32-bit word q of a raw vector (q a compile-time constant after unrolling)
+__device__ __forceinline__ u32 word(const Raw<4>& r, int) { return r.x; }
+__device__ __forceinline__ u32 word(const Raw<8>& r, int q) { return q == 0 ? r.x : r.y; }
+__device__ __forceinline__ u32 word(const Raw<16>& r, int q) { return q == 0 ? r.x : q == 1 ? r.y : q == 2 ? r.z : r.w; }
+__device__ __forceinline__ u32 word(const Raw<32>& r, int q) {
+  return q == 0 ? r.x : q == 1 ? r.y : q == 2 ? r.z : q == 3 ? r.w : q == 4 ? r.a : q == 5 ? r.b : q == 6 ? r.c : r.d;
+}
 
 // streaming (read-once) global loads: no L1 allocation
 __device__ __forceinline__ Raw<2> ldg(const Raw<2>* p) {
@@ -327,6 +334,20 @@ __device__ __forceinline__ f2 fma2(f2 a, f2 b, f2 c) {
   u64 r; asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(pk2(a)), "l"(pk2(b)), "l"(pk2(c))); return upk2(r);
 }
 __device__ __forceinline__ f2 abs2(f2 a) { return f2{fabsf(a.x), fabsf(a.y)}; }
+// sm_100a mixed-precision adds: fp32 <- (bf16 | f16 element of a packed word) + fp32,
+// the 16-bit operand widened exactly inside the FHADD (no separate unpack)
+__device__ __forceinline__ f2 hadd2_bf16(u32 w, f2 c) {
+  f2 r;
+  asm("{ .reg .b16 lo, hi; mov.b32 {lo, hi}, %2;\n add.rn.f32.bf16 %0, lo, %3;\n add.rn.f32.bf16 %1, hi, %4; }"
+      : "=f"(r.x), "=f"(r.y) : "r"(w), "f"(c.x), "f"(c.y));
+  return r;
+}
+__device__ __forceinline__ f2 hadd2_f16(u32 w, f2 c) {
+  f2 r;
+  asm("{ .reg .b16 lo, hi; mov.b32 {lo, hi}, %2;\n add.rn.f32.f16 %0, lo, %3;\n add.rn.f32.f16 %1, hi, %4; }"
+      : "=f"(r.x), "=f"(r.y) : "r"(w), "f"(c.x), "f"(c.y));
+  return r;
+}
 __device__ __forceinline__ f2 neg2(f2 a) { return f2{-a.x, -a.y}; }
 __device__ __forceinline__ f2 max2(f2 a, f2 b) { return f2{nmax(a.x, b.x), nmax(a.y, b.y)}; }
 __device__ __forceinline__ f2 min2(f2 a, f2 b) { return f2{nmin(a.x, b.x), nmin(a.y, b.y)}; }

@@ -895,7 +895,9 @@ void plan_workspace(Plan& p) {
         if (slots[s].kind == k && slots[s].free_after < def) { chosen = static_cast<int>(s); break; }
       if (chosen < 0) {
         slots.push_back({k, -1, goff});
-        goff = align(goff + static_cast<size_t>(R) * (k == ASTITCH_FULL ? C : 1) * 4);
+        // ROWVEC buffers hold 2 R floats: the value and, for a cancellation-
+        // prone row sum demoted to global (FORCE_GLOBAL), its lo part (R7b)
+        goff = align(goff + static_cast<size_t>(R) * (k == ASTITCH_FULL ? C : 2) * 4);
         chosen = static_cast<int>(slots.size()) - 1;
       }
       slots[chosen].free_after = last_read(id);

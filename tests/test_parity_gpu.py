@@ -778,3 +778,17 @@ def test_sharded_host_entry_point_virtual_ranks():
     for r, (hin, hout) in enumerate(hosts):
         for a, b in zip(dev[r], hout):
             assert np.array_equal(a, from_torch(b)), r
+
+
+@pytest.mark.parametrize("rows,cols,mean", [(7, 62, 1000.0), (8941, 894, -3.0e4), (3000, 36, 1000.0)])
+def test_parity_force_global_mean_far_from_spread(rows, cols, mean):
+    """FORCE_GLOBAL (row reductions demoted to HBM + grid barrier) keeps
+    reading R7b across the barrier: the demoted row sum is buffered as an
+    fp32 hi + lo pair (round-2 fuzz, seeds 328 / 333, found it plain fp32)."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    spec = specs.get("C4", rows=rows, cols=cols)
+    x = gen.generate("C4", spec)
+    x["x"] = (mean + 0.01 * x["x"].astype(np.float64)).astype(np.float32)
+    got, plan = run_gpu(spec, x, return_plan=True, flags=A.FLAG_FORCE_GLOBAL)
+    assert plan.describe()["mapping"]["template"] == "global_sweep"
+    _compare(spec, got, evaluate(spec, x))
