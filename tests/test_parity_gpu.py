@@ -792,3 +792,24 @@ def test_parity_force_global_mean_far_from_spread(rows, cols, mean):
     got, plan = run_gpu(spec, x, return_plan=True, flags=A.FLAG_FORCE_GLOBAL)
     assert plan.describe()["mapping"]["template"] == "global_sweep"
     _compare(spec, got, evaluate(spec, x))
+
+
+RESID_F16 = {
+    "name": "resid_f16", "rows": 3000, "cols": 256,
+    "inputs": [("x", "FULL", "F16"), ("r", "FULL", "BF16"), ("b", "COLVEC", "F32")], "mask": None,
+    "ops": [("bb", "broadcast", "COL", "b"), ("h", "binary", "ADD", "bb", "x"), ("h2", "binary", "ADD", "h", "r"),
+            ("e", "unary", "EXP", "x"), ("h3", "binary", "ADD", "x", "r"), ("s", "reduce", "SUM", "ROW", "h2")],
+    "outputs": [("h2", "F32"), ("h3", "F16"), ("s", "F32"), ("e", "F32")],
+}
+
+
+def test_mixed_precision_adds_fhadd():
+    """Adds of a bf16 / f16 FULL input and an fp32 value use sm_100a's
+    FHADD (add.rn.f32.{bf16,f16}): exact widening + one fp32 rounding, so the
+    results are bitwise those of unpack + FADD; oracle parity for both input
+    widths and both operand positions."""
+    x = gen.generate("fig6a", RESID_F16)
+    got, plan = run_gpu(RESID_F16, x, return_plan=True)
+    src = plan.source(0)
+    assert "hadd2_f16" in src and "hadd2_bf16" in src
+    _compare(RESID_F16, got, evaluate(RESID_F16, x))
