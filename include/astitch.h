@@ -113,10 +113,20 @@ astitch_status astitch_graph_input(astitch_graph_t g, astitch_kind kind, astitch
                                    astitch_value_t* out);
 /* A SCALAR constant (applied in fp32 on the device, fp64 in the oracle). */
 astitch_status astitch_graph_const(astitch_graph_t g, double v, astitch_value_t* out);
+/* Element-wise ops: same kind as the operand(s), applied per
+ * element in fp32 on the device.  MAX / MIN propagate NaN (reading R12).
+ * Integer POW exponents 0..8 are repeated multiplication (R11). */
 astitch_status astitch_graph_unary(astitch_graph_t g, astitch_unop op, astitch_value_t a,
                                    astitch_value_t* out);
 astitch_status astitch_graph_binary(astitch_graph_t g, astitch_binop op, astitch_value_t a,
                                     astitch_value_t b, astitch_value_t* out);
+/* Row (FULL -> ROWVEC) or column (FULL -> COLVEC) reduction.  Sums
+ * accumulate in fp32 with a fixed order (bitwise run-to-run deterministic,
+ * R13); a sum that is broadcast back into an add / sub (a mean) keeps the
+ * spread of its row / column (shifted or fp64 sums applied as hi + lo: R7b,
+ * R7c).  RMAX propagates NaN (R12).  A column reduction ends the pass over
+ * the rows: its consumers run after a grid barrier (global stitching) in the
+ * same kernel. */
 astitch_status astitch_graph_reduce(astitch_graph_t g, astitch_redop op, astitch_axis axis,
                                     astitch_value_t a, astitch_value_t* out);
 astitch_status astitch_graph_broadcast(astitch_graph_t g, astitch_axis axis, astitch_value_t a,
