@@ -105,6 +105,7 @@ struct Mapping {
   int single_wave_bps = 0;  // RowTeam: blocks/SM that give every row its own team in one wave (0 = off)
   bool sync_steps = false;  // block barrier at every row step of a persistent sweep (keeps the CTA's warps aligned)
   bool nonpersistent = false;  // RowTeam: one row group per CTA (the block scheduler orders the sweep)
+  int grid_waves = 0;       // PackedTile / RowTeam: grid = waves x resident CTAs (0 = the planner decides)
   int nslab = 1;            // GlobalSweep: column slabs of T x V x E columns (wide rows); CTA b owns slab b % nslab
   bool hoist_colvec = true; // keep COLVEC operands in registers across rows
   int tile_rows = 0;        // PackedTile rows per stage
@@ -142,6 +143,7 @@ struct Tuning {
   int sync = -1;            // 1 / 0: block barrier at every row step of a persistent sweep
   int prefetch = -1;        // 1: software-prefetch the next rows in the global sweep (off by default)
   int persistent = -1;      // 0: row teams on a non-persistent grid (one row group per CTA)
+  int waves = 0;            // packed tiles: grid = waves x the resident CTAs
   std::string text;         // the string it was parsed from (describe())
 };
 bool parse_tuning(const char* s, Tuning& t, std::string& err);

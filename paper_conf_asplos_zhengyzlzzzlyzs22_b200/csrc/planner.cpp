@@ -634,6 +634,7 @@ void select_mapping(Plan& p) {
       m.stages = pk_stages;
       m.rows_per_block = m.threads / m.team;
       m.smem_bytes = static_cast<int>(pk_smem());
+      m.grid_waves = tu.waves > 0 ? tu.waves : 0;
       m.bank_conflict_ways = lds128_conflict_ways(static_cast<int>(C) * es_min);
       why << "row of " << chunks << " x " << (E * es_min)
           << "B chunks does not tile a power-of-two team -> TMA-staged packed tiles, thread per row; ";
@@ -689,6 +690,7 @@ void select_mapping(Plan& p) {
       m.nonpersistent = !has_mask && !ragged && m.single_wave_bps == 0 &&
                         nfull_in * m.chunks_per_lane * E <= 16;
       if (tu.persistent >= 0) m.nonpersistent = tu.persistent == 0;
+      m.grid_waves = tu.waves > 0 ? tu.waves : 0;
       why << (m.single_wave_bps ? "one wave of teams (one row per team); " : "") << "row team of " << m.team << " lanes x " << m.chunks_per_lane << " chunks ("
           << m.rows_per_block << " rows / block, packing), regional via shuffles" << (m.team > 32 ? "+smem" : "")
           << "; ";
@@ -828,7 +830,20 @@ void retune_grid(Plan& p) {
     m.grid = std::max<int64_t>(1, work_units);
     m.vertical_trips = 1;
   } else {
-    m.grid = std::max<int64_t>(1, std::min(work_units, wave));
+    // Oversubscribed grids (non-cooperative templates): CTAs beyond the
+    // resident ones start as earlier CTAs finish, which balances the tail.
+    // Measured on B200 (scripts/sweeps/r02_waves*.txt): TMA packed tiles
+    // best at ~2.5 tiles per CTA (C4: 95.1 -> 86.1 us; 1 tile per CTA loses
+    // the TMA pipeline: 95.2 us); masked register row teams best at ~8 row
+    // steps per CTA (C3: 143.5 -> 140.4 us).  Packed varlen rows and
+    // unmasked heavy rows measured slower oversubscribed (C3v 78.5 vs 84+ us;
+    // LayerNorm+GELU [65536, 768] 52.2 vs 53.7 us): one wave.
+    int64_t target = wave;
+    if (m.tmpl == Template::PackedTile) target = std::max<int64_t>(wave, (work_units * 2 + 4) / 5);
+    else if (m.tmpl == Template::RowTeam && p.g.lengths_node >= 0 && p.g.segments_node < 0 && m.single_wave_bps == 0)
+      target = std::max<int64_t>(wave, std::min<int64_t>(wave * 16, work_units / 8));
+    if (m.grid_waves > 1 && (m.tmpl == Template::PackedTile || m.tmpl == Template::RowTeam)) target = wave * m.grid_waves;
+    m.grid = std::max<int64_t>(1, std::min(work_units, target));
     m.vertical_trips = (work_units + m.grid - 1) / m.grid;
   }
   // block barrier per row step of a persistent multi-trip sweep (the CTA's
