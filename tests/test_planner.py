@@ -261,8 +261,8 @@ def test_one_wave_row_teams_and_store_cap():
     assert m["vertical_trips"] == 1
     d, _, _ = describe("C2", rows=300)                     # 2 warps per SM: default blocks
     assert d["mapping"]["single_wave_bps"] == 0
-    d, _, _ = describe("C3")
-    assert d["mapping"]["blocks_per_sm"] == 3 and d["mapping"]["grid"] == 3 * 148
+    d, _, _ = describe("C3")      # 3 resident blocks of 256 per SM, an oversubscribed grid
+    assert d["mapping"]["blocks_per_sm"] == 3 and d["mapping"]["grid"] >= 3 * 148
     d, _, _ = describe("fig6a")
     assert d["mapping"]["blocks_per_sm"] == 8
 
