@@ -6,7 +6,7 @@ the row-scalar ops every lane of a team computes).  A ratio near 1 means every
 heavy element-wise op ran once per element (element/operator-level reuse,
 P:L194-L196): no producer was recomputed for its consumers.
 
-    python scripts/mufu_evidence.py [gpurun_out] > profiles/r01_mufu.md
+    python scripts/mufu_evidence.py [gpurun_out] [round] > profiles/<round>_mufu.md
 """
 import csv
 import io
@@ -67,12 +67,12 @@ def expected(cfg):
     return None, ""
 
 
-def main(out="gpurun_out"):
+def main(out="gpurun_out", rnd=""):
     print("# MUFU (transcendental) thread-instructions: executed vs needed (ncu source page)\n")
     print("| cfg | executed | by opcode | needed | ratio | counted as |")
     print("|---|---|---|---|---|---|")
     for cfg in ("C2", "C3", "C4", "C5", "C3v"):
-        rep = os.path.join(out, f"prof_{cfg}.ncu-rep")
+        rep = os.path.join(out, f"prof_{rnd}_{cfg}.ncu-rep" if rnd else f"prof_{cfg}.ncu-rep")
         if not os.path.exists(rep):
             continue
         got = mufu_counts(rep)
@@ -84,4 +84,4 @@ def main(out="gpurun_out"):
 
 
 if __name__ == "__main__":
-    main(*(sys.argv[1:2]))
+    main(*(sys.argv[1:3]))
