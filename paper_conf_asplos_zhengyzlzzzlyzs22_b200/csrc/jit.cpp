@@ -130,9 +130,11 @@ bool mkdirs(const std::string& d) {
   return true;
 }
 
-const char* kMagic = "ASTITCH-CUBIN-2";
+const char* kMagic = "ASTITCH-CUBIN-3";
 
-bool disk_load(const std::string& path, uint64_t key, size_t src_len, std::vector<char>& cubin, std::string& log) {
+bool disk_load(const std::string& path, uint64_t key, const std::string& src, std::vector<char>& cubin,
+               std::string& log) {
+  const size_t src_len = src.size();
   std::ifstream f(path, std::ios::binary);
   if (!f) return false;
   std::string magic;
@@ -141,6 +143,9 @@ bool disk_load(const std::string& path, uint64_t key, size_t src_len, std::vecto
   if (!std::getline(f, magic) || magic != kMagic) return false;
   if (!(f >> k >> sl >> ls >> cs) || k != key || sl != src_len || cs == 0 || cs > (1u << 30)) return false;
   f.get();  // newline
+  std::string stored(sl, '\0');  // the full source: a hash collision can never return a wrong cubin
+  if (sl && !f.read(&stored[0], static_cast<std::streamsize>(sl))) return false;
+  if (stored != src) return false;
   log.assign(ls, '\0');
   cubin.resize(cs);
   if (ls && !f.read(&log[0], static_cast<std::streamsize>(ls))) return false;
@@ -148,14 +153,16 @@ bool disk_load(const std::string& path, uint64_t key, size_t src_len, std::vecto
   return true;
 }
 
-void disk_store(const std::string& dir, const std::string& path, uint64_t key, size_t src_len,
+void disk_store(const std::string& dir, const std::string& path, uint64_t key, const std::string& src,
                 const std::vector<char>& cubin, const std::string& log) {
+  const size_t src_len = src.size();
   if (!mkdirs(dir)) return;
   const std::string tmp = path + ".tmp" + std::to_string(getpid());
   {
     std::ofstream f(tmp, std::ios::binary);
     if (!f) return;
     f << kMagic << "\n" << key << " " << src_len << " " << log.size() << " " << cubin.size() << "\n";
+    f.write(src.data(), static_cast<std::streamsize>(src.size()));
     f.write(log.data(), static_cast<std::streamsize>(log.size()));
     f.write(cubin.data(), static_cast<std::streamsize>(cubin.size()));
     if (!f) { std::remove(tmp.c_str()); return; }
@@ -191,7 +198,7 @@ bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<
   char hex[32];
   snprintf(hex, sizeof(hex), "%016llx", static_cast<unsigned long long>(key));
   const std::string path = dir.empty() ? "" : dir + "/" + hex + ".cubin";
-  if (!path.empty() && disk_load(path, key, src.size(), cubin, log)) {
+  if (!path.empty() && disk_load(path, key, src, cubin, log)) {
     std::lock_guard<std::mutex> lk(g_cache_mu);
     g_cache[src] = {cubin, log};
     if (cache_state) *cache_state = 2;
@@ -226,7 +233,7 @@ bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<
   cubin.resize(cs);
   n->cubin(prog, cubin.data());
   n->destroy(&prog);
-  if (!path.empty()) disk_store(dir, path, key, src.size(), cubin, log);
+  if (!path.empty()) disk_store(dir, path, key, src, cubin, log);
   std::lock_guard<std::mutex> lk(g_cache_mu);
   g_cache[src] = {cubin, log};
   return true;
