@@ -254,6 +254,7 @@ bool nvrtc_compile(const std::string& src, const std::string& name, std::vector<
                    std::string& log, std::string& err, int* cache_state = nullptr);
 const char* device_header_source();
 void set_cache_dir(const char* dir);  // "" disables the on-disk cubin cache
+bool log_enabled();                   // ASTITCH_LOG=1: plan summaries on stderr (diagnostics only)
 
 // driver.cpp — libcuda via dlopen
 struct Driver;

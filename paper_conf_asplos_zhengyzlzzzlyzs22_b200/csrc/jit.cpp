@@ -172,6 +172,16 @@ void disk_store(const std::string& dir, const std::string& path, uint64_t key, c
 
 }  // namespace
 
+// ASTITCH_LOG=1: one line per plan on stderr (template, grid, registers,
+// demotions, plan time).  Diagnostics only: it never changes a plan.
+bool log_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("ASTITCH_LOG");
+    return e && *e && *e != '0';
+  }();
+  return on;
+}
+
 void set_cache_dir(const char* dir) {
   std::lock_guard<std::mutex> lk(g_dir_mu);
   g_dir_set = true;

@@ -8,7 +8,19 @@
 
 #include "internal.h"
 
+// NVTX ranges (header-only nvtx3: a no-op unless a profiler injects its
+// library) around planning and every run, so nsys / ncu timelines show the
+// plan (JIT) phases and which plan launched which kernel
+#include <nvtx3/nvToolsExt.h>
+
 using namespace astitch;
+
+namespace {
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
 
 namespace {
 
@@ -235,6 +247,7 @@ astitch_status astitch_plan(astitch_graph_t gr, const astitch_plan_desc* desc, a
 astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc, const char* tuning,
                                astitch_plan_t* out) {
   if (!gr || !desc || !out) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL graph, desc or out");
+  NvtxRange nvtx("astitch_plan");
   *out = nullptr;
   if (desc->rows < 0) return fail(ASTITCH_ERR_SHAPE, "rows < 0");
   if (desc->cols < 1) return fail(ASTITCH_ERR_SHAPE, "cols < 1");
@@ -324,6 +337,14 @@ astitch_status astitch_plan_ex(astitch_graph_t gr, const astitch_plan_desc* desc
     }
     p.ms_total = ms_since(t_start);
     p.describe = describe_json(p);
+    if (log_enabled())
+      fprintf(stderr, "[astitch] plan %lldx%lld: %s, kernel %s grid %lld x %d threads, %d regs, %d B smem, "
+              "%zu demotion(s), %.1f ms (nvrtc %.1f ms, %d compiled, %d cached)\n",
+              static_cast<long long>(p.desc.rows), static_cast<long long>(p.desc.cols), template_name(p.map.tmpl),
+              p.kernels.empty() ? "-" : p.kernels[0].name.c_str(),
+              static_cast<long long>(p.kernels.empty() ? 0 : p.kernels[0].grid), p.map.threads,
+              p.kernels.empty() ? -1 : p.kernels[0].regs, p.map.smem_bytes, p.demotions.size(), p.ms_total,
+              p.ms_nvrtc, p.n_compiles, p.n_mem_hits + p.n_disk_hits);
     auto* h = new astitch_plan_s();
     h->p = std::move(plan);
     *out = h;
@@ -494,6 +515,7 @@ astitch_status astitch_run(astitch_plan_t h, const void* const* inputs, void* co
   if (!h) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL plan");
   const Plan& p = *h->p;
   if (p.desc.rows == 0) return ASTITCH_OK;
+  NvtxRange nvtx("astitch_run");
   astitch_status s = check_io(p, inputs, outputs, ws);
   if (s != ASTITCH_OK) return s;
   KernelParams kp = make_params(p, inputs, outputs, ws);
