@@ -813,3 +813,23 @@ def test_mixed_precision_adds_fhadd():
     src = plan.source(0)
     assert "hadd2_f16" in src and "hadd2_bf16" in src
     _compare(RESID_F16, got, evaluate(RESID_F16, x))
+
+
+@pytest.mark.parametrize("cfg,rows,cols,tune", [
+    ("C5", 40000, 1024, {"threads": 512, "sync": 0, "prefetch": 1}),     # round-1 global sweep mapping
+    ("C5", 40000, 1024, {"threads": 256, "bps": 4, "sync": 1}),
+    ("C4", 100003, 36, {"waves": 1}), ("C4", 100003, 36, {"waves": 36}),  # packed tiles: 1 wave / 1 tile per CTA
+    ("C3", 2048, 512, {"waves": 1}), ("C3", 2048, 512, {"persistent": 0}),
+    ("fig6a", 100001, 32, {"persistent": 1}), ("C1", 50000, 128, {"persistent": 0, "threads": 128}),
+    ("C2", 5000, 768, {"team": 16}), ("bn", 20000, 96, {"sync": 1, "prefetch": 0})])
+def test_parity_under_tuning_overrides(cfg, rows, cols, tune):
+    """astitch_plan_ex overrides reach every mapping knob the sweeps use;
+    each tuned plan still matches the oracle (the defaults are only the
+    fastest of these correct mappings)."""
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 256
+    x = gen.generate(cfg, spec)
+    got, plan = run_gpu(spec, x, return_plan=True, tune=tune)
+    assert plan.describe()["tuning"]
+    _compare(spec, got, evaluate(spec, x))
