@@ -824,7 +824,7 @@ void retune_grid(Plan& p) {
     const int64_t groups = std::max<int64_t>(1, std::min(work_units, wave / m.nslab));
     m.grid = groups * m.nslab;
     m.vertical_trips = (work_units + groups - 1) / groups;
-  } else if (m.tmpl == Template::RowTeam && m.nonpersistent) {
+  } else if (m.tmpl == Template::RowTeam && m.nonpersistent && work_units < (1LL << 31)) {
     // one row group per CTA: the hardware block scheduler streams the CTAs
     // through the rows in address order (no software prefetch needed)
     m.grid = std::max<int64_t>(1, work_units);
@@ -843,7 +843,7 @@ void retune_grid(Plan& p) {
     else if (m.tmpl == Template::RowTeam && p.g.lengths_node >= 0 && p.g.segments_node < 0 && m.single_wave_bps == 0)
       target = std::max<int64_t>(wave, std::min<int64_t>(wave * 16, work_units / 8));
     if (m.grid_waves > 1 && (m.tmpl == Template::PackedTile || m.tmpl == Template::RowTeam)) target = wave * m.grid_waves;
-    m.grid = std::max<int64_t>(1, std::min(work_units, target));
+    m.grid = std::max<int64_t>(1, std::min({work_units, target, static_cast<int64_t>(INT32_MAX)}));
     m.vertical_trips = (work_units + m.grid - 1) / m.grid;
   }
   // block barrier per row step of a persistent multi-trip sweep (the CTA's
