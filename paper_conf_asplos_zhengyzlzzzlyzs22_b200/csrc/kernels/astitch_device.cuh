@@ -570,8 +570,8 @@ __device__ __forceinline__ void wait_flags(const unsigned int* flags, int world,
 }
 
 // ------------------------------------------------------------------ global: grid barrier
-// Generation-counted, self-resetting barrier for a co-resident (cooperative)
-// grid.  bar[0] = arrival count, bar[1] = generation.  No memset per run.
+// Self-resetting barrier for a co-resident (cooperative) grid on the word
+// bar[0] (below).  No memset per run.
 __device__ __forceinline__ u32 ld_acquire(const u32* p) {
   u32 v; asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
 }
@@ -581,36 +581,43 @@ __device__ __forceinline__ void st_release(u32* p, u32 v) {
 __device__ __forceinline__ u32 atom_add_acqrel(u32* p, u32 v) {
   u32 old; asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory"); return old;
 }
-// Generation-counted barrier: the arrival count returns to 0 at the end of
-// every episode (so any grid size may reuse the workspace), the generation
-// word is bumped with release semantics by the last arriver, and waiters
-// poll it with acquire loads.  acq_rel on the arrival atomic publishes this
-// CTA's writes (ordered before it by __syncthreads); no extra fences.
+// Grid barrier on ONE self-resetting word (round 2): every CTA adds 1 except
+// CTA 0, which adds 2^31 - (nb - 1), so the word crosses a multiple of 2^31
+// -- its top bit flips -- exactly when the last CTA arrives, whatever the
+// arrival order; waiters poll that bit.  Each episode adds exactly 2^31, so
+// the word is again a multiple of 2^31 afterwards (no reset, any number of
+// barriers and runs; workspace_init zeroes it once).  A CTA already at the
+// next barrier cannot flip the bit back before everyone has left this one
+// (its partial contribution stays below 2^31).  One atomic per CTA and no
+// release store on the critical path: 1.2 us per barrier vs 1.9-2.0 us for
+// the round-1 count + generation pair (scripts/micro/barrier_compare.cu).
+// __threadfence before the arrival publishes this CTA's writes (ordered
+// before it by __syncthreads), the one after the wait acquires the others'.
+__device__ __forceinline__ u32 ld_volatile_u32(const u32* p) {
+  u32 v; asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
+}
 __device__ __forceinline__ void grid_barrier(u32* bar) {
   __syncthreads();
   if (threadIdx.x == 0) {
     const u32 nb = gridDim.x * gridDim.y * gridDim.z;
-    const u32 gen = ld_acquire(bar + 1);
-    const u32 arrived = atom_add_acqrel(bar, 1u);
-    if (arrived == nb - 1) {
-      asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(bar), "r"(0u) : "memory");
-      st_release(bar + 1, gen + 1);
-    } else {
+    const u32 add = (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0) ? (0x80000000u - (nb - 1u)) : 1u;
+    __threadfence();
+    const u32 old = atomicAdd(bar, add);
 #ifdef AS_BARRIER_TIMEOUT_NS
-      // debug build of the barrier (ASTITCH_FLAG_DEBUG_BARRIER): a block that
-      // never arrives (a non-resident grid, a corrupted workspace) makes the
-      // waiters trap after the bound instead of hanging the GPU
-      const unsigned long long t0 = globaltimer_ns();
-      while (ld_acquire(bar + 1) == gen) {
-        if (globaltimer_ns() - t0 > (unsigned long long)(AS_BARRIER_TIMEOUT_NS)) {
-          printf("astitch: grid barrier timeout (block %u of %u arrived count %u)\n", blockIdx.x, nb, ld_acquire(bar));
-          __trap();
-        }
+    // debug build of the barrier (ASTITCH_FLAG_DEBUG_BARRIER): a block that
+    // never arrives (a non-resident grid, a corrupted workspace) makes the
+    // waiters trap after the bound instead of hanging the GPU
+    const unsigned long long t0 = globaltimer_ns();
+    while (((old ^ ld_volatile_u32(bar)) & 0x80000000u) == 0u) {
+      if (globaltimer_ns() - t0 > (unsigned long long)(AS_BARRIER_TIMEOUT_NS)) {
+        printf("astitch: grid barrier timeout (block %u of %u, word %08x)\n", blockIdx.x, nb, ld_volatile_u32(bar));
+        __trap();
       }
-#else
-      while (ld_acquire(bar + 1) == gen) { }
-#endif
     }
+#else
+    while (((old ^ ld_volatile_u32(bar)) & 0x80000000u) == 0u) { }
+#endif
+    __threadfence();
   }
   __syncthreads();
 }
