@@ -1,0 +1,52 @@
+#!/usr/bin/env python
+"""Structural fuzz: seeded random stitch-op graphs (workloads/random_graphs.py:
+element-wise chains, row / column reductions, broadcasts, up to two column
+reduction levels) on random shapes, GPU vs the fp64 oracle.
+    python scripts/fuzz_graphs.py SEED0 N
+A case fails if any output misses the DESIGN.md rule at 10x the config
+tolerance (random chains can cancel; structural bugs give O(1) errors); the
+worst floored relative error is printed for every case."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+from oracle import evaluate  # noqa: E402
+from tests.harness import check_close, run_gpu, spec_tol  # noqa: E402
+from workloads import gen  # noqa: E402
+from workloads.random_graphs import random_graph  # noqa: E402
+
+
+def main():
+    s0, n = int(sys.argv[1]), int(sys.argv[2])
+    bad = 0
+    worst = 0.0
+    for seed in range(s0, s0 + n):
+        rng = np.random.default_rng(10_000 + seed)
+        rows = int(rng.choice([int(rng.integers(1, 100)), int(rng.integers(100, 5000)), int(rng.integers(5000, 30000))]))
+        cols = int(rng.choice([int(rng.integers(1, 64)), int(rng.integers(64, 1100)), int(rng.integers(1100, 6000))]))
+        cols = max(1, min(cols, 4_000_000 // rows))
+        spec = random_graph(seed, rows, cols)
+        x = gen.generate("fig6a", spec)
+        try:
+            got, plan = run_gpu(spec, x, return_plan=True)
+            ref = evaluate(spec, x)
+            errs = []
+            for name, dt in spec["outputs"]:
+                info = check_close(got[name], ref[name], dt, 10 * spec_tol(spec), name=name)
+                errs.append(info["max_rel_err_floored"])
+            w = max(errs)
+            worst = max(worst, w)
+            print(f"ok seed={seed} [{rows},{cols}] {plan.describe()['mapping']['template']} max_rel={w:.2e}", flush=True)
+        except Exception as e:
+            if "ASTITCH_ERR_UNSUPPORTED" in str(e):
+                print(f"unsupported seed={seed}: {str(e)[:120]}")
+                continue
+            bad += 1
+            print(f"FAIL seed={seed} [{rows},{cols}]: {str(e)[:400]}", flush=True)
+    print(f"graph fuzz done: {n} seeds, failures: {bad}, worst floored rel err {worst:.2e}")
+
+
+if __name__ == "__main__":
+    main()
