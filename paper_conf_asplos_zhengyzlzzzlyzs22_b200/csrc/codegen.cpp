@@ -298,9 +298,16 @@ struct Gen {
   std::vector<Stream> streams;
 
   // does any consumer of node i run in the current sweep?
-  bool node_used_in_phase(int i, bool /*post*/) const {
-    for (int u : I(i).consumers)
-      if (I(u).live && phase_of(u) == cur_level) return true;
+  bool node_used_in_phase(int i, bool post = false) const {
+    for (int u : I(i).consumers) {
+      if (!I(u).live) continue;
+      // broadcasts are folded into their consumers: look through them
+      if (N(u).type == NodeType::Bcast) {
+        if (node_used_in_phase(u, post)) return true;
+        continue;
+      }
+      if (phase_of(u) == cur_level) return true;
+    }
     return false;
   }
 
@@ -892,16 +899,25 @@ struct Gen {
                sfx + "[k / 2], " + ref2(nd.a, sfx) + ")";
     }
     std::string a = ref2(nd.a, sfx), b = ref2(nd.b, sfx);
-    auto lo = [&](int v) { return "as::bc2(s" + std::to_string(N(v).a) + sfx + "lo)"; };
-    auto clo = [&](int v) { return "as::f2{" + col_lo(v, "k") + ", " + col_lo(v, "k + 1") + "}"; };
-    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.b)) return "as::sub2(as::sub2(" + a + ", " + b + "), " + clo(nd.b) + ")";
-    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.a)) return "as::add2(as::sub2(" + a + ", " + b + "), " + clo(nd.a) + ")";
-    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.b)) return "as::add2(as::add2(" + a + ", " + b + "), " + clo(nd.b) + ")";
-    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.a)) return "as::add2(as::add2(" + a + ", " + b + "), " + clo(nd.a) + ")";
-    if (nd.sub == ASTITCH_SUB && precise_bcast(nd.b)) return "as::sub2(as::sub2(" + a + ", " + b + "), " + lo(nd.b) + ")";
-    if (nd.sub == ASTITCH_SUB && precise_bcast(nd.a)) return "as::add2(as::sub2(" + a + ", " + b + "), " + lo(nd.a) + ")";
-    if (nd.sub == ASTITCH_ADD && precise_bcast(nd.b)) return "as::add2(as::add2(" + a + ", " + b + "), " + lo(nd.b) + ")";
-    if (nd.sub == ASTITCH_ADD && precise_bcast(nd.a)) return "as::add2(as::add2(" + a + ", " + b + "), " + lo(nd.a) + ")";
+    // hi + lo operands (R7b row means, R7c column means): (a_hi ± b_hi) + (a_lo ± b_lo),
+    // every lo part that exists (both operands may carry one, e.g. m - m)
+    if (nd.type == NodeType::Binary && (nd.sub == ASTITCH_ADD || nd.sub == ASTITCH_SUB)) {
+      auto lo2 = [&](int v) -> std::string {
+        if (precise_bcast_col(v)) return "as::f2{" + col_lo(v, "k") + ", " + col_lo(v, "k + 1") + "}";
+        if (precise_bcast(v)) return "as::bc2(s" + std::to_string(N(v).a) + sfx + "lo)";
+        return "";
+      };
+      const std::string la = lo2(nd.a), lb = lo2(nd.b);
+      if (!la.empty() || !lb.empty()) {
+        const bool sub = nd.sub == ASTITCH_SUB;
+        std::string hi = std::string(sub ? "as::sub2(" : "as::add2(") + a + ", " + b + ")";
+        std::string lo;
+        if (!la.empty() && !lb.empty()) lo = std::string(sub ? "as::sub2(" : "as::add2(") + la + ", " + lb + ")";
+        else if (!la.empty()) lo = la;
+        else return std::string(sub ? "as::sub2(" : "as::add2(") + hi + ", " + lb + ")";
+        return "as::add2(" + hi + ", " + lo + ")";
+      }
+    }
     return binop2(nd.sub, nd.b, a, b);
   }
 
@@ -983,18 +999,22 @@ struct Gen {
   std::string col_lo(int v, const std::string& k) const { return "cp" + std::to_string(N(v).a) + "lo[" + k + "]"; }
   std::string full_binop(const Node& nd, const std::string& sfx) const {
     std::string a = ref(nd.a, "k", sfx), b = ref(nd.b, "k", sfx);
-    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.b)) return "((" + a + " - " + b + ") - " + col_lo(nd.b, "k") + ")";
-    if (nd.sub == ASTITCH_SUB && precise_bcast_col(nd.a)) return "((" + a + " - " + b + ") + " + col_lo(nd.a, "k") + ")";
-    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.b)) return "((" + a + " + " + b + ") + " + col_lo(nd.b, "k") + ")";
-    if (nd.sub == ASTITCH_ADD && precise_bcast_col(nd.a)) return "((" + a + " + " + b + ") + " + col_lo(nd.a, "k") + ")";
-    if (nd.sub == ASTITCH_SUB && precise_bcast(nd.b))
-      return "((" + a + " - " + b + ") - " + b + "lo)";
-    if (nd.sub == ASTITCH_SUB && precise_bcast(nd.a))
-      return "((" + a + " - " + b + ") + " + a + "lo)";
-    if (nd.sub == ASTITCH_ADD && precise_bcast(nd.b))
-      return "((" + a + " + " + b + ") + " + b + "lo)";
-    if (nd.sub == ASTITCH_ADD && precise_bcast(nd.a))
-      return "((" + a + " + " + b + ") + " + a + "lo)";
+    if (nd.sub == ASTITCH_ADD || nd.sub == ASTITCH_SUB) {  // hi + lo operands (R7b / R7c)
+      auto lo1 = [&](int v, const std::string& r) -> std::string {
+        if (precise_bcast_col(v)) return col_lo(v, "k");
+        if (precise_bcast(v)) return r + "lo";
+        return "";
+      };
+      const std::string la = lo1(nd.a, a), lb = lo1(nd.b, b);
+      if (!la.empty() || !lb.empty()) {
+        const std::string op = nd.sub == ASTITCH_SUB ? " - " : " + ";
+        std::string lo;
+        if (!la.empty() && !lb.empty()) lo = "(" + la + op + lb + ")";
+        else if (!la.empty()) lo = la;
+        else return "((" + a + op + b + ")" + op + lb + ")";
+        return "((" + a + op + b + ") + " + lo + ")";
+      }
+    }
     return binop(nd.sub, nd.b, a, b);
   }
 

@@ -319,6 +319,15 @@ void analyse(Plan& p) {
     for (int a : {nd.a, nd.b})
       if (a >= 0 && g.nodes[a].kind == ASTITCH_COLVEC && info[a].post) need[a] = true;
   }
+  // keep only chains that start at a precise column SUM (a MIN / MAX of an
+  // RMAX, for example, has no cancellation-prone sum behind it)
+  for (int i = 0; i < n; ++i) {
+    if (!info[i].precise_col || g.nodes[i].type == NodeType::Reduce) continue;
+    bool from_sum = false;
+    for (int a : {g.nodes[i].a, g.nodes[i].b})
+      if (a >= 0 && info[a].precise_col) from_sum = true;
+    info[i].precise_col = from_sum;
+  }
   for (int id : p.colreds)
     if (info[id].precise_col) ++p.n_precise_colreds;
 }
@@ -872,8 +881,10 @@ void plan_workspace(Plan& p) {
     off = align(off + static_cast<size_t>(nparts) * nslots * C * 4);
     w.colvals = off;
     // [post COLVEC hi][rank-local column totals][post COLVEC lo (R7c)]
+    bool any_precise_post = false;
+    for (int id : p.post_colvecs) any_precise_post |= p.info[id].precise_col;
     off = align(off + std::max<size_t>(p.post_colvecs.size(), 1) * C * 4 + C * 4 * p.colreds.size() +
-                (p.n_precise_colreds ? p.post_colvecs.size() * C * 4 : 0));
+                (any_precise_post ? p.post_colvecs.size() * C * 4 : 0));
     w.globals = off;
     // a6 memory reuse: a global buffer is live from the sweep that
     // writes it to the last sweep that reads it; a later value of the same

@@ -833,3 +833,19 @@ def test_parity_under_tuning_overrides(cfg, rows, cols, tune):
     got, plan = run_gpu(spec, x, return_plan=True, tune=tune)
     assert plan.describe()["tuning"]
     _compare(spec, got, evaluate(spec, x))
+
+
+@pytest.mark.parametrize("seed,rows,cols", [(19, 3386, 28), (51, 66, 1034), (102, 2750, 47), (156, 18410, 50),
+                                            (190, 22178, 30), (217, 21, 823), (262, 18417, 58),
+                                            (3, 700, 300), (7, 5000, 96), (11, 64, 2048)])
+def test_parity_random_graphs(seed, rows, cols):
+    """Seeded random stitch-op graphs (workloads/random_graphs.py): the first
+    seven are the round-2 structural-fuzz failures -- a ROWVEC input read
+    through a broadcast after a grid barrier (undefined row scalar), m - m of
+    one hi+lo column mean (one lo part dropped), and a MIN of a column max
+    taking the fp64 column path without its workspace."""
+    from workloads.random_graphs import random_graph
+    spec = random_graph(seed, rows, cols)
+    x = gen.generate("fig6a", spec)
+    got = run_gpu(spec, x)
+    _compare(spec, got, evaluate(spec, x), tol=10 * spec_tol(spec))
