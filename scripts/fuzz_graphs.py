@@ -20,6 +20,7 @@ from workloads.random_graphs import random_graph  # noqa: E402
 
 def main():
     s0, n = int(sys.argv[1]), int(sys.argv[2])
+    wide = "--wide" in sys.argv
     bad = 0
     worst = 0.0
     for seed in range(s0, s0 + n):
@@ -27,10 +28,13 @@ def main():
         rows = int(rng.choice([int(rng.integers(1, 100)), int(rng.integers(100, 5000)), int(rng.integers(5000, 30000))]))
         cols = int(rng.choice([int(rng.integers(1, 64)), int(rng.integers(64, 1100)), int(rng.integers(1100, 6000))]))
         cols = max(1, min(cols, 4_000_000 // rows))
-        spec = random_graph(seed, rows, cols)
+        spec = random_graph(seed, rows, cols, wide=wide)
+        flags = 0
+        if wide:
+            flags = int(rng.choice([0, 0, 0, 0, 0, 2, 4, 64]))
         x = gen.generate("fig6a", spec)
         try:
-            got, plan = run_gpu(spec, x, return_plan=True)
+            got, plan = run_gpu(spec, x, return_plan=True, flags=flags)
             ref = evaluate(spec, x)
             errs = []
             for name, dt in spec["outputs"]:
@@ -38,7 +42,8 @@ def main():
                 errs.append(info["max_rel_err_floored"])
             w = max(errs)
             worst = max(worst, w)
-            print(f"ok seed={seed} [{rows},{cols}] {plan.describe()['mapping']['template']} max_rel={w:.2e}", flush=True)
+            print(f"ok seed={seed} [{rows},{cols}] flags={flags} {plan.describe()['mapping']['template']} max_rel={w:.2e}",
+                  flush=True)
         except Exception as e:
             if "ASTITCH_ERR_UNSUPPORTED" in str(e):
                 print(f"unsupported seed={seed}: {str(e)[:120]}")

@@ -12,14 +12,16 @@ SAFE_UNARY = ["NEG", "ABS", "TANH", "SIGMOID", "GELU_TANH", "ERF", "GELU_TANH_GR
 BINARY = ["ADD", "SUB", "MUL", "MAX", "MIN"]
 
 
-def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None) -> dict:
+def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide: bool = False) -> dict:
+    """wide=True: also random F16 inputs, BF16 / F16 outputs and key-padding
+    masks (the "wide" fuzz); False keeps the round-2 regression seeds stable."""
     rng = np.random.default_rng(seed)
     ops, inputs = [], []
     vals = {"FULL": [], "ROWVEC": [], "COLVEC": []}
     nfull = int(rng.integers(1, 4))
     for i in range(nfull):
         n = f"x{i}"
-        inputs.append((n, "FULL", str(rng.choice(["F32", "BF16"]))))
+        inputs.append((n, "FULL", str(rng.choice(["F32", "BF16", "F16"] if wide else ["F32", "BF16"]))))
         vals["FULL"].append(n)
     if rng.random() < 0.5:
         inputs.append(("rv", "ROWVEC", "F32"))
@@ -102,5 +104,12 @@ def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None) -> d
             outs.append((cand[-1], "F32"))
     if not outs:
         outs.append((vals["FULL"][0], "F32"))
-    return {"name": f"random_{seed}", "rows": rows, "cols": cols, "inputs": inputs, "mask": None, "ops": ops,
+    mask = None
+    if wide:
+        outs = [(n, str(rng.choice(["F32", "BF16", "F16"])) if kinds.get(n) == "FULL" else "F32") for n, _ in outs]
+        if rng.random() < 0.25:
+            rps = int(rng.integers(1, 200))
+            inputs.append(("L", "LENGTHS", "I32"))
+            mask = {"lengths": "L", "rows_per_segment": rps}
+    return {"name": f"random_{seed}", "rows": rows, "cols": cols, "inputs": inputs, "mask": mask, "ops": ops,
             "outputs": outs}
