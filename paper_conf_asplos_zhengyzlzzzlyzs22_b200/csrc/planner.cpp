@@ -258,12 +258,17 @@ void analyse(Plan& p) {
     // a pre-barrier FULL / ROWVEC value read after the barrier (by anything
     // but the column reduction that accumulates it before the barrier)
     // (broadcasts are folded into their consumers: look through them)
+    // (a column reduction accumulates in the sweep of its operand's level:
+    // it reads v after the barrier iff that operand sits above v's level,
+    // e.g. the broadcast of a row reduction demoted by FORCE_GLOBAL)
     std::function<bool(int, int)> later_use = [&](int v, int lvl) {
       for (int u : info[v].consumers) {
         if (!info[u].live) continue;
         if (g.nodes[u].type == NodeType::Bcast) {
           if (later_use(u, lvl)) return true;
-        } else if (info[u].level > lvl && info[u].cls != OpClass::ReduceCol) {
+        } else if (info[u].cls == OpClass::ReduceCol) {
+          if (info[g.nodes[u].a].level > lvl) return true;
+        } else if (info[u].level > lvl) {
           return true;
         }
       }

@@ -32,7 +32,7 @@ def half_ulp(ref: np.ndarray, dtype: str) -> np.ndarray:
     return np.where(a > 0, np.exp2(e - mant - 1), 0.0)
 
 
-def check_close(gpu: np.ndarray, ref: np.ndarray, dtype: str, tol: float, name: str = "") -> dict:
+def check_close(gpu: np.ndarray, ref: np.ndarray, dtype: str, tol: float, name: str = "", atol: float = 0.0) -> dict:
     gpu = np.asarray(gpu, dtype=np.float64)
     ref = np.asarray(ref, dtype=np.float64)
     assert gpu.shape == ref.shape, (name, gpu.shape, ref.shape)
@@ -49,7 +49,7 @@ def check_close(gpu: np.ndarray, ref: np.ndarray, dtype: str, tol: float, name: 
     err = np.abs(gpu - ref)
     # + FLT_MIN: subnormal fp32 results may flush to zero (the kernels'
     # MUFU ops are .ftz; reading R21)
-    bound = tol * np.maximum(np.abs(ref), s) + half_ulp(ref, dtype) + FLT_MIN
+    bound = tol * np.maximum(np.abs(ref), s) + half_ulp(ref, dtype) + FLT_MIN + atol
     bad = err > bound
     info = {"max_abs_err": float(err.max()) if err.size else 0.0,
             "max_rel_err_floored": float((err / np.maximum(np.maximum(np.abs(ref), s), 1e-300)).max()) if err.size else 0.0,

@@ -849,3 +849,20 @@ def test_parity_random_graphs(seed, rows, cols):
     x = gen.generate("fig6a", spec)
     got = run_gpu(spec, x)
     _compare(spec, got, evaluate(spec, x), tol=10 * spec_tol(spec))
+
+
+@pytest.mark.parametrize("seed,rows,cols,flags", [(1349, 27971, 52, 2), (1070, 64, 4082, 0), (1003, 900, 200, 0),
+                                                  (1011, 4000, 64, 4)])
+def test_parity_random_graphs_wide(seed, rows, cols, flags):
+    """Wide-mode random graphs (f16 inputs, bf16 / f16 outputs, masks,
+    ablation flags).  1349: under FORCE_GLOBAL a column reduction of a
+    broadcast demoted row reduction reads it after the barrier (it must be
+    buffered).  Rule at 10x tolerance + 1e-5 absolute (1070 sums a row's
+    centred values: exactly 0 by cancellation)."""
+    from workloads.random_graphs import random_graph
+    spec = random_graph(seed, rows, cols, wide=True)
+    x = gen.generate("fig6a", spec)
+    got = run_gpu(spec, x, flags=flags)
+    ref = evaluate(spec, x)
+    for name, dt in spec["outputs"]:
+        check_close(got[name], ref[name], dt, 10 * spec_tol(spec), name=name, atol=1e-5)
