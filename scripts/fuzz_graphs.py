@@ -24,12 +24,20 @@ def main():
     wide = "--wide" in sys.argv
     bad = 0
     worst = 0.0
+    templates = {}
     for seed in range(s0, s0 + n):
         rng = np.random.default_rng(10_000 + seed)
         rows = int(rng.choice([int(rng.integers(1, 100)), int(rng.integers(100, 5000)), int(rng.integers(5000, 30000))]))
         cols = int(rng.choice([int(rng.integers(1, 64)), int(rng.integers(64, 1100)), int(rng.integers(1100, 6000))]))
-        cols = max(1, min(cols, 4_000_000 // rows))
-        spec = random_graph(seed, rows, cols, wide=wide)
+        kw = {}
+        if "--long" in sys.argv:      # few long rows, row-wise graphs: split_row / row_stream
+            rows, cols = int(rng.integers(1, 40)), int(rng.integers(30_000, 160_000))
+            kw = {"colred": False}
+        if "--tiny" in sys.argv:      # many tiny rows, row-wise, no column vectors: TMA packed tiles
+            rows, cols = int(rng.integers(4096, 60_000)), int(rng.choice([9, 12, 20, 36, 44, 60, 100]))
+            kw = {"colred": False, "colvec": False}
+        cols = max(1, min(cols, 6_000_000 // rows))
+        spec = random_graph(seed, rows, cols, wide=wide, **kw)
         flags = 0
         if wide:
             flags = int(rng.choice([0, 0, 0, 0, 0, 2, 4, 64]))
@@ -47,13 +55,14 @@ def main():
             worst = max(worst, w)
             print(f"ok seed={seed} [{rows},{cols}] flags={flags} {plan.describe()['mapping']['template']} max_rel={w:.2e}",
                   flush=True)
+            templates[plan.describe()["mapping"]["template"]] = templates.get(plan.describe()["mapping"]["template"], 0) + 1
         except Exception as e:
             if "ASTITCH_ERR_UNSUPPORTED" in str(e):
                 print(f"unsupported seed={seed}: {str(e)[:120]}")
                 continue
             bad += 1
             print(f"FAIL seed={seed} [{rows},{cols}]: {str(e)[:400]}", flush=True)
-    print(f"graph fuzz done: {n} seeds, failures: {bad}, worst floored rel err {worst:.2e}")
+    print(f"graph fuzz done: {n} seeds, failures: {bad}, worst floored rel err {worst:.2e}, templates {templates}")
 
 
 if __name__ == "__main__":

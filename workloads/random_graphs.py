@@ -12,7 +12,8 @@ SAFE_UNARY = ["NEG", "ABS", "TANH", "SIGMOID", "GELU_TANH", "ERF", "GELU_TANH_GR
 BINARY = ["ADD", "SUB", "MUL", "MAX", "MIN"]
 
 
-def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide: bool = False) -> dict:
+def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide: bool = False,
+                 colred: bool = True, colvec: bool = True) -> dict:
     """wide=True: also random F16 inputs, BF16 / F16 outputs and key-padding
     masks (the "wide" fuzz); False keeps the round-2 regression seeds stable."""
     rng = np.random.default_rng(seed)
@@ -26,7 +27,7 @@ def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide
     if rng.random() < 0.5:
         inputs.append(("rv", "ROWVEC", "F32"))
         vals["ROWVEC"].append("rv")
-    if rng.random() < 0.5:
+    if rng.random() < 0.5 and colvec:
         inputs.append(("cv", "COLVEC", "F32"))
         vals["COLVEC"].append("cv")
     k = [0]
@@ -72,7 +73,7 @@ def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide
                 ops.append((new(kind), "binary", op, a, b))
         elif choice < 0.8 and vals["FULL"]:                  # reduction of a FULL value
             a = str(rng.choice(vals["FULL"]))
-            axis = "ROW" if (rng.random() < 0.6 or ncolred >= 2) else "COL"
+            axis = "ROW" if (rng.random() < 0.6 or ncolred >= 2 or not colred) else "COL"
             red = str(rng.choice(["SUM", "RMAX"]))
             r = new("ROWVEC" if axis == "ROW" else "COLVEC")
             ops.append((r, "reduce", red, axis, a))
@@ -107,7 +108,7 @@ def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide
     mask = None
     if wide:
         outs = [(n, str(rng.choice(["F32", "BF16", "F16"])) if kinds.get(n) == "FULL" else "F32") for n, _ in outs]
-        if rng.random() < 0.25:
+        if rng.random() < 0.25 and colvec:
             rps = int(rng.integers(1, 200))
             inputs.append(("L", "LENGTHS", "I32"))
             mask = {"lengths": "L", "rows_per_segment": rps}
