@@ -295,7 +295,8 @@ astitch_status astitch_run_host_pipelined(astitch_plan_t p, const void* const* h
  * Row-sharded execution (BASELINE north_star (4)): each process owns a
  * contiguous row range and a plan built with shard_rank / shard_world.
  * Row-local subgraphs need no communication.  Column reductions are combined
- * with one ncclAllReduce(sum, fp32) of the per-rank partials on `stream`,
+ * with one ncclAllReduce per column reduction (fp32 sum, or int32 max of
+ * order keys for RMAX) of the per-rank partials on `stream`,
  * then the column consumers run in a small epilogue kernel. */
 astitch_status astitch_comm_unique_id(uint8_t id[128]);
 astitch_status astitch_comm_create(int32_t world, int32_t rank, const uint8_t id[128],
@@ -310,11 +311,23 @@ astitch_status astitch_run_sharded(astitch_plan_t p, astitch_comm_t c, const voi
  *            column totals at ws + offset (ncolred x cols floats, see below);
  *   stage 1: column consumers (+ the FULL sweep after the barrier) reading the
  *            combined totals from the same place.
- * astitch_plan_colpart reports the byte offset in ws and the float count.
+ * astitch_plan_colpart reports the byte offset in ws and the 4-byte word
+ * count: ncolred slots of `cols` words each, slot q in the order
+ * astitch_plan_colpart_ops reports.  A SUM slot holds fp32 column totals
+ * (combine: fp32 sum across ranks); an RMAX slot holds int32 ORDER KEYS of
+ * the fp32 column maxima (combine: int32 max across ranks) -- the key is
+ * monotone in the float order with NaN canonicalised to the largest key, so
+ * an integer max propagates NaN as the unsharded RMAX does (reading R12),
+ * which an fp32 max (ncclMax) would not.  astitch_run_sharded does exactly
+ * this with ncclAllReduce(ncclFloat32, ncclSum) / (ncclInt32, ncclMax).
  * Plans without a column reduction: stage 0 = astitch_run, stage 1 = no-op. */
 astitch_status astitch_run_shard_stage(astitch_plan_t p, int32_t stage, const void* const* inputs,
                                        void* const* outputs, void* ws, void* stream);
 astitch_status astitch_plan_colpart(astitch_plan_t p, size_t* byte_offset, size_t* count);
+/* The combine each colpart slot needs: ops[q] = ASTITCH_SUM or ASTITCH_RMAX.
+ * *n = the number of column reductions (always written); ops may be NULL only
+ * when that is 0; cap < *n -> ASTITCH_ERR_INVALID_ARGUMENT. */
+astitch_status astitch_plan_colpart_ops(astitch_plan_t p, int32_t* ops, size_t cap, size_t* n);
 /* Fused sharded run: the column-reduction exchange happens
  * INSIDE the stitched kernel over peer memory instead of an ncclAllReduce +
  * epilogue launch.  Each rank owns an exchange buffer (astitch_peer_create:

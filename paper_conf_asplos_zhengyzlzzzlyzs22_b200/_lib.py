@@ -103,6 +103,7 @@ _sig = {
     "astitch_run_sharded": (ct.c_int, [_vp, _vp, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
     "astitch_run_shard_stage": (ct.c_int, [_vp, ct.c_int32, ct.POINTER(_vp), ct.POINTER(_vp), _vp, _vp]),
     "astitch_plan_colpart": (ct.c_int, [_vp, ct.POINTER(ct.c_size_t), ct.POINTER(ct.c_size_t)]),
+    "astitch_plan_colpart_ops": (ct.c_int, [_vp, _i32p, ct.c_size_t, ct.POINTER(ct.c_size_t)]),
     "astitch_peer_create": (ct.c_int, [_vp, ct.POINTER(_vp), ct.c_char_p]),
     "astitch_peer_open": (ct.c_int, [_vp, ct.c_int32, ct.c_char_p]),
     "astitch_peer_link": (ct.c_int, [_vp, ct.c_int32, _vp]),

@@ -1472,6 +1472,14 @@ struct Gen {
         bool mx = N(p.colreds[q]).sub == ASTITCH_RMAX;
         std::string slot = "colpart[" + std::to_string(q) + "LL * C + col]";
         std::string t = "t" + std::to_string(p.colreds[q]);
+        if (mx && role == ROLE_SHARD_MAIN) {
+          // sharded stage 0: a MAX slot holds int32 order keys (as::okey) so
+          // the cross-rank combine is an integer max that keeps NaN (R12)
+          std::string islot = "((int*)colpart)[" + std::to_string(q) + "LL * C + col]";
+          o << "        " << islot << " = as::okey((p.flags & 1) ? as::nmax(as::okey_dec(" << islot << "), " << t
+            << ") : " << t << ");\n";
+          continue;
+        }
         o << "        " << slot << " = (p.flags & 1) ? "
           << (mx ? "as::nmax(" + slot + ", " + t + ")" : "(" + slot + " + " + t + ")") << " : " << t << ";\n";
       }
@@ -2096,8 +2104,12 @@ struct Gen {
       o << "  const float* colpart = (const float*)((const char*)p.ws + "
         << (p.ws.colvals + p.post_colvecs.size() * C * 4) << "LL);\n";
       o << "  for (long long col = blockIdx.x * 256LL + threadIdx.x; col < C; col += gridDim.x * 256LL) {\n";
-      for (size_t q = 0; q < p.colreds.size(); ++q)
-        o << "    const float t" << p.colreds[q] << " = colpart[" << q << "LL * C + col];\n";
+      for (size_t q = 0; q < p.colreds.size(); ++q) {
+        if (N(p.colreds[q]).sub == ASTITCH_RMAX)  // int32 order keys (stage 0)
+          o << "    const float t" << p.colreds[q] << " = as::okey_dec(((const int*)colpart)[" << q << "LL * C + col]);\n";
+        else
+          o << "    const float t" << p.colreds[q] << " = colpart[" << q << "LL * C + col];\n";
+      }
       emit_colvec_chain("t");
       o << "  }\n}\n";
       return o.str();

@@ -164,9 +164,12 @@ astitch_status astitch_run_sharded(astitch_plan_t h, astitch_comm_t c, const voi
   const size_t C = static_cast<size_t>(p.desc.cols);
   char* colpart = static_cast<char*>(ws) + p.ws.colvals + p.post_colvecs.size() * C * 4;
   for (size_t q = 0; q < p.colreds.size(); ++q) {
-    ncclRedOp_t op = p.g.nodes[p.colreds[q]].sub == ASTITCH_RMAX ? ncclMax : ncclSum;
+    // MAX slots hold int32 order keys (codegen: as::okey): an integer max
+    // keeps NaN, which ncclMax on fp32 would drop (reading R12)
+    const bool mx = p.g.nodes[p.colreds[q]].sub == ASTITCH_RMAX;
     float* buf = reinterpret_cast<float*>(colpart) + q * C;
-    ncclResult_t r = n->AllReduce(buf, buf, C, ncclFloat32, op, c->comm, static_cast<cudaStream_t>(stream));
+    ncclResult_t r = n->AllReduce(buf, buf, C, mx ? ncclInt32 : ncclFloat32, mx ? ncclMax : ncclSum, c->comm,
+                                  static_cast<cudaStream_t>(stream));
     if (r != ncclSuccess) return fail(ASTITCH_ERR_NCCL, std::string("ncclAllReduce: ") + n->GetErrorString(r));
   }
   for (size_t i = 1; i < p.shard_kernels.size(); ++i)
@@ -306,6 +309,16 @@ astitch_status astitch_plan_colpart(astitch_plan_t h, size_t* byte_offset, size_
   const size_t C = static_cast<size_t>(p.desc.cols);
   *byte_offset = p.ws.colvals + p.post_colvecs.size() * C * 4;
   *count = p.colreds.size() * C;
+  return ASTITCH_OK;
+}
+
+astitch_status astitch_plan_colpart_ops(astitch_plan_t h, int32_t* ops, size_t cap, size_t* n) {
+  if (!h || !n) return fail(ASTITCH_ERR_INVALID_ARGUMENT, "NULL argument");
+  const Plan& p = *h->p;
+  *n = p.colreds.size();
+  if (cap < p.colreds.size() || (!ops && !p.colreds.empty()))
+    return fail(ASTITCH_ERR_INVALID_ARGUMENT, "ops buffer smaller than the number of column reductions");
+  for (size_t q = 0; q < p.colreds.size(); ++q) ops[q] = p.g.nodes[p.colreds[q]].sub == ASTITCH_RMAX ? ASTITCH_RMAX : ASTITCH_SUM;
   return ASTITCH_OK;
 }
 

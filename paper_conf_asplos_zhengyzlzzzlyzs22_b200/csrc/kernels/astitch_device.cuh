@@ -283,6 +283,14 @@ __device__ __forceinline__ float rcp(float x) { float r; asm("rcp.approx.ftz.f32
 // numpy max does; fmaxf would drop it).  One FMNMX with the .NaN modifier.
 __device__ __forceinline__ float nmax(float a, float b) { float r; asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r; }
 __device__ __forceinline__ float nmin(float a, float b) { float r; asm("min.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r; }
+// Order key of a float for an INTEGER max across ranks (ncclMax on int32):
+// monotone in the float order, NaN canonicalised to the largest key, so the
+// sharded column RMAX propagates NaN like nmax (an fp32 ncclMax would drop it).
+__device__ __forceinline__ int okey(float x) {
+  const int b = (x != x) ? 0x7fc00000 : __float_as_int(x);
+  return b >= 0 ? b : (b ^ 0x7fffffff);
+}
+__device__ __forceinline__ float okey_dec(int k) { return __int_as_float(k >= 0 ? k : (k ^ 0x7fffffff)); }
 __device__ __forceinline__ double dmaxn(double a, double b) { return (a != a || b != b) ? a + b : fmax(a, b); }
 __device__ __forceinline__ double dminn(double a, double b) { return (a != a || b != b) ? a + b : fmin(a, b); }
 __device__ __forceinline__ float rsq(float x) { float r; asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x)); return r; }

@@ -173,6 +173,14 @@ class ShardedPlan:
         check(lib.astitch_plan_colpart(self.plan.handle, ct.byref(off), ct.byref(n)), "astitch_plan_colpart")
         return off.value, n.value
 
+    def colpart_ops(self):
+        """Per colpart slot: "sum" (fp32 totals, combine by fp32 sum) or "max"
+        (int32 order keys, combine by int32 max); astitch_plan_colpart_ops."""
+        n = ct.c_size_t()
+        buf = (ct.c_int32 * 64)()
+        check(lib.astitch_plan_colpart_ops(self.plan.handle, buf, 64, ct.byref(n)), "astitch_plan_colpart_ops")
+        return ["max" if buf[i] == 1 else "sum" for i in range(n.value)]
+
     def kernels_per_run(self) -> int:
         d = self.plan.describe()
         if self.world > 1 and d["shard_kernels"] > 0 and self.peer is None:

@@ -1,0 +1,135 @@
+#!/usr/bin/env python
+"""Structural fuzz of the row-sharded path: seeded random
+stitch-op graphs (workloads/random_graphs.py, one column-reduction level, the
+sharded planner's scope) split over 2-4 VIRTUAL ranks on one GPU, run both
+ways the library offers and compared with the fp64 oracle on the whole problem:
+  staged  astitch_run_shard_stage(0) on every rank, the rank-local column
+          partials combined on the device in rank order (tests/harness.py
+          virtual_allreduce, standing in for the NCCL allreduce: fp32 sum,
+          int32 max of the RMAX order keys),
+          then astitch_run_shard_stage(1);
+  fused   astitch_run_fused: every rank's one cooperative kernel pushes its
+          partials into all ranks' exchange slots over (here: local) peer
+          memory and combines them in rank order, all ranks running together
+          on their own streams, each plan sized for 148/world SMs.
+Column outputs must be bitwise equal across ranks.  Masked graphs take mask_row_ranges' shards.
+    python scripts/fuzz_sharded.py SEED0 N"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+from oracle import evaluate  # noqa: E402
+from tests.harness import check_close, device_inputs, from_torch, spec_tol, virtual_allreduce  # noqa: E402
+from workloads import gen  # noqa: E402
+from workloads.random_graphs import random_graph  # noqa: E402
+
+
+def shard_inputs(spec, x, b, n):
+    kinds = {nm: k for nm, k, _ in spec["inputs"]}
+    xs = {}
+    for k, v in x.items():
+        if kinds.get(k) in ("FULL", "ROWVEC"):
+            xs[k] = v[b:b + n]
+        elif kinds.get(k) == "LENGTHS":
+            rps = spec["mask"]["rows_per_segment"]
+            xs[k] = v[b // rps: -(-(b + n) // rps)]
+        else:
+            xs[k] = v
+    return xs
+
+
+def gather(spec, ranks, kinds):
+    got = {}
+    for j, (name, _) in enumerate(spec["outputs"]):
+        if kinds[name] == "COLVEC":
+            vals = [from_torch(rk["outs"][j]) for rk in ranks]
+            for v in vals[1:]:
+                assert np.array_equal(v, vals[0]), f"{name}: ranks disagree"
+            got[name] = vals[0]
+        else:
+            got[name] = np.concatenate([from_torch(rk["outs"][j]) for rk in ranks])
+    return got
+
+
+def main():
+    import torch
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import PeerExchange, ShardedPlan, mask_row_ranges
+    s0, n = int(sys.argv[1]), int(sys.argv[2])
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    bad = cases = 0
+    worst = 0.0
+    for seed in range(s0, s0 + n):
+        rng = np.random.default_rng(20_000 + seed)
+        world = int(rng.integers(2, 5))
+        rows = int(rng.choice([int(rng.integers(world, 200)), int(rng.integers(200, 5000)), int(rng.integers(5000, 30000))]))
+        cols = int(rng.choice([int(rng.integers(1, 64)), int(rng.integers(64, 1100)), int(rng.integers(1100, 4000))]))
+        cols = max(1, min(cols, 4_000_000 // rows))
+        spec = random_graph(seed, rows, cols, wide=True)
+        if spec.get("mask") and -(-rows // spec["mask"]["rows_per_segment"]) < world:
+            spec["mask"]["rows_per_segment"] = max(1, rows // world)      # at least one segment per rank
+        x = gen.generate("fig6a", spec)
+        g = A.Graph.from_spec(spec)
+        if spec.get("mask"):
+            rr = mask_row_ranges(x["L"], spec["mask"]["rows_per_segment"], cols, rows, world)
+        else:
+            rr = [None] * world
+        try:
+            ref = evaluate(spec, x)
+            results = {}
+            for mode in ("staged", "fused"):
+                ranks = []
+                for r in range(world):
+                    sp = ShardedPlan(g, rows, cols, world, r, 0, sm_count=sms // world if mode == "fused" else 0,
+                                     row_range=rr[r])
+                    b, nr = sp.row_begin, sp.row_count
+                    ins = device_inputs(dict(spec, rows=nr), shard_inputs(spec, x, b, nr))
+                    ranks.append({"sp": sp, "ins": ins, "outs": sp.plan.alloc_outputs(),
+                                  "ws": sp.plan.alloc_workspace(), "st": torch.cuda.Stream()})
+                kinds = {nm: k for nm, (k, _) in zip([o[0] for o in spec["outputs"]], ranks[0]["sp"].plan.outputs)}
+                torch.cuda.synchronize()
+                if mode == "staged":
+                    for rk in ranks:
+                        rk["sp"].run_stage(0, rk["ins"], rk["outs"], rk["ws"])
+                    virtual_allreduce([(rk["sp"], rk["ws"]) for rk in ranks])
+                    for rk in ranks:
+                        rk["sp"].run_stage(1, rk["ins"], rk["outs"], rk["ws"])
+                else:
+                    for rk in ranks:
+                        rk["sp"].peer = PeerExchange(rk["sp"].plan)
+                    for rk in ranks:
+                        for ot in ranks:
+                            if ot is not rk:
+                                rk["sp"].peer.link(ot["sp"].rank, ot["sp"].peer)
+                    for rk in ranks:
+                        rk["sp"].run(rk["ins"], rk["outs"], ws=rk["ws"], stream=rk["st"])
+                torch.cuda.synchronize()
+                if mode == "fused":
+                    for rk in ranks:
+                        assert not rk["sp"].peer.timed_out(), "fused exchange timed out"
+                results[mode] = gather(spec, ranks, kinds)
+            errs = []
+            for name, dt in spec["outputs"]:
+                info = check_close(results["fused"][name], ref[name], dt, 10 * spec_tol(spec), name=name, atol=1e-5)
+                errs.append(info["max_rel_err_floored"])
+                check_close(results["staged"][name], ref[name], dt, 10 * spec_tol(spec), name=name + " staged",
+                            atol=1e-5)
+            w = max(errs)
+            worst = max(worst, w)
+            cases += 1
+            desc = ranks[0]["sp"].plan.describe()
+            print(f"ok seed={seed} world={world} [{rows},{cols}] mask={bool(spec.get('mask'))} "
+                  f"{desc['mapping']['template']} shard_kernels={desc['shard_kernels']} max_rel={w:.2e}", flush=True)
+        except Exception as e:
+            if "ASTITCH_ERR_UNSUPPORTED" in str(e):
+                print(f"unsupported seed={seed}: {str(e)[:120]}")
+                continue
+            bad += 1
+            print(f"FAIL seed={seed} world={world} [{rows},{cols}]: {str(e)[:400]}", flush=True)
+    print(f"sharded fuzz done: {cases} cases, failures: {bad}, worst floored rel err {worst:.2e}")
+
+
+if __name__ == "__main__":
+    main()

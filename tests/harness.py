@@ -107,3 +107,30 @@ def run_gpu(spec: dict, inputs: dict, flags: int = 0, plan=None, return_plan=Fal
     if return_plan:
         return res, plan
     return res
+
+
+def virtual_allreduce(shards):
+    """Test stand-in for astitch_run_sharded's collective when every rank's
+    plan runs on one GPU: shards = [(ShardedPlan, workspace)], combined in
+    rank order in place -- fp32 sum for SUM slots, int32 max of the order keys
+    for RMAX slots (include/astitch.h, astitch_plan_colpart)."""
+    import torch
+    sp0 = shards[0][0]
+    off0, cnt = sp0.colpart()
+    if not cnt:
+        return
+    ops = sp0.colpart_ops()
+    C = cnt // len(ops)
+    for sp, _ in shards:
+        assert sp.colpart()[1] == cnt and sp.colpart_ops() == ops
+    for q, op in enumerate(ops):
+        dt = torch.int32 if op == "max" else torch.float32
+        parts = []
+        for sp, ws in shards:
+            off = sp.colpart()[0] + 4 * q * C     # each rank's own offset (depends on its grid)
+            parts.append(ws[off: off + 4 * C].view(dt))
+        total = parts[0].clone()
+        for p_ in parts[1:]:
+            total = torch.maximum(total, p_) if op == "max" else total + p_
+        for p_ in parts:
+            p_.copy_(total)

@@ -120,6 +120,25 @@ def test_shard_rows_partition():
         A.shard_rows(10, 2, 2)
 
 
+def test_colpart_ops_per_slot():
+    """astitch_plan_colpart_ops: the combine each colpart slot needs (SUM
+    totals vs RMAX order keys), in colpart slot order; a too-small buffer is
+    an error that still reports the count."""
+    from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import ShardedPlan
+    spec = {"name": "mix", "rows": 1000, "cols": 64, "inputs": [("x", "FULL", "F32")], "mask": None,
+            "ops": [("s", "reduce", "SUM", "COL", "x"), ("m", "reduce", "RMAX", "COL", "x")],
+            "outputs": [("s", "F32"), ("m", "F32")]}
+    sp = ShardedPlan(A.Graph.from_spec(spec), 1000, 64, 2, 1, -1, flags=A.FLAG_NO_COMPILE)
+    assert sorted(sp.colpart_ops()) == ["max", "sum"]
+    assert sp.colpart()[1] == 2 * 64
+    n = ct.c_size_t()
+    buf = (ct.c_int32 * 1)()
+    assert _lib.lib.astitch_plan_colpart_ops(sp.plan.handle, buf, 1, ct.byref(n)) != 0 and n.value == 2
+    row = specs.get("C2", rows=64)
+    sp2 = ShardedPlan(A.Graph.from_spec(row), 64, 768, 2, 0, -1, flags=A.FLAG_NO_COMPILE)
+    assert sp2.colpart_ops() == [] and _lib.lib.astitch_plan_colpart_ops(sp2.plan.handle, None, 0, ct.byref(n)) == 0
+
+
 def test_io_signature_and_workspace():
     spec = specs.get("C5", rows=4096)
     p = A.Plan(A.Graph.from_spec(spec), 4096, 1024, device=-1, flags=A.FLAG_NO_COMPILE)

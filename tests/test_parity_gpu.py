@@ -187,7 +187,7 @@ def test_virtual_shards(cfg, rows, cols, world):
     import torch
     import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
     from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import ShardedPlan
-    from tests.harness import device_inputs, from_torch
+    from tests.harness import device_inputs, from_torch, virtual_allreduce
     spec = specs.get(cfg, rows=rows, cols=cols)
     if spec.get("mask"):
         spec["mask"]["rows_per_segment"] = 512
@@ -211,17 +211,7 @@ def test_virtual_shards(cfg, rows, cols, world):
         ranks.append((sp, ins, outs, ws, b, n))
     for sp, ins, outs, ws, *_ in ranks:
         sp.run_stage(0, ins, outs, ws)
-    cnt = ranks[0][0].colpart()[1]
-    if cnt:
-        # each rank's own offset (the workspace layout depends on its grid)
-        parts = []
-        for sp, _, _, ws, *_ in ranks:
-            off, n_ = sp.colpart()
-            assert n_ == cnt
-            parts.append(ws[off: off + 4 * cnt].view(torch.float32))
-        total = torch.stack(parts).sum(0)
-        for p_ in parts:
-            p_.copy_(total)
+    virtual_allreduce([(sp, ws) for sp, _, _, ws, *_ in ranks])
     for sp, ins, outs, ws, *_ in ranks:
         sp.run_stage(1, ins, outs, ws)
     torch.cuda.synchronize()
@@ -583,6 +573,58 @@ def _virtual_ranks(spec, x, world):
             if other is not sp:
                 sp.peer.link(other.rank, other.peer)
     return ranks
+
+
+def test_nan_propagation_r12_sharded_and_chunked():
+    """R12 across the row-sharded and chunked paths: a column whose only NaN
+    sits in one rank's (or one chunk's) rows must come out NaN.  Stage 0 stores
+    RMAX partials as int32 order keys (NaN = the largest key), so the staged
+    combine (an integer max, like ncclMax on ncclInt32), the fused exchange
+    (max.NaN) and the chunk accumulation all keep it; an fp32 max would not."""
+    import torch
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from paper_conf_asplos_zhengyzlzzzlyzs22_b200.dist import ShardedPlan
+    from tests.harness import device_inputs, from_torch, to_torch, virtual_allreduce
+    spec = dict(NAN_COL, rows=3000)
+    rng = np.random.default_rng(13)
+    x = {"x": rng.standard_normal((3000, 256)).astype(np.float32), "w": rng.standard_normal(256).astype(np.float32)}
+    x["x"][2990, 5] = np.nan          # last rank / last chunk only
+    x["x"][10, 200] = np.nan          # first rank only
+    x["x"][:, 77] = -np.inf           # all -inf column: the identity must not turn it into NaN
+    ref = evaluate(spec, x)
+    assert np.isnan(ref["cm"][[5, 200]]).all() and ref["cm"][77] == -np.inf
+    g = A.Graph.from_spec(spec)
+    world = 3
+    shards = []
+    for r in range(world):
+        sp = ShardedPlan(g, 3000, 256, world, r, 0)
+        b, n = sp.row_begin, sp.row_count
+        xs = {k: (v[b:b + n] if getattr(v, "ndim", 0) == 2 else v) for k, v in x.items()}
+        shards.append((sp, device_inputs(dict(spec, rows=n), xs), sp.plan.alloc_outputs(), sp.plan.alloc_workspace()))
+    assert shards[0][0].colpart_ops() == ["max"]
+    for sp, ins, outs, ws in shards:
+        sp.run_stage(0, ins, outs, ws)
+    virtual_allreduce([(sp, ws) for sp, _, _, ws in shards])
+    for sp, ins, outs, ws in shards:
+        sp.run_stage(1, ins, outs, ws)
+    torch.cuda.synchronize()
+    j = [o for o, _ in spec["outputs"]].index("cm")
+    for _, _, outs, _ in shards:
+        check_close(from_torch(outs[j]), ref["cm"], "F32", spec_tol(spec), "cm staged")
+    ranks = _virtual_ranks(spec, x, world)
+    for sp, ins, outs, ws, st in ranks:
+        sp.run(ins, outs, ws=ws, stream=st)
+    torch.cuda.synchronize()
+    for _, _, outs, _, _ in ranks:
+        check_close(from_torch(outs[j]), ref["cm"], "F32", spec_tol(spec), "cm fused")
+    p = A.Plan(g, 3000, 256, device=0)
+    host_in = [to_torch(x[n], d, None).pin_memory() for n, _, d in spec["inputs"]]
+    dev_in = [torch.empty_like(h, device="cuda") for h in host_in]
+    dev_out = p.alloc_outputs()
+    host_out = [torch.empty(t.shape, dtype=t.dtype).pin_memory() for t in dev_out]
+    p.run_host(host_in, host_out, dev_in, dev_out, chunks=4)
+    torch.cuda.synchronize()
+    check_close(from_torch(host_out[j]), ref["cm"], "F32", spec_tol(spec), "cm chunked")
 
 
 @pytest.mark.parametrize("K", [1, 3, 4])
