@@ -261,6 +261,15 @@ struct Gen {
     if (I(u).cls == OpClass::ReduceCol) return I(N(u).a).level;
     return I(u).level;
   }
+  // is node u evaluated in the current sweep?  Its own level's, plus the
+  // later sweeps that recompute it instead of reading an HBM buffer (R22)
+  bool runs_here(int u) const { return phase_of(u) == cur_level || ((I(u).remat_mask >> cur_level) & 1u); }
+  int last_run(int u) const {
+    int l = phase_of(u);
+    for (int b = l + 1; b < 32; ++b)
+      if ((I(u).remat_mask >> b) & 1u) l = b;
+    return l;
+  }
 
   // byte offset of the lo parts of post-barrier COLVEC values (R7c)
   long long colvals_lo() const {
@@ -306,7 +315,7 @@ struct Gen {
         if (node_used_in_phase(u, post)) return true;
         continue;
       }
-      if (phase_of(u) == cur_level) return true;
+      if (runs_here(u)) return true;
     }
     return false;
   }
@@ -576,7 +585,7 @@ struct Gen {
       (void)post;
       // only the ops of this sweep's level; a column reduction accumulates in
       // the sweep of its operand (earlier levels come from HBM buffers)
-      if (phase_of(i) != cur_level) continue;
+      if (!runs_here(i)) continue;
       // COLVEC values: level 0 hoisted per lane, later ones finalised per column
       if (nd.kind == ASTITCH_COLVEC && !(nd.type == NodeType::Reduce && nd.axis == ASTITCH_AXIS_COL)) continue;
       std::string id = std::to_string(i);
@@ -658,7 +667,7 @@ struct Gen {
         {
           const Node& sn = N(src);
           if (mx && sn.type == NodeType::Binary && sn.sub == ASTITCH_MUL && sn.kind == ASTITCH_FULL &&
-              phase_of(src) == cur_level) {
+              runs_here(src)) {
             if (N(sn.b).type == NodeType::Const && N(sn.b).cval > 0) { post_scale = flit(N(sn.b).cval); src = sn.a; }
             else if (N(sn.a).type == NodeType::Const && N(sn.a).cval > 0) { post_scale = flit(N(sn.a).cval); src = sn.b; }
           }
@@ -875,7 +884,7 @@ struct Gen {
           std::string nbs = "as::bc2(-(" + bs + ") * 1.4426950408889634f)";
           const Node& x = N(a.a);
           if (x.type == NodeType::Binary && x.sub == ASTITCH_MUL && x.kind == ASTITCH_FULL &&
-              phase_of(a.a) == cur_level) {
+              runs_here(a.a)) {
             if (N(x.b).type == NodeType::Const)
               return "as::ex2_2(as::fma2(" + ref2(x.a, sfx) + ", as::bc2(" +
                      flit(N(x.b).cval * 1.4426950408889634) + "), " + nbs + "))";
@@ -942,7 +951,7 @@ struct Gen {
           std::string nbs = "(-(" + bs + ") * 1.4426950408889634f)";
           const Node& x = N(a.a);
           if (x.type == NodeType::Binary && x.sub == ASTITCH_MUL && x.kind == ASTITCH_FULL &&
-              phase_of(a.a) == cur_level) {
+              runs_here(a.a)) {
             if (N(x.b).type == NodeType::Const)
               return "as::ex2(fmaf(" + ref(x.a, "k", sfx) + ", " + flit(N(x.b).cval * 1.4426950408889634) + ", " +
                      nbs + "))";
@@ -1602,7 +1611,7 @@ struct Gen {
       const Node& un = N(u);
       if (un.type == NodeType::Bcast) {
         for (int w : I(u).consumers)
-          if (I(w).live && phase_of(w) >= lv) return true;
+          if (I(w).live && last_run(w) >= lv) return true;
         continue;
       }
       if (un.kind == ASTITCH_COLVEC) {
@@ -1610,7 +1619,7 @@ struct Gen {
         if (read_later(u)) return true;         // same level: computed from it, recursively
         continue;
       }
-      if (phase_of(u) >= lv) return true;       // FULL / ROWVEC consumer in a later sweep
+      if (last_run(u) >= lv) return true;       // FULL / ROWVEC consumer in a later sweep
     }
     return false;
   }

@@ -80,6 +80,7 @@ struct NodeInfo {
   Scheme scheme = Scheme::Local;
   bool global_full = false;    // FULL value buffered in HBM across the barrier
   bool precise_col = false;    // cancellation-prone column value: fp64 sum, applied as hi+lo (R7c)
+  unsigned remat_mask = 0;     // bit L: FULL value recomputed in the sweep of level L (instead of an HBM buffer)
   std::vector<int> consumers;
 };
 
@@ -144,6 +145,7 @@ struct Tuning {
   int prefetch = -1;        // 1: software-prefetch the next rows in the global sweep (off by default)
   int persistent = -1;      // 0: row teams on a non-persistent grid (one row group per CTA)
   int waves = 0;            // packed tiles: grid = waves x the resident CTAs
+  int remat = -1;           // 0: buffer every FULL value read after a barrier in HBM (no recomputation)
   std::string text;         // the string it was parsed from (describe())
 };
 bool parse_tuning(const char* s, Tuning& t, std::string& err);

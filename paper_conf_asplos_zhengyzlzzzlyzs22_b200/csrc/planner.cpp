@@ -161,6 +161,61 @@ void analyse(Plan& p) {
   if (p.max_level > 4)
     throw Error{ASTITCH_ERR_UNSUPPORTED, "more than 4 dependent column reductions (grid barriers)"};
 
+  // Recomputation instead of an HBM buffer (reading R22).  A FULL element-wise
+  // value read in a later barrier level (BatchNorm's centred x, Fig. 7(a)'s
+  // power.1) is, in the paper's global scheme, written to HBM by its own
+  // sweep and read back by the later one: 4 + 4 B per element in fp32.  When
+  // the FULL inputs its element-wise cone starts from cost fewer bytes per
+  // element than that, the later sweep re-reads those inputs and recomputes
+  // the cone instead (row scalars and column values it needs are tiny
+  // buffers).  Same ops in the same order as the buffered value (up to the
+  // compiler's FMA contraction).  Off under FORCE_GLOBAL (the ablation
+  // measures buffering) and with remat=0.
+  auto phase = [&](int u) { return info[u].cls == OpClass::ReduceCol ? info[g.nodes[u].a].level : info[u].level; };
+  if (p.max_level > 0 && !force_global && p.tune.remat != 0) {
+    auto ew_full = [&](int v) {
+      const Node& nd = g.nodes[v];
+      return v >= 0 && info[v].live && nd.kind == ASTITCH_FULL &&
+             (nd.type == NodeType::Unary || nd.type == NodeType::Binary);
+    };
+    for (int v = n - 1; v >= 0; --v) {
+      if (!ew_full(v)) continue;
+      unsigned later = 0;
+      for (int u : info[v].consumers)
+        if (info[u].live && g.nodes[u].type != NodeType::Bcast && info[u].cls != OpClass::ReduceCol &&
+            phase(u) > info[v].level)
+          later |= 1u << phase(u);
+      later |= info[v].remat_mask;  // levels where a recomputed consumer needs it
+      if (!later) continue;
+      // the element-wise cone of v and the FULL inputs it starts from
+      std::vector<int> cone, stack = {v};
+      std::vector<bool> seen(n, false);
+      std::vector<int> leaves;
+      bool ok = true;
+      while (!stack.empty() && ok) {
+        int w = stack.back();
+        stack.pop_back();
+        if (w < 0 || seen[w]) continue;
+        seen[w] = true;
+        const Node& wn = g.nodes[w];
+        if (ew_full(w)) {
+          cone.push_back(w);
+          stack.push_back(wn.a);
+          stack.push_back(wn.b);
+        } else if (wn.type == NodeType::Input && wn.kind == ASTITCH_FULL) {
+          leaves.push_back(w);
+        } else if (wn.kind == ASTITCH_FULL && wn.type != NodeType::Bcast) {
+          ok = false;  // (not reached: FULL values are inputs, broadcasts or element-wise)
+        }
+      }
+      if (!ok || cone.size() > 32) continue;
+      int bytes = 0;
+      for (int x : leaves) bytes += dtype_size(g.nodes[x].dtype);
+      if (bytes >= 8) continue;  // the fp32 buffer's write + read is no more
+      for (int w : cone) info[w].remat_mask |= later;
+    }
+  }
+
   // a2 step 1: dominant candidates = reduces, heavy EW followed by a broadcast,
   // and the outputs of the stitch op.
   std::vector<bool> is_output(n, false);
@@ -261,25 +316,31 @@ void analyse(Plan& p) {
     // (a column reduction accumulates in the sweep of its operand's level:
     // it reads v after the barrier iff that operand sits above v's level,
     // e.g. the broadcast of a row reduction demoted by FORCE_GLOBAL)
-    std::function<bool(int, int)> later_use = [&](int v, int lvl) {
+    // (a consumer also runs in the sweeps that recompute it, R22; a level
+    // where the value itself is recomputed needs no buffer)
+    std::function<bool(int, int, unsigned)> later_use = [&](int v, int lvl, unsigned own) {
       for (int u : info[v].consumers) {
         if (!info[u].live) continue;
         if (g.nodes[u].type == NodeType::Bcast) {
-          if (later_use(u, lvl)) return true;
+          if (later_use(u, lvl, own)) return true;
         } else if (info[u].cls == OpClass::ReduceCol) {
           if (info[g.nodes[u].a].level > lvl) return true;
-        } else if (info[u].level > lvl) {
-          return true;
+        } else {
+          const unsigned runs = (1u << info[u].level) | info[u].remat_mask;
+          if ((runs & ~own) >> (lvl + 1)) return true;
         }
       }
       return false;
     };
-    auto used_after_barrier = [&](int v) { return later_use(v, info[v].level); };
+    auto used_after_barrier = [&](int v) { return later_use(v, info[v].level, info[v].remat_mask); };
     if (c != OpClass::Const && c != OpClass::Input && g.nodes[i].type != NodeType::Bcast &&
         (g.nodes[i].kind == ASTITCH_FULL || g.nodes[i].kind == ASTITCH_ROWVEC) && used_after_barrier(i)) {
       s = Scheme::Global;
       info[i].global_full = true;
     }
+    // crosses the barrier by recomputation from the HBM inputs (R22): still
+    // the global scheme of the paper, without the buffer
+    if (info[i].remat_mask >> (info[i].level + 1) && info[i].candidate) s = Scheme::Global;
     if (c == OpClass::Input && g.nodes[i].kind == ASTITCH_FULL && used_after_barrier(i))
       info[i].global_full = true;  // re-read from HBM after the barrier
     bool has_live_consumer = false;
@@ -1003,7 +1064,15 @@ std::string describe_json(const Plan& p) {
       << ",\"candidate\":" << (in.candidate ? "true" : "false")
       << ",\"dominant\":" << (in.dominant ? "true" : "false")
       << ",\"sub_dominant\":" << (in.sub_dominant ? "true" : "false") << ",\"group\":" << in.group
-      << ",\"scheme\":\"" << scheme_name(in.scheme) << "\"}";
+      << ",\"scheme\":\"" << scheme_name(in.scheme) << "\"";
+    if (in.remat_mask) {  // levels whose sweeps recompute this value (R22)
+      o << ",\"recomputed_at\":[";
+      bool first = true;
+      for (int b = 0; b < 32; ++b)
+        if ((in.remat_mask >> b) & 1u) { o << (first ? "" : ",") << b; first = false; }
+      o << "]";
+    }
+    o << "}";
   }
   o << "],\"groups\":[";
   for (size_t k = 0; k < p.groups.size(); ++k) {

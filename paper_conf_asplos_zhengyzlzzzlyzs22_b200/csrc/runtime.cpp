@@ -223,7 +223,8 @@ bool parse_tuning(const char* s, Tuning& t, std::string& err) {
         {"tile_rows", &t.tile_rows}, {"tile_threads", &t.tile_threads}, {"split", &t.split},
         {"split_threads", &t.split_threads}, {"stream", &t.stream}, {"stage", &t.stage},
         {"stage_kb", &t.stage_kb}, {"portable_clusters", &t.portable_clusters},
-        {"sync", &t.sync}, {"prefetch", &t.prefetch}, {"persistent", &t.persistent}, {"waves", &t.waves}};
+        {"sync", &t.sync}, {"prefetch", &t.prefetch}, {"persistent", &t.persistent}, {"waves", &t.waves},
+        {"remat", &t.remat}};
     bool found = false;
     for (auto& kv : keys)
       if (key == kv.k) { *kv.f = iv; found = true; }

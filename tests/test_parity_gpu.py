@@ -575,6 +575,55 @@ def _virtual_ranks(spec, x, world):
     return ranks
 
 
+@pytest.mark.parametrize("cfg,rows,cols,far", [("bn", 3001, 96, False), ("bn", 2, 4513, True), ("bn", 20011, 256, True),
+                                               ("fig7a", 4099, 200, False), ("fig7a", 37, 1025, False)])
+def test_parity_recompute_vs_buffer_r22(cfg, rows, cols, far):
+    """Reading R22: a FULL value read after a later barrier is recomputed from
+    the re-read inputs (default) instead of buffered in HBM (remat=0); both
+    plans meet the oracle rule, including column means far from the spread
+    (R7c's hi + lo column values feed the recomputed centred x)."""
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    x = gen.generate(cfg, spec)
+    if far:
+        x["x"] = (3.0e4 + 0.01 * x["x"].astype(np.float64)).astype(np.float32)
+    ref = evaluate(spec, x)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    got0, plan0 = run_gpu(spec, x, return_plan=True, tune="remat=0")
+    assert plan.describe()["workspace"]["total"] < plan0.describe()["workspace"]["total"]   # no R x C buffer
+    assert any(o.get("recomputed_at") for o in plan.describe()["ops"])
+    _compare(spec, got, ref)
+    _compare(spec, got0, ref)
+
+
+def test_parity_recompute_masked_random_graphs():
+    """R22 on seeded random two-level graphs with key-padding masks (the mask
+    is re-applied to the re-read inputs of the recomputing sweep)."""
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    from workloads.random_graphs import random_graph
+    found = []
+    for seed in range(3000, 6000):       # host planning only: pick masked graphs that recompute
+        rng = np.random.default_rng(seed)
+        spec = random_graph(seed, int(rng.integers(50, 3000)), int(rng.integers(8, 700)), wide=True)
+        if not spec.get("mask"):
+            continue
+        try:
+            d = A.Plan(A.Graph.from_spec(spec), spec["rows"], spec["cols"], device=-1,
+                       flags=A.FLAG_NO_COMPILE).describe()
+        except A.AstitchError:
+            continue
+        if any(o.get("recomputed_at") for o in d["ops"]):
+            found.append((seed, spec))
+        if len(found) == 5:
+            break
+    assert len(found) == 5
+    for seed, spec in found:
+        x = gen.generate("fig6a", spec)
+        got = run_gpu(spec, x)
+        ref = evaluate(spec, x)
+        for name, dt in spec["outputs"]:
+            check_close(got[name], ref[name], dt, 10 * spec_tol(spec), name=f"seed {seed}:{name}", atol=1e-5)
+
+
 def test_nan_propagation_r12_sharded_and_chunked():
     """R12 across the row-sharded and chunked paths: a column whose only NaN
     sits in one rank's (or one chunk's) rows must come out NaN.  Stage 0 stores

@@ -89,8 +89,11 @@ def test_fig5_heavy_producer_once_per_row():
 def test_fig7a_schemes_match_paper():
     """P:L198: regional for reduce.1, global for power.1 and reduce.2,
     independent for multiply.1, local for the others; final dominants reduce.1
-    and reduce.2, sub-dominants power.1 and multiply.1."""
-    d, ops, _ = describe("fig7a")
+    and reduce.2, sub-dominants power.1 and multiply.1.  The paper's
+    global scheme buffers power.1 in HBM: the plan with recomputation off
+    (remat=0)."""
+    d, ops, _ = describe("fig7a", tune="remat=0")
+    assert d["global_fulls"] == [ops["power1"]["id"]] and "recomputed_at" not in ops["power1"]
     assert ops["reduce1"]["scheme"] == "regional"
     assert ops["power1"]["scheme"] == "global"
     assert ops["reduce2"]["scheme"] == "global"
@@ -101,6 +104,34 @@ def test_fig7a_schemes_match_paper():
     assert ops["power1"]["sub_dominant"] and ops["multiply1"]["sub_dominant"]
     assert len(d["groups"]) == 2
     assert d["needs_sweep2"] and d["kernel_count"] == 1
+
+
+def test_fig7a_power1_recomputed_not_buffered():
+    """Reading R22 (default plan): power.1 still crosses the barrier (global
+    scheme), but the level-1 sweep re-reads x (4 B / element) and recomputes
+    add.1 and power.1 instead of writing and re-reading an fp32 buffer (8 B);
+    only the row scalar divide.1 is buffered (R floats + its lo part)."""
+    d, ops, _ = describe("fig7a")
+    assert ops["power1"]["scheme"] == "global" and ops["power1"]["recomputed_at"] == [1]
+    assert ops["add1"]["recomputed_at"] == [1] and ops["add1"]["scheme"] == "local"
+    assert d["global_fulls"] == [ops["divide1"]["id"]] and ops["divide1"]["scheme"] == "global"
+    assert ops["reduce1"]["scheme"] == "regional" and ops["multiply1"]["scheme"] == "independent"
+    # BatchNorm: the centred x of the variance level is recomputed for the
+    # normalising sweep (level 2), no FULL buffer at all
+    d, ops, _ = describe("bn", rows=100_000, cols=256)
+    assert d["global_fulls"] == [] and ops["xc"]["recomputed_at"] == [2]
+    # two fp32 inputs (8 B) cost as much as the buffer: buffered
+    spec = {"name": "two_in", "rows": 5000, "cols": 64, "inputs": [("x", "FULL", "F32"), ("y", "FULL", "F32")],
+            "mask": None, "ops": [("xy", "binary", "MUL", "x", "y"), ("s", "reduce", "SUM", "COL", "xy"),
+                                  ("sb", "broadcast", "COL", "s"), ("o", "binary", "SUB", "xy", "sb")],
+            "outputs": [("o", "F32")]}
+    g = A.Graph.from_spec(spec)
+    d = A.Plan(g, 5000, 64, device=-1, flags=A.FLAG_NO_COMPILE).describe()
+    assert d["global_fulls"] == [g.names["xy"]]
+    spec["inputs"] = [("x", "FULL", "BF16"), ("y", "FULL", "BF16")]
+    g = A.Graph.from_spec(spec)
+    d = A.Plan(g, 5000, 64, device=-1, flags=A.FLAG_NO_COMPILE).describe()
+    assert d["global_fulls"] == [] and d["ops"][g.names["xy"]]["recomputed_at"] == [1]
 
 
 def test_fig6_selector_branches():
@@ -151,12 +182,16 @@ def test_remote_stitching_one_kernel():
 
 def test_batchnorm_two_barrier_levels():
     """Dependent column reductions (BatchNorm: mean, then variance): levels
-    1 and 2, the centred values buffered in HBM (global), one kernel."""
-    d, ops, p = describe("bn")
+    1 and 2, the centred values read again after the 2nd barrier (global:
+    buffered in HBM with remat=0, recomputed from x by default, R22), one
+    kernel."""
+    d, ops, p = describe("bn", tune="remat=0")
     assert ops["s1"]["class"] == "reduce_col" and ops["s2"]["class"] == "reduce_col"
     assert ops["s1"]["scheme"] == "global" and ops["s2"]["scheme"] == "global"
     assert ops["xc"]["scheme"] == "global"                 # read again after the 2nd barrier
     assert len(d["global_fulls"]) == 1
+    d, ops, p = describe("bn")
+    assert ops["xc"]["scheme"] == "global" and d["global_fulls"] == []
     assert d["kernel_count"] == 1 and d["mapping"]["template"] == "global_sweep"
     # per level: partials -> barrier -> finalise -> barrier (publish) -> next sweep
     assert p.source(0).count("as::grid_barrier(bar);") == 4
