@@ -1426,6 +1426,132 @@ struct Gen {
     o << "  }\n";
   }
 
+  // ------------------------------------------------------------ tma_sweep
+  // Global sweep with address-ordered dynamic row tiles (reading R23): a
+  // producer warp takes tile indices from a workspace counter and stages the
+  // tile's rows of every FULL input in a ring of shared-memory stages with
+  // bulk copies (cp.async.bulk, mbarrier complete_tx); the compute teams read
+  // their rows from shared memory, store FULL outputs from registers, sum
+  // each column over their rows of the tile in fp32 (fixed order) and
+  // deposit that tile partial into an exact binned accumulator (as::bins_add),
+  // so the column totals do not depend on which CTA took which tile.
+  // Column MAX is order-independent as it is (nmax).
+  bool binned(int id) const { return m.tma_sweep && N(id).sub != ASTITCH_RMAX; }
+  void emit_tma_sweep() {
+    cur_level = 0;
+    collect_streams(false);
+    const int TR = m.tma_rows, S = m.tma_stages, TM = RPB;
+    const int CT = TM * T;  // compute threads (the producer warp follows)
+    std::vector<long long> soff(streams.size()), rb(streams.size());
+    long long stage_bytes = 0;
+    for (size_t s = 0; s < streams.size(); ++s) {
+      rb[s] = C * dtype_size(streams[s].dt);
+      soff[s] = static_cast<long long>(S) * TR * stage_bytes;  // placeholder, fixed below
+      stage_bytes += rb[s];
+    }
+    // ring layout: stream s occupies S x TR rows starting at S * TR * (sum of earlier row bytes)
+    {
+      long long acc = 0;
+      for (size_t s = 0; s < streams.size(); ++s) { soff[s] = static_cast<long long>(S) * TR * acc; acc += rb[s]; }
+    }
+    o << "  constexpr int TR = " << TR << ", NSTG = " << S << ", CT = " << CT << ";\n";
+    o << "  extern __shared__ __align__(128) unsigned char tma_smem[];\n";
+    o << "  __shared__ __align__(8) unsigned long long tma_full[NSTG], tma_empty[NSTG];\n";
+    o << "  __shared__ int tma_tile[NSTG];\n";
+    o << "  unsigned int* tctr = (unsigned int*)((char*)p.ws + " << (p.ws.barrier + 64) << "LL);\n";
+    o << "  const int NTILES = (int)((R + TR - 1) / TR);\n";
+    o << "  const unsigned sbase_ = as::smem_addr(tma_smem);\n";
+    o << "  if (threadIdx.x == 0) {\n    for (int s = 0; s < NSTG; ++s) { as::mbar_init(as::smem_addr(&tma_full[s]), 1u); "
+         "as::mbar_init(as::smem_addr(&tma_empty[s]), (unsigned)(CT / 32)); }\n    as::fence_mbar_init();\n  }\n";
+    o << "  __syncthreads();\n";
+    // accumulators that live across tiles
+    for (int id : p.colreds) {
+      if (binned(id)) {
+        o << "  int bJ" << id << " = AS_BIN_EMPTY;\n  long long bh" << id << "[NE], bl" << id << "[NE];\n  float bs" << id
+          << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) { bh" << id << "[k] = 0; bl" << id << "[k] = 0; bs" << id
+          << "[k] = 0.f; }\n";
+      } else {
+        o << "  float acc" << id << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) acc" << id << "[k] = -AS_INF;\n";
+      }
+    }
+    // producer: one elected thread of the extra warp
+    o << "  if (threadIdx.x >= CT) {\n    if (threadIdx.x == CT) {\n";
+    o << "      for (int kt = 0;; ++kt) {\n";
+    o << "        const int st = kt % NSTG;\n";
+    o << "        if (kt >= NSTG) as::mbar_wait(as::smem_addr(&tma_empty[st]), (unsigned)((kt / NSTG - 1) & 1));\n";
+    o << "        const int tile = (int)atomicAdd(tctr, 1u);\n";
+    o << "        tma_tile[st] = tile;\n";
+    o << "        const unsigned fb = as::smem_addr(&tma_full[st]);\n";
+    o << "        if (tile >= NTILES) { asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(fb) : \"memory\"); break; }\n";
+    o << "        const int trows = min(TR, R - tile * TR);\n";
+    o << "        as::mbar_expect_tx(fb, (unsigned)(trows * " << stage_bytes << "LL));\n";
+    for (size_t s = 0; s < streams.size(); ++s) {
+      o << "        as::bulk_g2s(as::smem_addr(tma_smem + " << soff[s] << "LL + (long long)st * TR * " << rb[s]
+        << "LL), (const char*)p.in[" << N(streams[s].node).input_index << "] + (long long)tile * TR * " << rb[s]
+        << "LL, (unsigned)(trows * " << rb[s] << "LL), fb);\n";
+    }
+    o << "      }\n    }\n  } else {\n";
+    // consumers
+    o << "  for (int kt = 0;; ++kt) {\n";
+    o << "    const int st = kt % NSTG;\n";
+    o << "    as::mbar_wait(as::smem_addr(&tma_full[st]), (unsigned)((kt / NSTG) & 1));\n";
+    o << "    const int tile = tma_tile[st];\n";
+    o << "    if (tile >= NTILES) break;\n";
+    o << "    const int trows = min(TR, R - tile * TR);\n";
+    for (int id : p.colreds)
+      if (binned(id))
+        o << "    float acc" << id << "[NE];\n#pragma unroll\n    for (int k = 0; k < NE; ++k) acc" << id << "[k] = 0.f;\n";
+    o << "#pragma unroll\n    for (int rr_ = 0; rr_ < TR / RPB; ++rr_) {\n";
+    o << "    const int rl_ = team + RPB * rr_;\n";
+    o << "    const int row0 = tile * TR + rl_;\n";
+    o << "    const bool act0 = rl_ < trows;\n";
+    o << "    const int lim0 = (int)C;\n    (void)lim0;\n";
+    for (size_t s = 0; s < streams.size(); ++s) {
+      o << "    " << raw_t(streams[s]) << " r" << s << "_u0[V];\n";
+      o << "    r" << s << "_u0[0] = act0 ? as::lds_chunk<" << nb(streams[s].dt) << ">(sbase_ + (unsigned)(" << soff[s]
+        << "LL + ((long long)st * TR + rl_) * " << rb[s] << "LL + (long long)lane * " << nb(streams[s].dt) << ")) : "
+        << raw_t(streams[s]) << "{};\n";
+    }
+    emit_row_block(false, "_u0", "row0", "act0", "lim0");
+    o << "    }\n";
+    // release the stage, then deposit the tile partials
+    o << "    __syncwarp();\n    if ((threadIdx.x & 31) == 0) asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(as::smem_addr(&tma_empty[st])) : \"memory\");\n";
+    for (int id : p.colreds)
+      if (binned(id)) o << "    as::bins_add<NE>(bJ" << id << ", bh" << id << ", bl" << id << ", bs" << id << ", acc" << id << ");\n";
+    o << "  }\n  }\n";
+    // CTA combine (teams in order) -> partial slot of this CTA; the ring is free now
+    const int ncr = static_cast<int>(p.colreds.size());
+    const int NS = nslots();
+    o << "  {\n    char* part = (char*)p.ws + " << p.ws.partials << "LL;\n";
+    for (int q = 0; q < ncr; ++q) {
+      int id = p.colreds[q];
+      o << "    __syncthreads();\n";
+      if (binned(id)) {
+        o << "    {\n      as::BinSlot* sc_ = (as::BinSlot*)tma_smem;  // [team][lane][k]\n";
+        o << "      if (threadIdx.x < CT) {\n#pragma unroll\n        for (int k = 0; k < NE; ++k) { as::BinSlot b_; b_.J = bJ" << id
+          << "; b_.sp = bs" << id << "[k]; b_.hi = bh" << id << "[k]; b_.lo = bl" << id << "[k]; b_.pad = 0; sc_[(team * T + lane) * NE + k] = b_; }\n      }\n";
+        o << "      __syncthreads();\n";
+        o << "      for (int c_ = threadIdx.x; c_ < (int)C; c_ += blockDim.x) {\n";
+        o << "        const int l_ = c_ / E, k_ = c_ % E;\n";
+        o << "        as::BinSlot a_ = sc_[l_ * NE + k_];\n";
+        o << "        for (int t_ = 1; t_ < RPB; ++t_) { const as::BinSlot b_ = sc_[(t_ * T + l_) * NE + k_]; "
+             "as::bins_merge(a_.J, a_.hi, a_.lo, a_.sp, b_.J, b_.hi, b_.lo, b_.sp); }\n";
+        o << "        ((as::BinSlot*)part)[((long long)blockIdx.x * " << NS << " + " << q << ") * C + c_] = a_;\n";
+        o << "      }\n    }\n";
+      } else {
+        o << "    {\n      float* sc_ = (float*)tma_smem;\n";
+        o << "      if (threadIdx.x < CT) {\n#pragma unroll\n        for (int k = 0; k < NE; ++k) sc_[(team * T + lane) * NE + k] = acc" << id
+          << "[k];\n      }\n      __syncthreads();\n";
+        o << "      for (int c_ = threadIdx.x; c_ < (int)C; c_ += blockDim.x) {\n";
+        o << "        const int l_ = c_ / E, k_ = c_ % E;\n        float a_ = sc_[l_ * NE + k_];\n";
+        o << "        for (int t_ = 1; t_ < RPB; ++t_) a_ = as::nmax(a_, sc_[(t_ * T + l_) * NE + k_]);\n";
+        o << "        ((as::BinSlot*)part)[((long long)blockIdx.x * " << NS << " + " << q << ") * C + c_].sp = a_;\n";
+        o << "      }\n    }\n";
+      }
+    }
+    o << "  }\n";
+  }
+
   // partial rows of column `col` combined by the finalise: every CTA's, or
   // (column slabs) the CTAs of col's slab, r = slab + k * NSLAB, in k order
   std::string fin_r0() const { return slab ? "(int)(col / SLABW) + pi * NSLAB" : "pi"; }
@@ -1454,6 +1580,27 @@ struct Gen {
       if (phase_of(id) != cur_level) continue;
       bool mx = N(id).sub == ASTITCH_RMAX;
       std::string ident = mx ? "-AS_INF" : "0.f";
+      if (binned(id)) {  // tma_sweep: merge the CTAs' binned accumulators (exact, any order: R23)
+        o << "      float t" << id << ";\n      {\n";
+        o << "        as::BinSlot a_; a_.J = AS_BIN_EMPTY; a_.sp = 0.f; a_.hi = 0; a_.lo = 0; a_.pad = 0;\n";
+        o << "        if (own) for (int r = pi; r < G; r += P) { const as::BinSlot b_ = as::ld_cg_bins((const as::BinSlot*)part + ((long long)r * "
+          << NS << " + " << q << ") * C + col); as::bins_merge(a_.J, a_.hi, a_.lo, a_.sp, b_.J, b_.hi, b_.lo, b_.sp); }\n";
+        o << "        as::BinSlot* fs_ = (as::BinSlot*)tma_smem;\n        fs_[threadIdx.x] = a_;\n        __syncthreads();\n";
+        o << "        for (int s = P / 2; s > 0; s /= 2) {\n          if (pi < s) { as::BinSlot c_ = fs_[threadIdx.x]; const as::BinSlot d_ = fs_[threadIdx.x + s]; "
+             "as::bins_merge(c_.J, c_.hi, c_.lo, c_.sp, d_.J, d_.hi, d_.lo, d_.sp); fs_[threadIdx.x] = c_; }\n          __syncthreads();\n        }\n";
+        o << "        const as::BinSlot r_ = fs_[threadIdx.x - pi];\n        __syncthreads();\n";
+        o << "        t" << id << " = (float)as::bins_value_d(r_.J, r_.hi, r_.lo, r_.sp);\n      }\n";
+        continue;
+      }
+      if (m.tma_sweep) {  // tma_sweep column MAX: the CTA maxima sit in the slots' sp words
+        o << "      float t" << id << " = -AS_INF;\n";
+        o << "      if (own) for (int r = pi; r < G; r += P) t" << id << " = as::nmax(t" << id
+          << ", as::ld_cg(&((const as::BinSlot*)part + ((long long)r * " << NS << " + " << q << ") * C + col)->sp));\n";
+        o << "      fin_smem[threadIdx.x] = t" << id << ";\n      __syncthreads();\n";
+        o << "      for (int s = P / 2; s > 0; s /= 2) { if (pi < s) fin_smem[threadIdx.x] = as::nmax(fin_smem[threadIdx.x], fin_smem[threadIdx.x + s]); __syncthreads(); }\n";
+        o << "      t" << id << " = fin_smem[threadIdx.x - pi];\n      __syncthreads();\n";
+        continue;
+      }
       if (pc(id)) {  // fp64 combine of the hi + lo partials (R7c)
         o << "      double t" << id << "d = 0.0;\n";
         o << "      if (own) for (int r = " << fin_r0() << "; r < G; r += " << fin_rs() << ") t" << id
@@ -2135,6 +2282,26 @@ struct Gen {
       o << "  const unsigned int xgen = *(volatile unsigned int*)((unsigned char*)p.xbuf + " << kXGen << ") + 1u;\n";
       o << "  if (blockIdx.x == 0 && threadIdx.x == 0) *(volatile unsigned int*)((unsigned char*)p.xbuf + " << kXErr
         << ") = 0u;\n";
+    }
+    if (m.tma_sweep && role != ROLE_SHARD_SWEEP2) {
+      // tma_sweep: one barrier level (planner), sweep -> CTA partials -> grid
+      // barrier -> finalise (+ fused exchange)
+      emit_colvecs(false);
+      emit_pre_colvec_outputs();
+      emit_tma_sweep();
+      o << "  as::grid_barrier(bar);\n";
+      // every producer has taken its last tile: reset the counter for the next run
+      o << "  if (blockIdx.x == 0 && threadIdx.x == 0) *tctr = 0u;\n";
+      if (role == ROLE_SHARD_MAIN) {
+        emit_column_finalize(false);
+      } else if (role == ROLE_FUSED) {
+        emit_column_finalize(false);
+        emit_fused_exchange();
+      } else {
+        emit_column_finalize(true);
+      }
+      o << "}\n";
+      return o.str();
     }
     if (role == ROLE_SHARD_SWEEP2) {  // sharded plans have one barrier level
       cur_level = 1;

@@ -119,6 +119,14 @@ struct Mapping {
   int64_t vertical_trips = 1;
   double lane_util = 1.0;
   int smem_bytes = 0;       // dynamic shared memory per block
+  // GlobalSweep as tma_sweep: row tiles of tma_rows rows staged in a ring of
+  // tma_stages shared-memory stages by bulk copies (UBLKCP) that one producer
+  // warp issues for tiles taken from a workspace counter (address order);
+  // rows_per_block teams of T lanes compute from shared memory; column sums
+  // in exact binned accumulators (order-independent, reading R23)
+  bool tma_sweep = false;
+  int tma_rows = 0;
+  int tma_stages = 0;
   int bank_conflict_ways = 1;
   std::string reason;       // selector decision trace
 };
@@ -146,6 +154,8 @@ struct Tuning {
   int persistent = -1;      // 0: row teams on a non-persistent grid (one row group per CTA)
   int waves = 0;            // packed tiles: grid = waves x the resident CTAs
   int remat = -1;           // 0: buffer every FULL value read after a barrier in HBM (no recomputation)
+  int tma = -1;             // 0: never plan a global sweep as tma_sweep, 1: whenever eligible (default)
+  int tma_rows = 0, tma_stages = 0, tma_teams = 0;  // tma_sweep tile rows / ring stages / compute teams
   std::string text;         // the string it was parsed from (describe())
 };
 bool parse_tuning(const char* s, Tuning& t, std::string& err);

@@ -632,6 +632,91 @@ __device__ __forceinline__ void grid_barrier(u32* bar) {
 // L2-coherent load of data written earlier in the same kernel by other blocks
 __device__ __forceinline__ float ld_cg(const float* p) { return __ldcg(p); }
 
+// ------------------------------------------------------------------ global: exact binned column sums
+// Order-independent column sums for sweeps whose row tiles are handed out
+// dynamically (tma_sweep, reading R23): which CTA sums which tile depends on
+// scheduling, so an fp32 accumulator would round differently run to run.
+// Instead every deposit x (an fp32 tile partial) is added EXACTLY to two
+// int64 bins of a 64-bit fixed-point window aligned to multiples of 32 bits:
+// |x| = m * 2^(bi - 160) with m the 24-bit significand and bi = biased
+// exponent + 10; window J holds bits [32J, 32J + 64) (lo bin: [32J, 32J+32),
+// hi bin: [32J+32, 32J+64)); x contributes its truncation (toward zero) at
+// the window's bottom, slice by slice, sign applied.  The window only moves
+// up (to fit the largest |x| seen: J = (e + 1) >> 5), dropping the lo bin;
+// slices never carry between bins, so the total is
+//   sum over deposits of trunc(x at the FINAL window),
+// the final window being that of the largest |x| anywhere: independent of
+// the deposit order and of how deposits are split across threads and CTAs.
+// Inf / NaN deposits go to an fp32 side sum (any mix of +-inf / NaN sums to
+// the same value in any order).  Precision: >= 32 bits below the largest
+// deposit per deposit (fp32 tile partials carry 24).
+#define AS_BIN_EMPTY (-1000)
+template <int NE>
+__device__ __forceinline__ void bins_add(int& J, long long* hi, long long* lo, float* sp, const float* x) {
+  u32 mx = 0u;  // largest finite |x| bit pattern (monotone in |x|)
+#pragma unroll
+  for (int k = 0; k < NE; ++k) {
+    const u32 a = __float_as_uint(x[k]) & 0x7fffffffu;
+    mx = max(mx, a < 0x7f800000u ? a : 0u);
+  }
+  if (mx != 0u) {
+    const int need = (int)(max(mx >> 23, 1u) + 1u) >> 5;
+    if (need > J) {
+      if (need == J + 1) {
+#pragma unroll
+        for (int k = 0; k < NE; ++k) { lo[k] = hi[k]; hi[k] = 0; }
+      } else {
+#pragma unroll
+        for (int k = 0; k < NE; ++k) { lo[k] = 0; hi[k] = 0; }
+      }
+      J = need;
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < NE; ++k) {
+    const u32 u = __float_as_uint(x[k]);
+    const u32 e = (u >> 23) & 0xffu;
+    if (e == 0xffu) { sp[k] += x[k]; continue; }
+    const u32 m = (u & 0x7fffffu) | (e ? 0x800000u : 0u);
+    const int d = min((int)(e ? e : 1u) + 10 - 32 * J, 40);  // bit offset of m in the window (<= 40)
+    const u64 v = d >= 0 ? ((u64)m << d) : (d > -24 ? (u64)(m >> (-d)) : 0ull);
+    const long long vl = (long long)(v & 0xffffffffull), vh = (long long)(v >> 32);
+    if (u >> 31) { lo[k] -= vl; hi[k] -= vh; } else { lo[k] += vl; hi[k] += vh; }
+  }
+}
+// merge accumulator (J2, hi2, lo2, sp2) into (J, hi, lo, sp): align both to
+// the higher window (dropping whole bins), then add exactly
+__device__ __forceinline__ void bins_merge(int& J, long long& hi, long long& lo, float& sp, int J2, long long hi2,
+                                           long long lo2, float sp2) {
+  sp += sp2;
+  if (J2 > J) {
+    if (J2 == J + 1) { lo = hi; hi = 0; } else { lo = 0; hi = 0; }
+    J = J2;
+  }
+  if (J2 == J) { hi += hi2; lo += lo2; }
+  else if (J2 == J - 1) { lo += hi2; }
+}
+// the accumulator's value: one fp64 rounding of the exact total, then fp32
+__device__ __forceinline__ double bins_value_d(int J, long long hi, long long lo, float sp) {
+  if (sp != 0.f) return (double)sp;  // +-inf or NaN deposits decide (finite parts cannot change them)
+  if (J == AS_BIN_EMPTY) return 0.0;
+  return ldexp((double)hi, 32 * (J + 1) - 160) + ldexp((double)lo, 32 * J - 160);
+}
+// one accumulator in the workspace (32 bytes: J, sp, hi, lo)
+struct BinSlot { int J; float sp; long long hi, lo, pad; };
+// L2-coherent load of a slot written by another CTA earlier in the kernel
+__device__ __forceinline__ BinSlot ld_cg_bins(const BinSlot* p) {
+  const Raw<16> a = ldg_cg(reinterpret_cast<const Raw<16>*>(p));
+  const Raw<8> b = ldg_cg(reinterpret_cast<const Raw<8>*>(p) + 2);
+  BinSlot s;
+  s.J = static_cast<int>(a.x);
+  s.sp = __uint_as_float(a.y);
+  s.hi = static_cast<long long>((static_cast<u64>(a.w) << 32) | a.z);
+  s.lo = static_cast<long long>((static_cast<u64>(b.y) << 32) | b.x);
+  s.pad = 0;
+  return s;
+}
+
 // ------------------------------------------------------------------ packed: TMA bulk + mbarrier
 __device__ __forceinline__ u32 smem_addr(const void* p) {
   return static_cast<u32>(__cvta_generic_to_shared(p));

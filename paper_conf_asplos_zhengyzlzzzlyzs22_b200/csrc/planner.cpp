@@ -599,6 +599,72 @@ void select_mapping(Plan& p) {
     }
     why << (has_colred ? "column reduce -> global sweep (vertical packing, grid barrier); "
                        : "FORCE_GLOBAL: row reductions demoted to global (HBM + grid barrier); ");
+    // tma_sweep (reading R23): element-wise + column-reduction graphs with one
+    // barrier level.  Row tiles are staged in shared memory by bulk copies
+    // (UBLKCP) that one producer warp issues for tiles taken from a counter in
+    // address order; the teams compute from shared memory.  Measured on B200
+    // (scripts/micro/tma_stream.cu, c5_dyn.cu): address-ordered tiles move
+    // C5's 2R:1W mix at 7.0 TB/s where any static ownership of rows (register
+    // or bulk-copy loads alike) stays at 6.5-6.6.  Dynamic ownership makes
+    // per-CTA fp32 column partials scheduling-dependent, so column sums go
+    // to exact binned accumulators (bins_add): the totals stay bitwise
+    // deterministic (R13).  Each lane owns E = 4 columns (8 B bf16 / 16 B
+    // fp32 chunks; E = 8 past 2048 columns), teams of T = C / E lanes share
+    // the tile's rows (TR / teams rows per lane per tile, one deposit each).
+    {
+      // one sweep: every FULL value and every column reduction's operand at
+      // level 0 (column values after the barrier are per-column epilogue work)
+      bool one_sweep = true;
+      for (size_t i = 0; i < g.nodes.size(); ++i) {
+        if (!p.info[i].live) continue;
+        if (g.nodes[i].kind == ASTITCH_FULL && p.info[i].level > 0) one_sweep = false;
+        if (p.info[i].cls == OpClass::ReduceCol && p.info[g.nodes[i].a].level > 0) one_sweep = false;
+      }
+      bool ok = tu.tma != 0 && !no_tma && has_colred && one_sweep && !has_rowred && !has_rowvec &&
+                !has_mask && !ragged && m.nslab == 1 && p.n_precise_colreds == 0 && p.global_fulls.empty() &&
+                R < (1LL << 30) && (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0 && es_max <= 4;
+      int64_t rowbytes = 0;
+      for (int id : g.inputs) {
+        const Node& nd = g.nodes[id];
+        if (nd.kind != ASTITCH_FULL || !p.info[id].live) continue;
+        if ((C * dtype_size(nd.dtype)) % 16) ok = false;  // bulk copies: 16-byte rows
+        rowbytes += C * dtype_size(nd.dtype);
+      }
+      const int Et = C / 4 > 512 ? 8 : 4;
+      ok = ok && rowbytes > 0 && C % Et == 0 && (C / Et) % 32 == 0 && C / Et <= 512;
+      if (ok) {
+        const int T = static_cast<int>(C / Et);
+        const int TM = (tu.tma_teams >= 1 && tu.tma_teams * T <= 1024) ? tu.tma_teams : std::max(1, 512 / T);
+        const int S = (tu.tma_stages >= 2 && tu.tma_stages <= 8) ? tu.tma_stages : 3;
+        const int64_t budget = p.smem_optin - 8 * 1024;  // static smem: barriers, finalise scratch
+        int64_t TR = std::min<int64_t>(64, budget / (S * rowbytes));
+        if (tu.tma_rows > 0) TR = tu.tma_rows;
+        TR -= TR % TM;
+        const int64_t ring = S * TR * rowbytes;
+        // the CTA combine of the teams' accumulators reuses the ring
+        const int64_t comb = static_cast<int64_t>(TM) * T * (Et * 20 + 4);
+        if (TR >= std::max(4, TM) && ring <= budget && ring >= comb) {
+          m.tma_sweep = true;
+          m.vec_elems = E = Et;
+          m.chunks = static_cast<int>(C / Et);
+          m.team = T;
+          m.chunks_per_lane = 1;
+          m.lane_util = 1.0;
+          m.rows_per_block = TM;
+          m.threads = TM * T + 32;  // + one producer warp
+          m.row_unroll = 1;
+          m.prefetch = false;
+          m.hoist_colvec = true;
+          m.tma_rows = static_cast<int>(TR);
+          m.tma_stages = S;
+          m.smem_bytes = static_cast<int>(ring);
+          m.blocks_per_sm = 1;
+          why << "tma_sweep: " << TR << "-row tiles x " << S << " stages (" << ring << " B smem), " << TM
+              << " teams x " << T << " lanes x " << Et << " columns, producer warp, address-ordered tiles, exact "
+              << "binned column sums (R23); ";
+        }
+      }
+    }
   } else {
     // ---------------------------------------------------------- row-wise
     // Masked rows: a chunk index spans T*E columns across the team, and the
@@ -894,6 +960,12 @@ void retune_grid(Plan& p) {
     int64_t clusters = std::max<int64_t>(1, std::min(work_units, wave / m.split));
     m.grid = clusters * m.split;
     m.vertical_trips = (work_units + clusters - 1) / clusters;
+  } else if (m.tmpl == Template::GlobalSweep && m.tma_sweep) {
+    // one CTA per SM (the ring fills its shared memory); tiles are taken
+    // from the counter, so the grid never needs more CTAs than tiles
+    const int64_t tiles = (R + m.tma_rows - 1) / m.tma_rows;
+    m.grid = std::max<int64_t>(1, std::min<int64_t>(tiles, wave));
+    m.vertical_trips = (tiles + m.grid - 1) / m.grid;
   } else if (m.tmpl == Template::GlobalSweep && m.nslab > 1) {
     // column slabs: nslab CTAs per row group, grid a multiple of nslab
     const int64_t groups = std::max<int64_t>(1, std::min(work_units, wave / m.nslab));
@@ -924,10 +996,10 @@ void retune_grid(Plan& p) {
   // block barrier per row step of a persistent multi-trip sweep (the CTA's
   // warps stay on the same rows): default for the global sweep (measured on
   // B200); tuning sync=0/1 overrides
-  m.sync_steps = (m.tmpl == Template::GlobalSweep) && m.vertical_trips >= 32 && !m.prefetch;
+  m.sync_steps = (m.tmpl == Template::GlobalSweep) && m.vertical_trips >= 32 && !m.prefetch && !m.tma_sweep;
   if (p.tune.sync >= 0)
     m.sync_steps = p.tune.sync == 1 && m.vertical_trips > 1 &&
-                   (m.tmpl == Template::GlobalSweep || m.tmpl == Template::RowTeam);
+                   (m.tmpl == Template::GlobalSweep || m.tmpl == Template::RowTeam) && !m.tma_sweep;
   plan_workspace(p);
 }
 
@@ -944,7 +1016,8 @@ void plan_workspace(Plan& p) {
     const int64_t nparts = p.map.grid;
     // partial slots: one per column reduction + a lo slot per precise sum (R7c)
     const size_t nslots = p.colreds.size() + static_cast<size_t>(p.n_precise_colreds);
-    off = align(off + static_cast<size_t>(nparts) * nslots * C * 4);
+    // (tma_sweep: a 32-byte binned accumulator per slot and column, as::BinSlot)
+    off = align(off + static_cast<size_t>(nparts) * nslots * C * (p.map.tma_sweep ? 32 : 4));
     w.colvals = off;
     // [post COLVEC hi][rank-local column totals][post COLVEC lo (R7c)]
     bool any_precise_post = false;
@@ -1119,7 +1192,8 @@ std::string describe_json(const Plan& p) {
     << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"sync_steps\":" << (m.sync_steps ? "true" : "false") << ",\"nslab\":" << m.nslab << ",\"nonpersistent\":" << (m.nonpersistent ? "true" : "false")
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
-    << ",\"grid\":" << m.grid
+    << ",\"tma_sweep\":" << (m.tma_sweep ? "true" : "false") << ",\"tma_rows\":" << m.tma_rows
+    << ",\"tma_stages\":" << m.tma_stages << ",\"grid\":" << m.grid
     << ",\"blocks_per_sm\":" << m.blocks_per_sm << ",\"reg_cap\":" << m.reg_cap
     << ",\"vertical_trips\":" << m.vertical_trips << ",\"smem_bytes\":" << m.smem_bytes
     << ",\"lds128_conflict_ways\":" << m.bank_conflict_ways << ",\"reason\":\"" << esc(m.reason)

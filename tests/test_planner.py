@@ -352,6 +352,9 @@ def test_global_sweep_block_combine_fits_smem():
         s = specs.get(name, rows=rows, cols=cols)
         d = A.Plan(A.Graph.from_spec(s), rows, cols, device=-1, flags=A.FLAG_NO_COMPILE).describe()
         m = d["mapping"]
+        if m["tma_sweep"]:  # the bulk-copy ring fills one CTA's shared memory (the combine reuses it)
+            assert m["smem_bytes"] <= 227 * 1024 - 8 * 1024 and m["blocks_per_sm"] == 1, (name, cols, m)
+            continue
         assert m["smem_bytes"] <= 96 * 1024, (name, cols, m)
         assert m["rows_per_block"] == 1 or m["smem_bytes"] > 0
 
