@@ -1467,9 +1467,9 @@ struct Gen {
     // accumulators that live across tiles
     for (int id : p.colreds) {
       if (binned(id)) {
-        o << "  int bJ" << id << " = AS_BIN_EMPTY;\n  long long bh" << id << "[NE], bl" << id << "[NE];\n  float bs" << id
-          << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) { bh" << id << "[k] = 0; bl" << id << "[k] = 0; bs" << id
-          << "[k] = 0.f; }\n";
+        o << "  int bJ" << id << "[NE];\n  long long bh" << id << "[NE], bl" << id << "[NE];\n  float bs" << id
+          << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) { bJ" << id << "[k] = AS_BIN_EMPTY; bh" << id << "[k] = 0; bl" << id
+          << "[k] = 0; bs" << id << "[k] = 0.f; }\n";
       } else {
         o << "  float acc" << id << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) acc" << id << "[k] = -AS_INF;\n";
       }
@@ -1529,7 +1529,7 @@ struct Gen {
       if (binned(id)) {
         o << "    {\n      as::BinSlot* sc_ = (as::BinSlot*)tma_smem;  // [team][lane][k]\n";
         o << "      if (threadIdx.x < CT) {\n#pragma unroll\n        for (int k = 0; k < NE; ++k) { as::BinSlot b_; b_.J = bJ" << id
-          << "; b_.sp = bs" << id << "[k]; b_.hi = bh" << id << "[k]; b_.lo = bl" << id << "[k]; b_.pad = 0; sc_[(team * T + lane) * NE + k] = b_; }\n      }\n";
+          << "[k]; b_.sp = bs" << id << "[k]; b_.hi = bh" << id << "[k]; b_.lo = bl" << id << "[k]; b_.pad = 0; sc_[(team * T + lane) * NE + k] = b_; }\n      }\n";
         o << "      __syncthreads();\n";
         o << "      for (int c_ = threadIdx.x; c_ < (int)C; c_ += blockDim.x) {\n";
         o << "        const int l_ = c_ / E, k_ = c_ % E;\n";

@@ -645,40 +645,31 @@ __device__ __forceinline__ float ld_cg(const float* p) { return __ldcg(p); }
 // up (to fit the largest |x| seen: J = (e + 1) >> 5), dropping the lo bin;
 // slices never carry between bins, so the total is
 //   sum over deposits of trunc(x at the FINAL window),
-// the final window being that of the largest |x| anywhere: independent of
+// the final window being that of the column's largest |x|: independent of
 // the deposit order and of how deposits are split across threads and CTAs.
+// One window per column (a column's precision never depends on another's).
 // Inf / NaN deposits go to an fp32 side sum (any mix of +-inf / NaN sums to
 // the same value in any order).  Precision: >= 32 bits below the largest
 // deposit per deposit (fp32 tile partials carry 24).
 #define AS_BIN_EMPTY (-1000)
 template <int NE>
-__device__ __forceinline__ void bins_add(int& J, long long* hi, long long* lo, float* sp, const float* x) {
-  u32 mx = 0u;  // largest finite |x| bit pattern (monotone in |x|)
-#pragma unroll
-  for (int k = 0; k < NE; ++k) {
-    const u32 a = __float_as_uint(x[k]) & 0x7fffffffu;
-    mx = max(mx, a < 0x7f800000u ? a : 0u);
-  }
-  if (mx != 0u) {
-    const int need = (int)(max(mx >> 23, 1u) + 1u) >> 5;
-    if (need > J) {
-      if (need == J + 1) {
-#pragma unroll
-        for (int k = 0; k < NE; ++k) { lo[k] = hi[k]; hi[k] = 0; }
-      } else {
-#pragma unroll
-        for (int k = 0; k < NE; ++k) { lo[k] = 0; hi[k] = 0; }
-      }
-      J = need;
-    }
-  }
+__device__ __forceinline__ void bins_add(int* J, long long* hi, long long* lo, float* sp, const float* x) {
 #pragma unroll
   for (int k = 0; k < NE; ++k) {
     const u32 u = __float_as_uint(x[k]);
-    const u32 e = (u >> 23) & 0xffu;
-    if (e == 0xffu) { sp[k] += x[k]; continue; }
+    const u32 a = u & 0x7fffffffu;
+    if (a >= 0x7f800000u) { sp[k] += x[k]; continue; }  // inf / nan (rare)
+    const u32 e = a >> 23;
+    // window of this column: J = (e + 1) >> 5 fits |x| (top bit <= 32J + 63);
+    // moving up drops the lo bin (one step) or both (more)
+    const int need = a ? (int)(max(e, 1u) + 1u) >> 5 : AS_BIN_EMPTY;
+    if (need > J[k]) {
+      lo[k] = need == J[k] + 1 ? hi[k] : 0;
+      hi[k] = 0;
+      J[k] = need;
+    }
     const u32 m = (u & 0x7fffffu) | (e ? 0x800000u : 0u);
-    const int d = min((int)(e ? e : 1u) + 10 - 32 * J, 40);  // bit offset of m in the window (<= 40)
+    const int d = min((int)(e ? e : 1u) + 10 - 32 * J[k], 40);  // bit offset of m in the window (<= 40)
     const u64 v = d >= 0 ? ((u64)m << d) : (d > -24 ? (u64)(m >> (-d)) : 0ull);
     const long long vl = (long long)(v & 0xffffffffull), vh = (long long)(v >> 32);
     if (u >> 31) { lo[k] -= vl; hi[k] -= vh; } else { lo[k] += vl; hi[k] += vh; }

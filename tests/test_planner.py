@@ -371,3 +371,25 @@ def test_group_mappings_follow_their_dominants():
           "ops": [("e", "unary", "EXP", "x"), ("n", "unary", "NEG", "e")], "outputs": [("n", "F32")]}
     p = A.Plan(A.Graph.from_spec(ew), 100, 64, device=-1, flags=A.FLAG_NO_COMPILE)
     assert all("element-wise only" in x["schedule"] or "dominant" in x for x in p.describe()["group_mappings"])
+
+
+def test_tma_sweep_selection():
+    """tma_sweep (R23) for one-sweep element-wise + column-reduction graphs
+    (C5 and its shapes); not for row reductions (fig7a), dependent column
+    levels (BatchNorm), masks, or when switched off (tuning tma=0, NO_TMA)."""
+    def m(name, rows=4096, cols=None, **kw):
+        s = specs.get(name, rows=rows, cols=cols)
+        return A.Plan(A.Graph.from_spec(s), rows, s["cols"], device=-1, flags=kw.get("flags", A.FLAG_NO_COMPILE),
+                      tune=kw.get("tune")).describe()["mapping"]
+    c5 = m("C5")
+    assert c5["tma_sweep"] and c5["vec_elems"] == 4 and c5["team"] == 256 and c5["rows_per_block"] == 1
+    assert c5["threads"] == 288 and c5["tma_stages"] == 3 and c5["tma_rows"] == 16
+    assert c5["smem_bytes"] == 3 * 16 * 4096 and c5["grid"] == 148
+    assert m("C5", cols=512)["rows_per_block"] == 2                  # >= 8 compute warps
+    assert m("C5", cols=4096)["vec_elems"] == 8                      # > 512 lanes of 4 columns
+    assert not m("C5", cols=100)["tma_sweep"]                        # lanes not a multiple of a warp
+    assert not m("C5", cols=16384)["tma_sweep"]                      # column slabs instead
+    assert not m("C5", tune="tma=0")["tma_sweep"]
+    assert not m("C5", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_TMA)["tma_sweep"]
+    assert not m("fig7a")["tma_sweep"] and not m("bn", rows=3000, cols=128)["tma_sweep"]
+    assert m("C5", rows=7)["grid"] == 1                              # never more CTAs than tiles

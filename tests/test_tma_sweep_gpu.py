@@ -1,0 +1,126 @@
+"""GPU tests of the tma_sweep global sweep (reading R23): address-ordered
+dynamic row tiles staged by bulk copies, column sums in exact binned
+accumulators.  The tile order changes from run to run and with the grid size;
+the column totals must not (bitwise), and must match the fp64 oracle under the
+DESIGN.md rule, including non-finite and extreme-range columns.
+"""
+
+import numpy as np
+import pytest
+
+from oracle import evaluate
+from tests.harness import check_close, run_gpu, spec_tol
+from workloads import gen, specs
+
+pytestmark = pytest.mark.gpu
+
+
+def _plan(spec, **kw):
+    import torch
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    return A.Plan(A.Graph.from_spec(spec), spec["rows"], spec["cols"], device=torch.cuda.current_device(), **kw)
+
+
+def test_tma_sweep_chosen_for_c5():
+    spec = specs.get("C5", rows=4096)
+    m = _plan(spec).describe()["mapping"]
+    assert m["tma_sweep"] and m["template"] == "global_sweep"
+    assert m["threads"] == m["rows_per_block"] * m["team"] + 32   # + the producer warp
+    assert m["blocks_per_sm"] == 1 and m["smem_bytes"] == m["tma_stages"] * m["tma_rows"] * 2 * 1024 * 2
+
+
+@pytest.mark.parametrize("rows", [1, 17, 20011])
+def test_tma_sweep_order_independent_bitwise(rows):
+    """Grids of 148, 37 and 5 CTAs take the tiles in different orders and
+    groupings; the binned totals are identical bit for bit, and so is dz."""
+    spec = specs.get("C5", rows=rows)
+    x = gen.generate("C5", spec)
+    ref = evaluate(spec, x)
+    outs = []
+    for sms in (0, 37, 5):
+        p = _plan(spec, sm_count=sms)
+        assert p.describe()["mapping"]["tma_sweep"]
+        got = run_gpu(spec, x, plan=p)
+        for name, dt in spec["outputs"]:
+            check_close(got[name], ref[name], dt, spec_tol(spec), name=f"C5[{rows}] sms={sms}:{name}")
+        outs.append(got)
+    for got in outs[1:]:
+        for k in got:
+            assert np.array_equal(got[k], outs[0][k]), k
+
+
+def test_tma_sweep_static_sweep_still_correct():
+    """tune tma=0 keeps the register global sweep (static row ownership)."""
+    spec = specs.get("C5", rows=3005)
+    x = gen.generate("C5", spec)
+    ref = evaluate(spec, x)
+    p = _plan(spec, tune="tma=0")
+    assert not p.describe()["mapping"]["tma_sweep"]
+    got = run_gpu(spec, x, plan=p)
+    for name, dt in spec["outputs"]:
+        check_close(got[name], ref[name], dt, spec_tol(spec), name=name)
+
+
+COLSUM = {
+    "name": "colsum_edge", "rows": 2003, "cols": 256,
+    "inputs": [("x", "FULL", "F32")], "mask": None,
+    "ops": [("s", "reduce", "SUM", "COL", "x"), ("m", "reduce", "RMAX", "COL", "x")],
+    "outputs": [("s", "F32"), ("m", "F32")],
+}
+
+
+def test_tma_sweep_extreme_columns():
+    """Non-finite deposits (R12 / R23: +inf, +inf and -inf -> NaN, NaN),
+    huge dynamic range, exact cancellation, zeros and subnormals."""
+    rng = np.random.default_rng(23)
+    R, C = COLSUM["rows"], COLSUM["cols"]
+    x = rng.standard_normal((R, C)).astype(np.float32)
+    x[:, 0] = 1.0
+    x[1234, 0] = 1.0e30                      # window jumps to 2^100 late in the sweep
+    x[5, 1] = 3.0e38; x[6, 1] = -3.0e38       # cancels exactly; the rest is truncated below 2^96
+    x[100, 2] = np.inf
+    x[3, 3] = np.inf; x[2000, 3] = -np.inf    # -> NaN
+    x[77, 4] = np.nan
+    x[:, 5] = 0.0
+    x[:, 6] = np.float32(1e-40)               # subnormal deposits
+    x[:, 7] = np.where(np.arange(R) % 2 == 0, 1.0 + 2.0 ** -20, -1.0).astype(np.float32)
+    x[:, 8] = -np.abs(x[:, 8]) * 1e-30        # tiny, all negative
+    x[:, 9] = np.float32(2.0 ** 60) * np.sign(x[:, 9])
+    xin = {"x": x}
+    p = _plan(COLSUM)
+    assert p.describe()["mapping"]["tma_sweep"]
+    got = run_gpu(COLSUM, xin, plan=p)
+    ref = evaluate(COLSUM, xin)
+    assert np.isposinf(got["s"][2]) and np.isnan(got["s"][3]) and np.isnan(got["s"][4])
+    assert np.isnan(got["m"][4]) and np.isposinf(got["m"][2])
+    assert got["s"][5] == 0.0
+    # exact cases: column 7 = (R // 2 + 1) * 2^-20 exactly, column 0 = 1e30 + (R - 1)
+    assert got["s"][7] == np.float32(ref["s"][7])
+    assert got["s"][0] == np.float32(ref["s"][0])
+    assert got["s"][9] == np.float32(ref["s"][9])
+    for name, dt in COLSUM["outputs"]:
+        check_close(got[name], ref[name], dt, spec_tol(COLSUM), name=name)
+    # columns 1 and 8 compared on their own scale (not floored by the RMS of the huge columns)
+    assert abs(got["s"][8] - ref["s"][8]) <= 1e-5 * abs(ref["s"][8])
+    # column 1: +-3e38 cancel exactly; the standard-normal rest is truncated
+    # at the window of 3e38 (2^128 -> bins from 2^64): the total is 0
+    assert got["s"][1] == 0.0 and abs(ref["s"][1]) < 1e3
+
+
+@pytest.mark.parametrize("cols,dt", [(2048, "BF16"), (4096, "BF16"), (512, "F32"), (384, "F32")])
+def test_tma_sweep_shapes(cols, dt):
+    """E = 4 / 8 lanes, one team (T = 512) or several, fp32 and bf16 rows."""
+    spec = specs.get("C5", rows=997, cols=cols)
+    if dt == "F32":
+        spec["inputs"] = [(n, k, "F32" if k == "FULL" else d) for n, k, d in spec["inputs"]]
+        spec["outputs"] = [(n, "F32") for n, _ in spec["outputs"]]
+    x = gen.generate("C5", spec)
+    ref = evaluate(spec, x)
+    p = _plan(spec)
+    assert p.describe()["mapping"]["tma_sweep"], p.describe()["mapping"]["reason"]
+    got = run_gpu(spec, x, plan=p)
+    for name, d in spec["outputs"]:
+        check_close(got[name], ref[name], d, spec_tol(spec), name=f"{cols}:{name}")
+    again = run_gpu(spec, x, plan=_plan(spec, sm_count=11))
+    for k in got:
+        assert np.array_equal(got[k], again[k]), k
