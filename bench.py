@@ -502,20 +502,37 @@ def main():
     if sp.peer is not None:
         exchange = check_fused_exchange(sp, dev_in[0], plan, ws, exchange)
 
-    # copy-kernel ceiling on the same number of bytes (practical roofline)
+    # copy-kernel ceiling on the same number of bytes (practical roofline),
+    # timed like the step: K launches of the same-bytes copy kernel captured
+    # in a CUDA graph over the same number of rotating buffer sets, so the
+    # small configs' launch / ramp latency is in the ceiling too
     half = (nbytes // 2) // 16 * 16
-    src = torch.empty(half, dtype=torch.uint8, device=f"cuda:{dev}")
-    dst = torch.empty_like(src)
-    for _ in range(3):
-        A.bench_copy(dev, src, dst, half)
-    ce0, ce1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    ce0.record(stream)
-    for _ in range(10):
-        A.bench_copy(dev, src, dst, half)
-    ce1.record(stream)
+    cbufs = [(torch.empty(half, dtype=torch.uint8, device=f"cuda:{dev}"),
+              torch.empty(half, dtype=torch.uint8, device=f"cuda:{dev}")) for _ in range(nsets)]
+    for i in range(3):
+        A.bench_copy(dev, *cbufs[i % nsets], half)
     torch.cuda.synchronize()
-    copy_gbs = 2 * half * 10 / (ce0.elapsed_time(ce1) * 1e-3) / 1e9
-    del src, dst
+    ce0, ce1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    try:
+        cgraph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(cgraph):
+            for i in range(args.steps):
+                A.bench_copy(dev, *cbufs[i % nsets], half)
+        cgraph.replay()
+        torch.cuda.synchronize()
+        ce0.record(stream)
+        cgraph.replay()
+        ce1.record(stream)
+    except Exception:  # pragma: no cover
+        torch.cuda.synchronize()
+        ce0.record(stream)
+        for i in range(args.steps):
+            A.bench_copy(dev, *cbufs[i % nsets], half)
+        ce1.record(stream)
+    torch.cuda.synchronize()
+    copy_us = ce0.elapsed_time(ce1) * 1e3 / args.steps
+    copy_gbs = 2 * half / (copy_us * 1e-6) / 1e9
+    del cbufs
 
     # K steps captured once into a CUDA graph (removes host launch overhead,
     # which otherwise dominates the us-scale configs); eager if capture fails
@@ -710,6 +727,7 @@ def main():
             "pct_of_8TBps": round(100.0 * gbs / world / 8000.0, 2),
             "compulsory_bytes_per_step": int(total_bytes),
             "copy_kernel_gbs": round(copy_gbs, 1),
+            "copy_kernel_us": round(copy_us, 3),
             "pct_of_copy_kernel": round(100.0 * achieved / copy_gbs, 2),
             "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": _traffic(cfg),
