@@ -1552,6 +1552,100 @@ struct Gen {
     o << "  }\n";
   }
 
+  // ------------------------------------------------------------ tma_team
+  // Row teams fed by a producer warp: tiles of TR rows are taken from a
+  // workspace counter (address order); lane r of the producer warp copies
+  // row r's valid prefix of every FULL input (rounded up to 16 bytes) into
+  // its slot of the stage with one bulk copy; the teams read their rows'
+  // chunks from shared memory and run the usual row body (masks, KF
+  // specialisation, stores).  The last CTA to finish resets the counters.
+  void emit_tma_team(const std::string& name) {
+    header(name, false);
+    collect_streams(false);
+    const int TR = m.tma_rows, S = m.tma_stages;
+    const int CT = RPB * T;
+    std::vector<long long> soff(streams.size()), slot(streams.size());
+    long long acc = 0;
+    for (size_t s = 0; s < streams.size(); ++s) {
+      slot[s] = (C * dtype_size(streams[s].dt) + 15) / 16 * 16;
+      soff[s] = static_cast<long long>(S) * TR * acc;
+      acc += slot[s];
+    }
+    emit_colvecs(false);
+    o << "  constexpr int TR = " << TR << ", NSTG = " << S << ", CT = " << CT << ";\n";
+    o << "  extern __shared__ __align__(128) unsigned char tma_smem[];\n";
+    o << "  __shared__ __align__(8) unsigned long long tma_full[NSTG], tma_empty[NSTG];\n";
+    o << "  __shared__ int tma_tile[NSTG];\n";
+    o << "  unsigned int* tctr = (unsigned int*)((char*)p.ws + " << (p.ws.barrier + 64) << "LL);\n";
+    o << "  unsigned int* tdone = (unsigned int*)((char*)p.ws + " << (p.ws.barrier + 68) << "LL);\n";
+    o << "  const int NTILES = (int)((R + TR - 1) / TR);\n";
+    o << "  const unsigned sbase_ = as::smem_addr(tma_smem);\n";
+    o << "  if (threadIdx.x == 0) {\n    for (int s = 0; s < NSTG; ++s) { as::mbar_init(as::smem_addr(&tma_full[s]), 1u); "
+         "as::mbar_init(as::smem_addr(&tma_empty[s]), (unsigned)(CT / 32)); }\n    as::fence_mbar_init();\n  }\n";
+    o << "  __syncthreads();\n";
+    // producer warp: lane r copies row r of the tile
+    o << "  if (threadIdx.x >= CT) {\n    const int pl = threadIdx.x - CT;\n";
+    o << "    for (int kt = 0;; ++kt) {\n";
+    o << "      const int st = kt % NSTG;\n";
+    o << "      if (kt >= NSTG) as::mbar_wait(as::smem_addr(&tma_empty[st]), (unsigned)((kt / NSTG - 1) & 1));\n";
+    o << "      int tile = 0;\n      if (pl == 0) tile = (int)atomicAdd(tctr, 1u);\n";
+    o << "      tile = __shfl_sync(0xffffffffu, tile, 0);\n";
+    o << "      const unsigned fb = as::smem_addr(&tma_full[st]);\n";
+    o << "      if (tile >= NTILES) {\n        if (pl == 0) { tma_tile[st] = tile; asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(fb) : \"memory\"); }\n        break;\n      }\n";
+    o << "      const int prow = tile * TR + pl;\n";
+    o << "      const bool pact = pl < TR && prow < R;\n";
+    o << "      " << limdecl("plim", "pact", "prow") << "\n      (void)plim;\n";
+    o << "      unsigned nbytes_ = 0;\n";
+    for (size_t s = 0; s < streams.size(); ++s) {
+      const int es = dtype_size(streams[s].dt);
+      o << "      const unsigned nb" << s << " = pact ? (unsigned)((min(plim, (int)C) * " << es << " + 15) & ~15) : 0u;\n";
+      o << "      nbytes_ += nb" << s << ";\n";
+    }
+    o << "#pragma unroll\n      for (int o_ = 16; o_ > 0; o_ /= 2) nbytes_ += __shfl_xor_sync(0xffffffffu, nbytes_, o_);\n";
+    o << "      if (pl == 0) { tma_tile[st] = tile; as::mbar_expect_tx(fb, nbytes_); }\n";
+    o << "      __syncwarp();\n";
+    for (size_t s = 0; s < streams.size(); ++s) {
+      o << "      if (nb" << s << ") as::bulk_g2s(sbase_ + (unsigned)(" << soff[s] << "LL + ((long long)st * TR + pl) * " << slot[s]
+        << "LL), (const char*)p.in[" << N(streams[s].node).input_index << "] + (long long)" << rowbase("prow", "plim")
+        << " * " << nb(streams[s].dt) << "LL, nb" << s << ", fb);\n";
+    }
+    o << "    }\n  } else {\n";
+    // consumers
+    o << "  for (int kt = 0;; ++kt) {\n";
+    o << "    const int st = kt % NSTG;\n";
+    o << "    as::mbar_wait(as::smem_addr(&tma_full[st]), (unsigned)((kt / NSTG) & 1));\n";
+    o << "    const int tile = tma_tile[st];\n";
+    o << "    if (tile >= NTILES) break;\n";
+    o << "#pragma unroll 1\n    for (int rr_ = 0; rr_ < TR / RPB; ++rr_) {\n";
+    o << "    const int rl_ = team + RPB * rr_;\n";
+    o << "    const int row0 = tile * TR + rl_;\n";
+    o << "    const bool act0 = row0 < R;\n";
+    // (a per-stage table of the lengths the producer lanes looked up measured
+    // slower on B200, C3 137.8 vs 136.1 us: one more register, a 4-byte spill)
+    o << "    " << limdecl("lim0", "act0", "row0") << "\n    (void)lim0;\n";
+    for (size_t s = 0; s < streams.size(); ++s) {
+      const Stream& stv = streams[s];
+      o << "    " << raw_t(stv) << " r" << s << "_u0[V];\n";
+      o << "#pragma unroll\n    for (int j = 0; j < V; ++j) {\n";
+      o << "      const long long c0 = " << chx("j") << " * E;\n";
+      std::string cond = "act0";
+      if (!exact || masked) cond += " && c0 < lim0";
+      o << "      if (" << cond << ") r" << s << "_u0[j] = as::lds_chunk<" << nb(stv.dt) << ">(sbase_ + (unsigned)(" << soff[s]
+        << "LL + ((long long)st * TR + rl_) * " << slot[s] << "LL + " << chx("j") << " * " << nb(stv.dt) << "LL));\n";
+      if (!absorb) o << "      else r" << s << "_u0[j] = " << raw_t(stv) << "{};\n";
+      o << "    }\n";
+    }
+    emit_row_block(false, "_u0", "row0", "act0", "lim0");
+    o << "    }\n";
+    o << "    __syncwarp();\n    if ((threadIdx.x & 31) == 0) asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(as::smem_addr(&tma_empty[st])) : \"memory\");\n";
+    o << "  }\n  }\n";
+    // the last CTA to finish resets the counters for the next run
+    o << "  __syncthreads();\n";
+    o << "  if (threadIdx.x == 0) {\n    __threadfence();\n    const unsigned d_ = atomicAdd(tdone, 1u);\n";
+    o << "    if (d_ == gridDim.x - 1) { *(volatile unsigned*)tctr = 0u; *(volatile unsigned*)tdone = 0u; __threadfence(); }\n  }\n";
+    o << "}\n";
+  }
+
   // partial rows of column `col` combined by the finalise: every CTA's, or
   // (column slabs) the CTAs of col's slab, r = slab + k * NSLAB, in k order
   std::string fin_r0() const { return slab ? "(int)(col / SLABW) + pi * NSLAB" : "pi"; }
@@ -2239,6 +2333,10 @@ struct Gen {
 
   // ------------------------------------------------------------ roles
   std::string run(const std::string& name) {
+    if (m.tmpl == Template::RowTeam && m.tma_team) {
+      emit_tma_team(name);
+      return o.str();
+    }
     if (m.tmpl == Template::PackedTile) {
       emit_packed(name);
       return o.str();

@@ -125,6 +125,9 @@ struct Mapping {
   // rows_per_block teams of T lanes compute from shared memory; column sums
   // in exact binned accumulators (order-independent, reading R23)
   bool tma_sweep = false;
+  // RowTeam as tma_team: the same producer warp / bulk-copy ring / address-
+  // ordered tiles for row-wise plans; one bulk copy per row (its valid prefix)
+  bool tma_team = false;
   int tma_rows = 0;
   int tma_stages = 0;
   int bank_conflict_ways = 1;
@@ -155,6 +158,7 @@ struct Tuning {
   int waves = 0;            // packed tiles: grid = waves x the resident CTAs
   int remat = -1;           // 0: buffer every FULL value read after a barrier in HBM (no recomputation)
   int tma = -1;             // 0: never plan a global sweep as tma_sweep, 1: whenever eligible (default)
+  int tma_team = -1;        // 1: row-team plans as tma_team, 0: never
   int tma_rows = 0, tma_stages = 0, tma_teams = 0;  // tma_sweep tile rows / ring stages / compute teams
   std::string text;         // the string it was parsed from (describe())
 };

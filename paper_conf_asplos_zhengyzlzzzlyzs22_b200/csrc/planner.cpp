@@ -924,8 +924,51 @@ void select_mapping(Plan& p) {
   // masked softmax, 2 KB of stores per warp step: 24 warps/SM 146 us, 32
   // warps 153.5 us, 16 warps 163 us).  Read-mostly rows (a row sum, fig6a:
   // 64 B of stores per warp step) keep the full occupancy.
+  // tma_team: row teams fed by the tma_sweep machinery -- a producer warp
+  // takes TR-row tiles from a counter in address order and bulk-copies each
+  // row's valid prefix (lane r of the warp: row r of the tile) into a ring of
+  // shared-memory stages; the teams compute from shared memory.  Rows must
+  // start 16-byte aligned in every FULL input.  Default for key-padding
+  // masked rows of >= 512 bytes (measured on B200, C3: 16-row tiles x 4
+  // stages, 3 CTAs/SM, 135.8 us vs 140.4 us for the oversubscribed register
+  // row teams; 1 CTA/SM with 128 KB rings 193 us); opt-in (tuning
+  // tma_team=1) elsewhere: packed varlen rows (C3v) measured equal (78.5 vs
+  // 78.1 us), unmasked rows are not better served than by register rows.
+  const bool tma_team_default = has_mask && !ragged && C * es_min >= 512;
+  if (m.tmpl == Template::RowTeam && (tu.tma_team == 1 || (tu.tma_team != 0 && tma_team_default)) && !no_tma &&
+      R < (1LL << 30) && es_max <= 4) {
+    bool ok = true;
+    int64_t pitch = 0;  // smem bytes of one row slot, all FULL inputs
+    for (int id : g.inputs) {
+      const Node& nd = g.nodes[id];
+      if (nd.kind != ASTITCH_FULL || !p.info[id].live) continue;
+      const int64_t rb = C * dtype_size(nd.dtype);
+      if (!ragged && rb % 16) ok = false;
+      pitch += (rb + 15) / 16 * 16;
+    }
+    const int S = (tu.tma_stages >= 2 && tu.tma_stages <= 8) ? tu.tma_stages : 4;
+    const int teams = (tu.tma_teams >= 1 && tu.tma_teams * m.team <= 1024) ? tu.tma_teams : m.rows_per_block;
+    // 16-row tiles, at least one row per team (<= 32: one producer lane per row)
+    const int TRq = tu.tma_rows > 0 ? tu.tma_rows : std::max(16, teams);
+    const int64_t ring = static_cast<int64_t>(S) * TRq * pitch;
+    if (ok && pitch > 0 && TRq <= 32 && TRq % teams == 0 && ring <= p.smem_optin - 8 * 1024) {
+      m.tma_team = true;
+      m.tma_rows = TRq;
+      m.tma_stages = S;
+      m.rows_per_block = teams;
+      m.threads = teams * m.team + 32;
+      m.row_unroll = 1;
+      m.prefetch = false;
+      m.nonpersistent = false;
+      m.single_wave_bps = 0;
+      m.grid_waves = 0;
+      m.smem_bytes = static_cast<int>(ring);
+      why << "tma_team: " << TRq << "-row tiles x " << S << " stages (" << ring << " B), " << teams << " teams, "
+          << "producer warp (one bulk copy per row), address-ordered tiles; ";
+    }
+  }
   int max_threads_sm = 2048;
-  if (m.tmpl == Template::RowTeam) {
+  if (m.tmpl == Template::RowTeam && !m.tma_team) {
     if (m.single_wave_bps > 0) {
       max_threads_sm = m.single_wave_bps * m.threads;
     } else {
@@ -964,6 +1007,10 @@ void retune_grid(Plan& p) {
     int64_t clusters = std::max<int64_t>(1, std::min(work_units, wave / m.split));
     m.grid = clusters * m.split;
     m.vertical_trips = (work_units + clusters - 1) / clusters;
+  } else if (m.tmpl == Template::RowTeam && m.tma_team) {
+    const int64_t tiles = (R + m.tma_rows - 1) / m.tma_rows;
+    m.grid = std::max<int64_t>(1, std::min<int64_t>(tiles, wave));
+    m.vertical_trips = (tiles + m.grid - 1) / m.grid;
   } else if (m.tmpl == Template::GlobalSweep && m.tma_sweep) {
     // one CTA per SM (the ring fills its shared memory); tiles are taken
     // from the counter, so the grid never needs more CTAs than tiles
@@ -1075,6 +1122,10 @@ void plan_workspace(Plan& p) {
     (void)n;
     p.gbuf_slots = static_cast<int>(slots.size());
     off = align(off + goff);
+  }
+  if (p.map.tmpl == Template::RowTeam && p.map.tma_team) {
+    w.barrier = off;  // [64]: tile counter, [68]: CTAs done (the last one resets both)
+    off = align(off + 256);
   }
   w.total = off;
   p.ws = w;
@@ -1196,7 +1247,8 @@ std::string describe_json(const Plan& p) {
     << ",\"prefetch\":" << (m.prefetch ? "true" : "false") << ",\"single_wave_bps\":" << m.single_wave_bps << ",\"sync_steps\":" << (m.sync_steps ? "true" : "false") << ",\"nslab\":" << m.nslab << ",\"nonpersistent\":" << (m.nonpersistent ? "true" : "false")
     << ",\"hoist_colvec\":" << (m.hoist_colvec ? "true" : "false") << ",\"tile_rows\":" << m.tile_rows
     << ",\"stages\":" << m.stages << ",\"split\":" << m.split << ",\"stage_row\":" << (m.stage_row ? "true" : "false")
-    << ",\"tma_sweep\":" << (m.tma_sweep ? "true" : "false") << ",\"tma_rows\":" << m.tma_rows
+    << ",\"tma_sweep\":" << (m.tma_sweep ? "true" : "false") << ",\"tma_team\":" << (m.tma_team ? "true" : "false")
+    << ",\"tma_rows\":" << m.tma_rows
     << ",\"tma_stages\":" << m.tma_stages << ",\"grid\":" << m.grid
     << ",\"blocks_per_sm\":" << m.blocks_per_sm << ",\"reg_cap\":" << m.reg_cap
     << ",\"vertical_trips\":" << m.vertical_trips << ",\"smem_bytes\":" << m.smem_bytes

@@ -224,7 +224,7 @@ bool parse_tuning(const char* s, Tuning& t, std::string& err) {
         {"split_threads", &t.split_threads}, {"stream", &t.stream}, {"stage", &t.stage},
         {"stage_kb", &t.stage_kb}, {"portable_clusters", &t.portable_clusters},
         {"sync", &t.sync}, {"prefetch", &t.prefetch}, {"persistent", &t.persistent}, {"waves", &t.waves},
-        {"remat", &t.remat}, {"tma", &t.tma}, {"tma_rows", &t.tma_rows}, {"tma_stages", &t.tma_stages}, {"tma_teams", &t.tma_teams}};
+        {"remat", &t.remat}, {"tma", &t.tma}, {"tma_rows", &t.tma_rows}, {"tma_stages", &t.tma_stages}, {"tma_teams", &t.tma_teams}, {"tma_team", &t.tma_team}};
     bool found = false;
     for (auto& kv : keys)
       if (key == kv.k) { *kv.f = iv; found = true; }

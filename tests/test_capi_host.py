@@ -148,7 +148,10 @@ def test_io_signature_and_workspace():
     spec = specs.get("C3", rows=8192)
     p = A.Plan(A.Graph.from_spec(spec), 8192, 512, device=-1, flags=A.FLAG_NO_COMPILE)
     assert p.inputs == [("FULL", "BF16"), ("LENGTHS", "I32")]
-    assert p.workspace_bytes() == 0
+    assert p.workspace_bytes() == 256                       # tma_team: tile counter + done counter
+    spec = specs.get("C2", rows=4096)
+    p = A.Plan(A.Graph.from_spec(spec), 4096, 768, device=-1, flags=A.FLAG_NO_COMPILE)
+    assert p.workspace_bytes() == 0                         # register row teams need none
 
 
 def test_binding_checks_tensors_against_the_plan():

@@ -141,8 +141,10 @@ def test_fig6_selector_branches():
     # light rows: one row group per CTA on a non-persistent grid (the block
     # scheduler orders the sweep); heavier rows: a persistent one-wave grid
     assert m["nonpersistent"] and m["grid"] * m["rows_per_block"] >= 750_000 and m["vertical_trips"] == 1
-    d, _, _ = describe("C3")      # masked rows: persistent prefetching teams, ~8 row steps per CTA
-    assert not d["mapping"]["nonpersistent"] and 6 <= d["mapping"]["vertical_trips"] <= 10
+    d, _, _ = describe("C3")      # masked rows: tma_team, 16-row tiles, one wave of ring CTAs
+    m = d["mapping"]
+    assert m["tma_team"] and m["tma_rows"] == 16 and m["tma_stages"] == 4 and not m["nonpersistent"]
+    assert m["threads"] == m["rows_per_block"] * m["team"] + 32 and m["grid"] == 148 * m["blocks_per_sm"]
     d, _, _ = describe("C2", rows=65536)   # heavy unmasked rows: one persistent wave
     assert d["mapping"]["grid"] <= d["mapping"]["blocks_per_sm"] * 148
     # <64,30000>: the paper's shape rule holds, but 120 KB rows are below the

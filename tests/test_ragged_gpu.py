@@ -38,11 +38,11 @@ def _valid_index(spec, x, E):
     return np.concatenate(valid), np.concatenate(tail)
 
 
-def _run(spec, x, fill):
+def _run(spec, x, fill, tune=None):
     import torch
     import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
     g = A.Graph.from_spec(spec)
-    plan = A.Plan(g, spec["rows"], spec["cols"], device=torch.cuda.current_device())
+    plan = A.Plan(g, spec["rows"], spec["cols"], device=torch.cuda.current_device(), tune=tune)
     ins = [to_torch(x[n], d) for n, _, d in spec["inputs"]]
     outs = plan.alloc_outputs()
     for o in outs:
@@ -52,9 +52,9 @@ def _run(spec, x, fill):
     return plan, outs
 
 
-def _check(spec, x, E=8):
+def _check(spec, x, E=8, tune=None):
     import torch
-    plan, outs = _run(spec, x, 0xFF)
+    plan, outs = _run(spec, x, 0xFF, tune=tune)
     ref = evaluate(spec, x)
     valid, tail = _valid_index(spec, x, E)
     for (name, dt), o in zip(spec["outputs"], outs):

@@ -124,3 +124,42 @@ def test_tma_sweep_shapes(cols, dt):
     again = run_gpu(spec, x, plan=_plan(spec, sm_count=11))
     for k in got:
         assert np.array_equal(got[k], again[k]), k
+
+
+# ---------------------------------------------------------------- tma_team
+@pytest.mark.parametrize("cfg,rows,cols,tune", [
+    ("C3", 3 * 256 + 7, None, "tma_team=1"), ("C3", 2048, None, "tma_team=1,tma_teams=32"),
+    ("C3", 1000, None, "tma_team=1,tma_rows=16,tma_stages=2"),
+    ("C3", 1000, None, "tma_team=1,tma_rows=16,tma_stages=4"),
+    ("C1", None, None, "tma_team=1"), ("C1", 50000, 128, "tma_team=1"),
+    ("C2", 300, 256, "tma_team=1"), ("C4", 20003, 36, "tma_team=1")])
+def test_tma_team_parity(cfg, rows, cols, tune):
+    """Row teams fed by the producer warp (one bulk copy per row's valid
+    prefix, address-ordered tiles) match the oracle, run after run."""
+    spec = specs.get(cfg, rows=rows, cols=cols)
+    if spec.get("mask"):
+        spec["mask"]["rows_per_segment"] = 256
+    if spec.get("segments"):
+        spec["segments"]["heads"] = 2
+        spec = gen.ragged_spec(spec, 3)
+    x = gen.generate(cfg, spec)
+    p = _plan(spec, tune=tune)
+    m = p.describe()["mapping"]
+    if m["template"] == "row_team":
+        assert m["tma_team"], m["reason"]
+    got = run_gpu(spec, x, plan=p)
+    ref = evaluate(spec, x)
+    for name, dt in spec["outputs"]:
+        check_close(got[name], ref[name], dt, spec_tol(spec), name=f"{cfg}:{name}")
+    again = run_gpu(spec, x, plan=p)
+    for k in got:
+        assert np.array_equal(got[k], again[k]), k
+
+
+@pytest.mark.parametrize("lengths,heads", [([37, 1, 8, 9, 64, 511, 512, 200], 2), ([100, 300, 37], 40)])
+def test_tma_team_ragged(lengths, heads):
+    from tests.test_ragged_gpu import _check, _spec
+    spec = _spec(lengths, heads=heads)
+    x = gen.generate("C3v", spec)
+    plan = _check(spec, x, tune="tma_team=1")
+    assert plan.describe()["mapping"]["tma_team"]
