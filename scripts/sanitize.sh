@@ -9,7 +9,7 @@ run() {  # tool config rows cols [flags] [tune]
      --iters 1 --flags $f ${t:+--tune $t} > gpurun_out/sanitize_$tag.txt 2>&1
   echo "$1 $2 [$3,$4] flags=$f ${t:+tune=$t }exit=$? $(grep -E 'ERROR SUMMARY' gpurun_out/sanitize_$tag.txt | tail -1)"
 }
-for tool in memcheck racecheck synccheck; do
+for tool in ${TOOLS:-memcheck racecheck synccheck}; do
   run $tool C1 37 129                      # row team, ragged
   run $tool C3 8192 512                    # masked row team, oversubscribed grid
   run $tool C4 5003 36                     # TMA packed tiles, tail tile, oversubscribed grid
@@ -21,4 +21,8 @@ for tool in memcheck racecheck synccheck; do
   run $tool bn 3000 96                     # three sweeps, fp64 column means (R7c)
   run $tool C4 3000 36 2                   # FORCE_GLOBAL: hi+lo ROWVEC buffers across barriers
   run $tool fig6a 50001 32                 # non-persistent row teams
+  run $tool C5 4099 1024 0 tma=0           # static register global sweep (tma_sweep off)
+  run $tool C5 997 4096                    # tma_sweep E=8, one team of 512 lanes
+  run $tool C3 4099 512 0 tma_team=0       # masked register row teams (tma_team off)
+  run $tool C1 5000 128 0 tma_team=1       # tma_team, unmasked rows, tail tile
 done
