@@ -1572,6 +1572,7 @@ struct Gen {
       acc += slot[s];
     }
     emit_colvecs(false);
+    emit_pre_colvec_outputs();  // COLVEC outputs of the row plan (block 0; fuzz seeds 4039 / 4161)
     o << "  constexpr int TR = " << TR << ", NSTG = " << S << ", CT = " << CT << ";\n";
     o << "  extern __shared__ __align__(128) unsigned char tma_smem[];\n";
     o << "  __shared__ __align__(8) unsigned long long tma_full[NSTG], tma_empty[NSTG];\n";

@@ -645,8 +645,9 @@ void select_mapping(Plan& p) {
         if (tu.tma_rows > 0) TR = tu.tma_rows;
         TR -= TR % TM;
         const int64_t ring = S * TR * rowbytes;
-        // the CTA combine of the teams' accumulators reuses the ring
-        const int64_t comb = static_cast<int64_t>(TM) * T * (Et * 20 + 4);
+        // the CTA combine of the teams' accumulators (one 32-byte as::BinSlot
+        // per lane column) and the finalise scratch reuse the ring
+        const int64_t comb = std::max<int64_t>(static_cast<int64_t>(TM) * T * Et * 32, (TM * T + 32) * 32);
         if (TR >= std::max(4, TM) && ring <= budget && ring >= comb) {
           m.tma_sweep = true;
           m.vec_elems = E = Et;

@@ -163,3 +163,18 @@ def test_tma_team_ragged(lengths, heads):
     x = gen.generate("C3v", spec)
     plan = _check(spec, x, tune="tma_team=1")
     assert plan.describe()["mapping"]["tma_team"]
+
+
+@pytest.mark.parametrize("seed,rows,cols,rowwise,flags", [(4039, 4606, 256, True, 0), (4161, 24271, 128, False, 64)])
+def test_tma_team_colvec_outputs_fuzz_seeds(seed, rows, cols, rowwise, flags):
+    """Graph-fuzz regressions (round 2, `--tma --wide`): a masked row plan
+    with COLVEC outputs (tanh(cv - cv), sqrt(|cv| + 1)) under tma_team left
+    them unwritten until the pre-barrier column outputs were emitted there."""
+    from workloads.random_graphs import random_graph
+    spec = random_graph(seed, rows, cols, wide=True, rowwise=rowwise)
+    x = gen.generate("fig6a", spec)
+    got, plan = run_gpu(spec, x, return_plan=True, flags=flags)
+    assert plan.describe()["mapping"]["tma_team"]
+    ref = evaluate(spec, x)
+    for name, dt in spec["outputs"]:
+        check_close(got[name], ref[name], dt, spec_tol(spec), name=name, atol=1e-5)

@@ -13,9 +13,11 @@ BINARY = ["ADD", "SUB", "MUL", "MAX", "MIN"]
 
 
 def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide: bool = False,
-                 colred: bool = True, colvec: bool = True) -> dict:
+                 colred: bool = True, colvec: bool = True, rowwise: bool = True) -> dict:
     """wide=True: also random F16 inputs, BF16 / F16 outputs and key-padding
-    masks (the "wide" fuzz); False keeps the round-2 regression seeds stable."""
+    masks (the "wide" fuzz); False keeps the round-2 regression seeds stable.
+    rowwise=False: no ROWVEC input and column reductions only (the one-sweep
+    graphs tma_sweep takes)."""
     rng = np.random.default_rng(seed)
     ops, inputs = [], []
     vals = {"FULL": [], "ROWVEC": [], "COLVEC": []}
@@ -24,7 +26,7 @@ def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide
         n = f"x{i}"
         inputs.append((n, "FULL", str(rng.choice(["F32", "BF16", "F16"] if wide else ["F32", "BF16"]))))
         vals["FULL"].append(n)
-    if rng.random() < 0.5:
+    if rng.random() < 0.5 and rowwise:
         inputs.append(("rv", "ROWVEC", "F32"))
         vals["ROWVEC"].append("rv")
     if rng.random() < 0.5 and colvec:
@@ -74,6 +76,10 @@ def random_graph(seed: int, rows: int, cols: int, n_ops: int | None = None, wide
         elif choice < 0.8 and vals["FULL"]:                  # reduction of a FULL value
             a = str(rng.choice(vals["FULL"]))
             axis = "ROW" if (rng.random() < 0.6 or ncolred >= 2 or not colred) else "COL"
+            if not rowwise:
+                if ncolred >= 2:
+                    continue
+                axis = "COL"
             red = str(rng.choice(["SUM", "RMAX"]))
             r = new("ROWVEC" if axis == "ROW" else "COLVEC")
             ops.append((r, "reduce", red, axis, a))
