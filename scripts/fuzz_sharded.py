@@ -11,9 +11,16 @@ ways the library offers and compared with the fp64 oracle on the whole problem:
   fused   astitch_run_fused: every rank's one cooperative kernel pushes its
           partials into all ranks' exchange slots over (here: local) peer
           memory and combines them in rank order, all ranks running together
-          on their own streams, each plan sized for 148/world SMs.
+          on their own streams, each plan sized for 148/world SMs at ONE
+          block per SM (tune bps=1): the ranks' cooperative grids must be
+          co-resident on ONE GPU, and ranks whose row counts differ (byte-
+          balanced masked shards) may plan different footprints; a rank of
+          2 CTAs/SM spread over 90 SMs left too few whole SMs for two ranks
+          of 1 CTA/SM and their flag waits hit the 5 s bound (seed 5165,
+          world 3 -- a harness artifact: on a multi-GPU box every rank has
+          its own GPU).
 Column outputs must be bitwise equal across ranks.  Masked graphs take mask_row_ranges' shards.
-    python scripts/fuzz_sharded.py SEED0 N"""
+    python scripts/fuzz_sharded.py SEED0 N [--tma]"""
 import os
 import sys
 
@@ -66,8 +73,14 @@ def main():
         world = int(rng.integers(2, 5))
         rows = int(rng.choice([int(rng.integers(world, 200)), int(rng.integers(200, 5000)), int(rng.integers(5000, 30000))]))
         cols = int(rng.choice([int(rng.integers(1, 64)), int(rng.integers(64, 1100)), int(rng.integers(1100, 4000))]))
+        kw = {}
+        if "--tma" in sys.argv:   # column counts / graphs the bulk-copy templates take
+            cols = 128 * int(rng.integers(1, 17))
+            kw = {"rowwise": bool(rng.random() < 0.3)}
         cols = max(1, min(cols, 4_000_000 // rows))
-        spec = random_graph(seed, rows, cols, wide=True)
+        if "--tma" in sys.argv:
+            cols = max(128, cols // 128 * 128)
+        spec = random_graph(seed, rows, cols, wide=True, **kw)
         if spec.get("mask") and -(-rows // spec["mask"]["rows_per_segment"]) < world:
             spec["mask"]["rows_per_segment"] = max(1, rows // world)      # at least one segment per rank
         x = gen.generate("fig6a", spec)
@@ -83,6 +96,7 @@ def main():
                 ranks = []
                 for r in range(world):
                     sp = ShardedPlan(g, rows, cols, world, r, 0, sm_count=sms // world if mode == "fused" else 0,
+                                     tune="bps=1" if mode == "fused" else None,
                                      row_range=rr[r])
                     b, nr = sp.row_begin, sp.row_count
                     ins = device_inputs(dict(spec, rows=nr), shard_inputs(spec, x, b, nr))
@@ -121,7 +135,7 @@ def main():
             cases += 1
             desc = ranks[0]["sp"].plan.describe()
             print(f"ok seed={seed} world={world} [{rows},{cols}] mask={bool(spec.get('mask'))} "
-                  f"{desc['mapping']['template']} shard_kernels={desc['shard_kernels']} max_rel={w:.2e}", flush=True)
+                  f"{desc['mapping']['template']}{'/tma_sweep' if desc['mapping'].get('tma_sweep') else ''}{'/tma_team' if desc['mapping'].get('tma_team') else ''} shard_kernels={desc['shard_kernels']} max_rel={w:.2e}", flush=True)
         except Exception as e:
             if "ASTITCH_ERR_UNSUPPORTED" in str(e):
                 print(f"unsupported seed={seed}: {str(e)[:120]}")
