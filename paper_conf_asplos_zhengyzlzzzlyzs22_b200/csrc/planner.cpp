@@ -952,7 +952,9 @@ void select_mapping(Plan& p) {
     // 16-row tiles, at least one row per team (<= 32: one producer lane per row)
     const int TRq = tu.tma_rows > 0 ? tu.tma_rows : std::max(16, teams);
     const int64_t ring = static_cast<int64_t>(S) * TRq * pitch;
-    if (ok && pitch > 0 && TRq <= 32 && TRq % teams == 0 && ring <= p.smem_optin - 8 * 1024) {
+    // whole compute warps (the producer warp follows them)
+    if (ok && pitch > 0 && TRq <= 32 && TRq % teams == 0 && (teams * m.team) % 32 == 0 &&
+        ring <= p.smem_optin - 8 * 1024) {
       m.tma_team = true;
       m.tma_rows = TRq;
       m.tma_stages = S;
