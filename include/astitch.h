@@ -242,7 +242,11 @@ astitch_status astitch_plan_destroy(astitch_plan_t p);
  * $HOME/.cache/astitch.  A cache hit skips NVRTC; describe()'s plan_time_ms
  * reports the plan's analysis / codegen / NVRTC / load times and the hits. */
 astitch_status astitch_set_cache_dir(const char* dir);
-/* Bytes of device workspace astitch_run needs (0 if none). */
+/* Bytes of device workspace astitch_run needs (0 if none).  Global-stage plans
+ * keep their grid barrier, column partials and buffers there; plans that take
+ * row tiles from a counter (tma_sweep / tma_team, R23) keep the tile
+ * counter there too (reset in-kernel after its last use, so one workspace
+ * serves any number of sequential runs and CUDA-graph replays). */
 astitch_status astitch_plan_workspace_bytes(astitch_plan_t p, size_t* bytes);
 /* JSON description: op classes, dominants, groups, schemes, mapping, grid,
  * smem, registers, kernel count, compulsory bytes.  *len = bytes needed
@@ -260,8 +264,9 @@ astitch_status astitch_plan_io(astitch_plan_t p, int32_t is_output, int32_t inde
                                astitch_kind* kind, astitch_dtype* dtype);
 
 /* ---------------------------------------------------------------- execution */
-/* Initialise a workspace once (zeroes the grid-barrier words).  Not needed
- * between runs: the barrier is generation-counted and self-resetting. */
+/* Initialise a workspace once (zeroes the grid-barrier and tile-counter
+ * words).  Not needed between runs: the barrier is self-resetting and the
+ * tile counters are reset by the kernel that used them. */
 astitch_status astitch_workspace_init(astitch_plan_t p, void* ws, void* stream);
 /* Runs the plan: one stitched kernel launch (cooperative when the plan has a
  * global stage) on `stream`.  inputs/outputs are device pointers in
