@@ -1437,35 +1437,67 @@ struct Gen {
   // so the column totals do not depend on which CTA took which tile.
   // Column MAX is order-independent as it is (nmax).
   bool binned(int id) const { return m.tma_sweep && N(id).sub != ASTITCH_RMAX; }
-  void emit_tma_sweep() {
-    cur_level = 0;
-    collect_streams(false);
-    const int TR = m.tma_rows, S = m.tma_stages, TM = RPB;
-    const int CT = TM * T;  // compute threads (the producer warp follows)
-    std::vector<long long> soff(streams.size()), rb(streams.size());
-    long long stage_bytes = 0;
-    for (size_t s = 0; s < streams.size(); ++s) {
-      rb[s] = C * dtype_size(streams[s].dt);
-      soff[s] = static_cast<long long>(S) * TR * stage_bytes;  // placeholder, fixed below
-      stage_bytes += rb[s];
-    }
-    // ring layout: stream s occupies S x TR rows starting at S * TR * (sum of earlier row bytes)
-    {
-      long long acc = 0;
-      for (size_t s = 0; s < streams.size(); ++s) { soff[s] = static_cast<long long>(S) * TR * acc; acc += rb[s]; }
-    }
+  // prologue (once per kernel): ring, mbarriers, the running stage counters
+  // of the producer (kt_p) and of the consumers (kt_c), which continue across
+  // barrier levels so the mbarrier phases stay in step
+  void emit_tma_prologue() {
+    const int TR = m.tma_rows, S = m.tma_stages;
+    const int CT = RPB * T;  // compute threads (the producer warp follows)
     o << "  constexpr int TR = " << TR << ", NSTG = " << S << ", CT = " << CT << ";\n";
     o << "  extern __shared__ __align__(128) unsigned char tma_smem[];\n";
     o << "  __shared__ __align__(8) unsigned long long tma_full[NSTG], tma_empty[NSTG];\n";
     o << "  __shared__ int tma_tile[NSTG];\n";
-    o << "  unsigned int* tctr = (unsigned int*)((char*)p.ws + " << (p.ws.barrier + 64) << "LL);\n";
     o << "  const int NTILES = (int)((R + TR - 1) / TR);\n";
     o << "  const unsigned sbase_ = as::smem_addr(tma_smem);\n";
+    o << "  int kt_p = 0, kt_c = 0;\n  (void)kt_p; (void)kt_c;\n";
     o << "  if (threadIdx.x == 0) {\n    for (int s = 0; s < NSTG; ++s) { as::mbar_init(as::smem_addr(&tma_full[s]), 1u); "
          "as::mbar_init(as::smem_addr(&tma_empty[s]), (unsigned)(CT / 32)); }\n    as::fence_mbar_init();\n  }\n";
     o << "  __syncthreads();\n";
+  }
+  // does a later barrier level sweep the rows again (FULL values or column
+  // reductions of a later level, recomputed values)?
+  bool sweep_after(int lv) const {
+    for (size_t i = 0; i < g.nodes.size(); ++i) {
+      if (!I(i).live) continue;
+      if (N(i).kind == ASTITCH_FULL && (I(i).level > lv || (I(i).remat_mask >> (lv + 1)) != 0u)) return true;
+      if (I(i).cls == OpClass::ReduceCol && phase_of(static_cast<int>(i)) > lv) return true;
+    }
+    return false;
+  }
+  // the tile counter of barrier level lv; [60]: CTAs done (the last resets them)
+  long long tctr_off(int lv) const { return static_cast<long long>(p.ws.barrier + 64 + 4 * lv); }
+  void emit_tma_epilogue() {
+    o << "  __syncthreads();\n";
+    o << "  if (threadIdx.x == 0) {\n    __threadfence();\n";
+    o << "    const unsigned d_ = atomicAdd((unsigned*)((char*)p.ws + " << (p.ws.barrier + 60) << "LL), 1u);\n";
+    o << "    if (d_ == gridDim.x - 1) {\n";
+    for (int lv = 0; lv <= p.max_level; ++lv)
+      o << "      *(volatile unsigned*)((char*)p.ws + " << tctr_off(lv) << "LL) = 0u;\n";
+    o << "      *(volatile unsigned*)((char*)p.ws + " << (p.ws.barrier + 60) << "LL) = 0u;\n      __threadfence();\n    }\n  }\n";
+  }
+
+  // one sweep (barrier level cur_level) of the tma_sweep: the producer warp
+  // stages this level's row streams (FULL inputs re-read, HBM buffers of
+  // earlier levels), the consumers compute this level's ops, deposit the tile
+  // partials of this level's column reductions, then the CTA combine writes
+  // this CTA's partial slots
+  void emit_tma_level() {
+    const int lv = cur_level;
+    collect_streams(lv > 0);
+    const int TR = m.tma_rows, S = m.tma_stages;
+    std::vector<long long> soff(streams.size()), rb(streams.size());
+    long long stage_bytes = 0;
+    for (size_t s = 0; s < streams.size(); ++s) {
+      rb[s] = C * dtype_size(streams[s].dt);
+      // ring layout: stream s occupies S x TR rows starting at S * TR * (sum of earlier row bytes)
+      soff[s] = static_cast<long long>(S) * TR * stage_bytes;
+      stage_bytes += rb[s];
+    }
+    std::vector<int> crs;
+    for (int id : p.colreds)
+      if (phase_of(id) == lv) crs.push_back(id);
     // accumulators that live across tiles
-    for (int id : p.colreds) {
+    for (int id : crs) {
       if (binned(id)) {
         o << "  int bJ" << id << "[NE];\n  long long bh" << id << "[NE], bl" << id << "[NE];\n  float bs" << id
           << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) { bJ" << id << "[k] = AS_BIN_EMPTY; bh" << id << "[k] = 0; bl" << id
@@ -1474,31 +1506,40 @@ struct Gen {
         o << "  float acc" << id << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) acc" << id << "[k] = -AS_INF;\n";
       }
     }
-    // producer: one elected thread of the extra warp
+    o << "  unsigned int* tctr = (unsigned int*)((char*)p.ws + " << tctr_off(lv) << "LL);\n";
+    // producer: one elected thread of the extra warp (after a level's
+    // barriers: the ring held generic-proxy scratch, order it before the
+    // bulk copies' async-proxy writes)
     o << "  if (threadIdx.x >= CT) {\n    if (threadIdx.x == CT) {\n";
-    o << "      for (int kt = 0;; ++kt) {\n";
-    o << "        const int st = kt % NSTG;\n";
-    o << "        if (kt >= NSTG) as::mbar_wait(as::smem_addr(&tma_empty[st]), (unsigned)((kt / NSTG - 1) & 1));\n";
+    if (lv > 0) o << "      as::fence_proxy_async_smem();\n";
+    o << "      for (;; ++kt_p) {\n";
+    o << "        const int st = kt_p % NSTG;\n";
+    o << "        if (kt_p >= NSTG) as::mbar_wait(as::smem_addr(&tma_empty[st]), (unsigned)((kt_p / NSTG - 1) & 1));\n";
     o << "        const int tile = (int)atomicAdd(tctr, 1u);\n";
     o << "        tma_tile[st] = tile;\n";
     o << "        const unsigned fb = as::smem_addr(&tma_full[st]);\n";
-    o << "        if (tile >= NTILES) { asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(fb) : \"memory\"); break; }\n";
+    o << "        if (tile >= NTILES) { asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(fb) : \"memory\"); ++kt_p; break; }\n";
     o << "        const int trows = min(TR, R - tile * TR);\n";
     o << "        as::mbar_expect_tx(fb, (unsigned)(trows * " << stage_bytes << "LL));\n";
     for (size_t s = 0; s < streams.size(); ++s) {
+      std::string src = streams[s].ws_buf ? "(const char*)p.ws + " + std::to_string(streams[s].ws_off) + "LL"
+                                          : "(const char*)p.in[" + std::to_string(N(streams[s].node).input_index) + "]";
       o << "        as::bulk_g2s(as::smem_addr(tma_smem + " << soff[s] << "LL + (long long)st * TR * " << rb[s]
-        << "LL), (const char*)p.in[" << N(streams[s].node).input_index << "] + (long long)tile * TR * " << rb[s]
-        << "LL, (unsigned)(trows * " << rb[s] << "LL), fb);\n";
+        << "LL), " << src << " + (long long)tile * TR * " << rb[s] << "LL, (unsigned)(trows * " << rb[s] << "LL), fb);\n";
     }
     o << "      }\n    }\n  } else {\n";
     // consumers
-    o << "  for (int kt = 0;; ++kt) {\n";
-    o << "    const int st = kt % NSTG;\n";
-    o << "    as::mbar_wait(as::smem_addr(&tma_full[st]), (unsigned)((kt / NSTG) & 1));\n";
+    o << "  for (;; ++kt_c) {\n";
+    o << "    const int st = kt_c % NSTG;\n";
+    o << "    as::mbar_wait(as::smem_addr(&tma_full[st]), (unsigned)((kt_c / NSTG) & 1));\n";
     o << "    const int tile = tma_tile[st];\n";
-    o << "    if (tile >= NTILES) break;\n";
+    // the sentinel's stage is released too when a later level's producer reuses it
+    if (sweep_after(lv))
+      o << "    if (tile >= NTILES) {\n      __syncwarp();\n      if ((threadIdx.x & 31) == 0) asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(as::smem_addr(&tma_empty[st])) : \"memory\");\n      ++kt_c;\n      break;\n    }\n";
+    else
+      o << "    if (tile >= NTILES) break;\n";
     o << "    const int trows = min(TR, R - tile * TR);\n";
-    for (int id : p.colreds)
+    for (int id : crs)
       if (binned(id))
         o << "    float acc" << id << "[NE];\n#pragma unroll\n    for (int k = 0; k < NE; ++k) acc" << id << "[k] = 0.f;\n";
     o << "#pragma unroll\n    for (int rr_ = 0; rr_ < TR / RPB; ++rr_) {\n";
@@ -1512,19 +1553,21 @@ struct Gen {
         << "LL + ((long long)st * TR + rl_) * " << rb[s] << "LL + (long long)lane * " << nb(streams[s].dt) << ")) : "
         << raw_t(streams[s]) << "{};\n";
     }
-    emit_row_block(false, "_u0", "row0", "act0", "lim0");
+    emit_row_block(lv > 0, "_u0", "row0", "act0", "lim0");
     o << "    }\n";
     // release the stage, then deposit the tile partials
     o << "    __syncwarp();\n    if ((threadIdx.x & 31) == 0) asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(as::smem_addr(&tma_empty[st])) : \"memory\");\n";
-    for (int id : p.colreds)
-      if (binned(id)) o << "    as::bins_add<NE>(bJ" << id << ", bh" << id << ", bl" << id << ", bs" << id << ", acc" << id << ");\n";
+    for (int id : crs)
+      if (binned(id))
+        o << "    as::bins_add<NE>(bJ" << id << ", bh" << id << ", bl" << id << ", bs" << id << ", acc" << id << ");\n";
     o << "  }\n  }\n";
+    if (crs.empty()) return;
     // CTA combine (teams in order) -> partial slot of this CTA; the ring is free now
-    const int ncr = static_cast<int>(p.colreds.size());
     const int NS = nslots();
     o << "  {\n    char* part = (char*)p.ws + " << p.ws.partials << "LL;\n";
-    for (int q = 0; q < ncr; ++q) {
+    for (size_t q = 0; q < p.colreds.size(); ++q) {
       int id = p.colreds[q];
+      if (phase_of(id) != lv) continue;
       o << "    __syncthreads();\n";
       if (binned(id)) {
         o << "    {\n      as::BinSlot* sc_ = (as::BinSlot*)tma_smem;  // [team][lane][k]\n";
@@ -2383,22 +2426,57 @@ struct Gen {
         << ") = 0u;\n";
     }
     if (m.tma_sweep && role != ROLE_SHARD_SWEEP2) {
-      // tma_sweep: one barrier level (planner), sweep -> CTA partials -> grid
-      // barrier -> finalise (+ fused exchange)
+      // tma_sweep: per barrier level, a bulk-copy sweep -> CTA partials ->
+      // grid barrier -> finalise (+ fused exchange) [-> grid barrier when a
+      // later level reads what it published]
       emit_colvecs(false);
       emit_pre_colvec_outputs();
-      emit_tma_sweep();
-      o << "  as::grid_barrier(bar);\n";
-      // every producer has taken its last tile: reset the counter for the next run
-      o << "  if (blockIdx.x == 0 && threadIdx.x == 0) *tctr = 0u;\n";
-      if (role == ROLE_SHARD_MAIN) {
-        emit_column_finalize(false);
-      } else if (role == ROLE_FUSED) {
-        emit_column_finalize(false);
-        emit_fused_exchange();
-      } else {
-        emit_column_finalize(true);
+      emit_tma_prologue();
+      const int D = p.max_level;
+      auto colred_at = [&](int lv) {
+        for (int id : p.colreds)
+          if (phase_of(id) == lv) return true;
+        return false;
+      };
+      auto sweep_at = [&](int lv) {
+        if (lv == 0) return true;
+        for (size_t i = 0; i < g.nodes.size(); ++i)
+          if (I(i).live && I(i).level == lv && N(i).kind == ASTITCH_FULL) return true;
+        for (size_t i = 0; i < g.nodes.size(); ++i)
+          if (I(i).live && N(i).kind == ASTITCH_FULL && ((I(i).remat_mask >> lv) & 1u)) return true;
+        return false;
+      };
+      auto later_work = [&](int lv) {
+        for (int l = lv + 1; l <= D; ++l)
+          if (sweep_at(l) || colred_at(l)) return true;
+        return false;
+      };
+      for (int lv = 0; lv <= D; ++lv) {
+        cur_level = lv;
+        const bool colred_here = colred_at(lv), sweep_here = sweep_at(lv);
+        if (!sweep_here && !colred_here) continue;
+        o << "  {  // ---- level " << lv << "\n";
+        if (lv > 0) emit_post_colvec_loads();
+        emit_tma_level();
+        if (colred_here) {
+          o << "  as::grid_barrier(bar);\n";
+          if (role == ROLE_SHARD_MAIN) {
+            emit_column_finalize(false);
+          } else if (role == ROLE_FUSED) {
+            emit_column_finalize(false);
+            emit_fused_exchange();
+            if (later_work(lv)) o << "  as::grid_barrier(bar);\n";
+          } else {
+            emit_column_finalize(true);
+            if (later_work(lv)) o << "  as::grid_barrier(bar);\n";
+          }
+        } else if (later_work(lv)) {
+          o << "  as::grid_barrier(bar);\n";
+        }
+        o << "  }\n";
+        if (role == ROLE_SHARD_MAIN) break;
       }
+      emit_tma_epilogue();
       o << "}\n";
       return o.str();
     }

@@ -612,16 +612,19 @@ void select_mapping(Plan& p) {
     // fp32 chunks; E = 8 past 2048 columns), teams of T = C / E lanes share
     // the tile's rows (TR / teams rows per lane per tile, one deposit each).
     {
-      // one sweep: every FULL value and every column reduction's operand at
-      // level 0 (column values after the barrier are per-column epilogue work)
+      // barrier levels (dependent column reductions, values read after a
+      // barrier) are swept one after the other by the same ring; sharded
+      // plans keep one sweep per kernel (their level-1 sweep is a separate
+      // role), precise column sums (R7c) need more than the bins' 32 bits
       bool one_sweep = true;
       for (size_t i = 0; i < g.nodes.size(); ++i) {
         if (!p.info[i].live) continue;
         if (g.nodes[i].kind == ASTITCH_FULL && p.info[i].level > 0) one_sweep = false;
         if (p.info[i].cls == OpClass::ReduceCol && p.info[g.nodes[i].a].level > 0) one_sweep = false;
       }
-      bool ok = tu.tma != 0 && !no_tma && has_colred && one_sweep && !has_rowred && !has_rowvec &&
-                !has_mask && !ragged && m.nslab == 1 && p.n_precise_colreds == 0 && p.global_fulls.empty() &&
+      const bool levels_ok = one_sweep || p.desc.shard_world <= 1;
+      bool ok = tu.tma != 0 && !no_tma && has_colred && levels_ok && !has_rowred && !has_rowvec &&
+                !has_mask && !ragged && m.nslab == 1 && p.n_precise_colreds == 0 &&
                 R < (1LL << 30) && (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0 && es_max <= 4;
       int64_t rowbytes = 0;
       for (int id : g.inputs) {
@@ -630,6 +633,8 @@ void select_mapping(Plan& p) {
         if ((C * dtype_size(nd.dtype)) % 16) ok = false;  // bulk copies: 16-byte rows
         rowbytes += C * dtype_size(nd.dtype);
       }
+      // fp32 HBM buffers of values read by later levels (upper bound of any level's streams)
+      rowbytes += static_cast<int64_t>(p.global_fulls.size()) * C * 4;
       const int Et = C / 4 > 512 ? 8 : 4;
       ok = ok && rowbytes > 0 && C % Et == 0 && (C / Et) % 32 == 0 && C / Et <= 512;
       if (ok) {

@@ -178,3 +178,23 @@ def test_tma_team_colvec_outputs_fuzz_seeds(seed, rows, cols, rowwise, flags):
     ref = evaluate(spec, x)
     for name, dt in spec["outputs"]:
         check_close(got[name], ref[name], dt, spec_tol(spec), name=name, atol=1e-5)
+
+
+@pytest.mark.parametrize("seed,rows,cols", [(704, 5000, 512), (1004, 20011, 256), (1190, 37, 1024)])
+def test_tma_sweep_barrier_levels(seed, rows, cols):
+    """tma_sweep over dependent barrier levels (a value read after a column
+    reduction's barrier, buffered in HBM or recomputed): the same ring and
+    mbarriers carry on across levels (the sentinel's stage released, a proxy
+    fence before the next level's bulk copies), one tile counter per level."""
+    from workloads.random_graphs import random_graph
+    spec = random_graph(seed, rows, cols, rowwise=False)
+    x = gen.generate("fig6a", spec)
+    got, plan = run_gpu(spec, x, return_plan=True)
+    d = plan.describe()
+    assert d["mapping"]["tma_sweep"]
+    ref = evaluate(spec, x)
+    for name, dt in spec["outputs"]:
+        check_close(got[name], ref[name], dt, spec_tol(spec), name=name, atol=1e-5)
+    again = run_gpu(spec, x, plan=plan)
+    for k in got:
+        assert np.array_equal(got[k], again[k]), k
