@@ -1437,6 +1437,12 @@ struct Gen {
   // so the column totals do not depend on which CTA took which tile.
   // Column MAX is order-independent as it is (nmax).
   bool binned(int id) const { return m.tma_sweep && N(id).sub != ASTITCH_RMAX; }
+  // byte address of (CTA g, partial slot q, column col) in the tma_sweep
+  // partial region (48-byte slots: as::BinSlot / as::BinSlotP / an fp32 max)
+  std::string slot_at(const std::string& base, const std::string& gi, int q, const std::string& col) const {
+    return "((const char*)(" + base + ") + (((long long)(" + gi + ") * " + std::to_string(nslots()) + " + " +
+           std::to_string(q) + ") * C + (" + col + ")) * 48LL)";
+  }
   // prologue (once per kernel): ring, mbarriers, the running stage counters
   // of the producer (kt_p) and of the consumers (kt_c), which continue across
   // barrier levels so the mbarrier phases stay in step
@@ -1498,7 +1504,11 @@ struct Gen {
       if (phase_of(id) == lv) crs.push_back(id);
     // accumulators that live across tiles
     for (int id : crs) {
-      if (binned(id)) {
+      if (binned(id) && pc(id)) {  // precise (R7c): fp64 tile partials, 4 x 16-bit bins
+        o << "  int bJ" << id << "[NE];\n  long long bq" << id << "[NE * 4];\n  float bs" << id
+          << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) { bJ" << id << "[k] = AS_BIN_EMPTY; bs" << id
+          << "[k] = 0.f; bq" << id << "[4 * k] = bq" << id << "[4 * k + 1] = bq" << id << "[4 * k + 2] = bq" << id << "[4 * k + 3] = 0; }\n";
+      } else if (binned(id)) {
         o << "  int bJ" << id << "[NE];\n  long long bh" << id << "[NE], bl" << id << "[NE];\n  float bs" << id
           << "[NE];\n#pragma unroll\n  for (int k = 0; k < NE; ++k) { bJ" << id << "[k] = AS_BIN_EMPTY; bh" << id << "[k] = 0; bl" << id
           << "[k] = 0; bs" << id << "[k] = 0.f; }\n";
@@ -1541,7 +1551,8 @@ struct Gen {
     o << "    const int trows = min(TR, R - tile * TR);\n";
     for (int id : crs)
       if (binned(id))
-        o << "    float acc" << id << "[NE];\n#pragma unroll\n    for (int k = 0; k < NE; ++k) acc" << id << "[k] = 0.f;\n";
+        o << "    " << (pc(id) ? "double" : "float") << " acc" << id << "[NE];\n#pragma unroll\n    for (int k = 0; k < NE; ++k) acc" << id
+          << "[k] = 0;\n";
     o << "#pragma unroll\n    for (int rr_ = 0; rr_ < TR / RPB; ++rr_) {\n";
     o << "    const int rl_ = team + RPB * rr_;\n";
     o << "    const int row0 = tile * TR + rl_;\n";
@@ -1557,19 +1568,34 @@ struct Gen {
     o << "    }\n";
     // release the stage, then deposit the tile partials
     o << "    __syncwarp();\n    if ((threadIdx.x & 31) == 0) asm volatile(\"mbarrier.arrive.shared::cta.b64 _, [%0];\" ::\"r\"(as::smem_addr(&tma_empty[st])) : \"memory\");\n";
-    for (int id : crs)
-      if (binned(id))
+    for (int id : crs) {
+      if (binned(id) && pc(id))
+        o << "    as::bins_add_p<NE>(bJ" << id << ", bq" << id << ", bs" << id << ", acc" << id << ");\n";
+      else if (binned(id))
         o << "    as::bins_add<NE>(bJ" << id << ", bh" << id << ", bl" << id << ", bs" << id << ", acc" << id << ");\n";
+    }
     o << "  }\n  }\n";
     if (crs.empty()) return;
     // CTA combine (teams in order) -> partial slot of this CTA; the ring is free now
-    const int NS = nslots();
     o << "  {\n    char* part = (char*)p.ws + " << p.ws.partials << "LL;\n";
     for (size_t q = 0; q < p.colreds.size(); ++q) {
       int id = p.colreds[q];
       if (phase_of(id) != lv) continue;
       o << "    __syncthreads();\n";
-      if (binned(id)) {
+      if (binned(id) && pc(id)) {
+        o << "    {\n      as::BinSlotP* sc_ = (as::BinSlotP*)tma_smem;  // [team][lane][k]\n";
+        o << "      if (threadIdx.x < CT) {\n#pragma unroll\n        for (int k = 0; k < NE; ++k) { as::BinSlotP b_; b_.J = bJ" << id
+          << "[k]; b_.sp = bs" << id << "[k]; b_.pad = 0;\n#pragma unroll\n          for (int q_ = 0; q_ < 4; ++q_) b_.b[q_] = bq" << id
+          << "[4 * k + q_];\n          sc_[(team * T + lane) * NE + k] = b_; }\n      }\n";
+        o << "      __syncthreads();\n";
+        o << "      for (int c_ = threadIdx.x; c_ < (int)C; c_ += blockDim.x) {\n";
+        o << "        const int l_ = c_ / E, k_ = c_ % E;\n";
+        o << "        as::BinSlotP a_ = sc_[l_ * NE + k_];\n";
+        o << "        for (int t_ = 1; t_ < RPB; ++t_) { const as::BinSlotP b_ = sc_[(t_ * T + l_) * NE + k_]; "
+             "as::bins_merge_p(a_.J, a_.b, a_.sp, b_.J, b_.b, b_.sp); }\n";
+        o << "        *(as::BinSlotP*)" << slot_at("part", "blockIdx.x", static_cast<int>(q), "c_") << " = a_;\n";
+        o << "      }\n    }\n";
+      } else if (binned(id)) {
         o << "    {\n      as::BinSlot* sc_ = (as::BinSlot*)tma_smem;  // [team][lane][k]\n";
         o << "      if (threadIdx.x < CT) {\n#pragma unroll\n        for (int k = 0; k < NE; ++k) { as::BinSlot b_; b_.J = bJ" << id
           << "[k]; b_.sp = bs" << id << "[k]; b_.hi = bh" << id << "[k]; b_.lo = bl" << id << "[k]; b_.pad = 0; sc_[(team * T + lane) * NE + k] = b_; }\n      }\n";
@@ -1579,7 +1605,7 @@ struct Gen {
         o << "        as::BinSlot a_ = sc_[l_ * NE + k_];\n";
         o << "        for (int t_ = 1; t_ < RPB; ++t_) { const as::BinSlot b_ = sc_[(t_ * T + l_) * NE + k_]; "
              "as::bins_merge(a_.J, a_.hi, a_.lo, a_.sp, b_.J, b_.hi, b_.lo, b_.sp); }\n";
-        o << "        ((as::BinSlot*)part)[((long long)blockIdx.x * " << NS << " + " << q << ") * C + c_] = a_;\n";
+        o << "        *(as::BinSlot*)" << slot_at("part", "blockIdx.x", static_cast<int>(q), "c_") << " = a_;\n";
         o << "      }\n    }\n";
       } else {
         o << "    {\n      float* sc_ = (float*)tma_smem;\n";
@@ -1588,7 +1614,7 @@ struct Gen {
         o << "      for (int c_ = threadIdx.x; c_ < (int)C; c_ += blockDim.x) {\n";
         o << "        const int l_ = c_ / E, k_ = c_ % E;\n        float a_ = sc_[l_ * NE + k_];\n";
         o << "        for (int t_ = 1; t_ < RPB; ++t_) a_ = as::nmax(a_, sc_[(t_ * T + l_) * NE + k_]);\n";
-        o << "        ((as::BinSlot*)part)[((long long)blockIdx.x * " << NS << " + " << q << ") * C + c_].sp = a_;\n";
+        o << "        ((as::BinSlot*)" << slot_at("part", "blockIdx.x", static_cast<int>(q), "c_") << ")->sp = a_;\n";
         o << "      }\n    }\n";
       }
     }
@@ -1718,11 +1744,23 @@ struct Gen {
       if (phase_of(id) != cur_level) continue;
       bool mx = N(id).sub == ASTITCH_RMAX;
       std::string ident = mx ? "-AS_INF" : "0.f";
+      if (binned(id) && pc(id)) {  // tma_sweep, precise (R7c): merge the CTAs' fp64 bins, value in fp64
+        o << "      float t" << id << ";\n      double t" << id << "d;\n      {\n";
+        o << "        as::BinSlotP a_; a_.J = AS_BIN_EMPTY; a_.sp = 0.f; a_.b[0] = a_.b[1] = a_.b[2] = a_.b[3] = 0; a_.pad = 0;\n";
+        o << "        if (own) for (int r = pi; r < G; r += P) { const as::BinSlotP b_ = as::ld_cg_binsp((const as::BinSlotP*)"
+          << slot_at("part", "r", q, "col") << "); as::bins_merge_p(a_.J, a_.b, a_.sp, b_.J, b_.b, b_.sp); }\n";
+        o << "        as::BinSlotP* fs_ = (as::BinSlotP*)tma_smem;\n        fs_[threadIdx.x] = a_;\n        __syncthreads();\n";
+        o << "        for (int s = P / 2; s > 0; s /= 2) {\n          if (pi < s) { as::BinSlotP c_ = fs_[threadIdx.x]; const as::BinSlotP d_ = fs_[threadIdx.x + s]; "
+             "as::bins_merge_p(c_.J, c_.b, c_.sp, d_.J, d_.b, d_.sp); fs_[threadIdx.x] = c_; }\n          __syncthreads();\n        }\n";
+        o << "        const as::BinSlotP r_ = fs_[threadIdx.x - pi];\n        __syncthreads();\n";
+        o << "        t" << id << "d = as::bins_value_p(r_.J, r_.b, r_.sp);\n        t" << id << " = (float)t" << id << "d;\n      }\n";
+        continue;
+      }
       if (binned(id)) {  // tma_sweep: merge the CTAs' binned accumulators (exact, any order: R23)
         o << "      float t" << id << ";\n      {\n";
         o << "        as::BinSlot a_; a_.J = AS_BIN_EMPTY; a_.sp = 0.f; a_.hi = 0; a_.lo = 0; a_.pad = 0;\n";
-        o << "        if (own) for (int r = pi; r < G; r += P) { const as::BinSlot b_ = as::ld_cg_bins((const as::BinSlot*)part + ((long long)r * "
-          << NS << " + " << q << ") * C + col); as::bins_merge(a_.J, a_.hi, a_.lo, a_.sp, b_.J, b_.hi, b_.lo, b_.sp); }\n";
+        o << "        if (own) for (int r = pi; r < G; r += P) { const as::BinSlot b_ = as::ld_cg_bins((const as::BinSlot*)"
+          << slot_at("part", "r", q, "col") << "); as::bins_merge(a_.J, a_.hi, a_.lo, a_.sp, b_.J, b_.hi, b_.lo, b_.sp); }\n";
         o << "        as::BinSlot* fs_ = (as::BinSlot*)tma_smem;\n        fs_[threadIdx.x] = a_;\n        __syncthreads();\n";
         o << "        for (int s = P / 2; s > 0; s /= 2) {\n          if (pi < s) { as::BinSlot c_ = fs_[threadIdx.x]; const as::BinSlot d_ = fs_[threadIdx.x + s]; "
              "as::bins_merge(c_.J, c_.hi, c_.lo, c_.sp, d_.J, d_.hi, d_.lo, d_.sp); fs_[threadIdx.x] = c_; }\n          __syncthreads();\n        }\n";
@@ -1733,7 +1771,7 @@ struct Gen {
       if (m.tma_sweep) {  // tma_sweep column MAX: the CTA maxima sit in the slots' sp words
         o << "      float t" << id << " = -AS_INF;\n";
         o << "      if (own) for (int r = pi; r < G; r += P) t" << id << " = as::nmax(t" << id
-          << ", as::ld_cg(&((const as::BinSlot*)part + ((long long)r * " << NS << " + " << q << ") * C + col)->sp));\n";
+          << ", as::ld_cg(&((const as::BinSlot*)" << slot_at("part", "r", q, "col") << ")->sp));\n";
         o << "      fin_smem[threadIdx.x] = t" << id << ";\n      __syncthreads();\n";
         o << "      for (int s = P / 2; s > 0; s /= 2) { if (pi < s) fin_smem[threadIdx.x] = as::nmax(fin_smem[threadIdx.x], fin_smem[threadIdx.x + s]); __syncthreads(); }\n";
         o << "      t" << id << " = fin_smem[threadIdx.x - pi];\n      __syncthreads();\n";

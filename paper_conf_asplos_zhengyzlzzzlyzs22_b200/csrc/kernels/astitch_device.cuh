@@ -693,8 +693,84 @@ __device__ __forceinline__ double bins_value_d(int J, long long hi, long long lo
   if (J == AS_BIN_EMPTY) return 0.0;
   return ldexp((double)hi, 32 * (J + 1) - 160) + ldexp((double)lo, 32 * J - 160);
 }
-// one accumulator in the workspace (32 bytes: J, sp, hi, lo)
+// one accumulator in the workspace (J, sp, hi, lo; slots are 48 bytes apart)
 struct BinSlot { int J; float sp; long long hi, lo, pad; };
+
+// Precise variant for fp64 tile partials (column sums whose mean is later
+// subtracted, reading R7c): four 16-bit-aligned int64 bins b[0..3] of a
+// 64-bit window on the absolute scale 2^-1100 (|x| = m * 2^(bi - 1100),
+// bi = biased fp64 exponent + 25); window J holds bits [16J, 16J + 64), so
+// the largest deposit keeps >= 48 bits (fp32 bins: >= 32).  Same exactness /
+// order independence as the fp32 bins.
+struct BinSlotP { int J; float sp; long long b[4]; long long pad; };
+__device__ __forceinline__ void binsp_shift(int& J, long long* b, int need) {
+  const int t = need - J;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) b[k] = (k + t < 4) ? b[(k + t) & 3] : 0;
+  J = need;
+}
+template <int NE>
+__device__ __forceinline__ void bins_add_p(int* J, long long* b, float* sp, const double* x) {
+#pragma unroll
+  for (int k = 0; k < NE; ++k) {
+    const u64 u = static_cast<u64>(__double_as_longlong(x[k]));
+    const u32 e = static_cast<u32>(u >> 52) & 0x7ffu;
+    if (e == 0x7ffu) { sp[k] += static_cast<float>(x[k]); continue; }
+    const u64 mn = u & 0xfffffffffffffull;
+    if (!(mn | e)) continue;
+    const int bi = (int)(e ? e : 1u) + 25;
+    const int need = (bi + 4) >> 4;
+    long long* bk = b + 4 * k;
+    if (need > J[k]) {
+      if (J[k] == AS_BIN_EMPTY || need - J[k] >= 4) { bk[0] = bk[1] = bk[2] = bk[3] = 0; J[k] = need; }
+      else binsp_shift(J[k], bk, need);
+    }
+    const u64 m = mn | (e ? (1ull << 52) : 0ull);
+    const int d = min(bi - 16 * J[k], 11);
+    const u64 v = d >= 0 ? (m << d) : (d > -53 ? (m >> (-d)) : 0ull);
+    const bool neg = (u >> 63) != 0ull;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const long long sl = static_cast<long long>((v >> (16 * q)) & 0xffffull);
+      bk[q] += neg ? -sl : sl;
+    }
+  }
+}
+__device__ __forceinline__ void bins_merge_p(int& J, long long* b, float& sp, int J2, const long long* b2, float sp2) {
+  sp += sp2;
+  if (J2 == AS_BIN_EMPTY) return;
+  if (J == AS_BIN_EMPTY || J2 - J >= 4) {
+    if (J2 > J) { b[0] = b[1] = b[2] = b[3] = 0; J = J2; }
+  } else if (J2 > J) {
+    binsp_shift(J, b, J2);
+  }
+  const int t = J - J2;  // >= 0: drop b2's lowest t bins
+#pragma unroll
+  for (int k = 0; k < 4; ++k)
+    if (k + t < 4) b[k] += b2[(k + t) & 3];
+}
+__device__ __forceinline__ double bins_value_p(int J, const long long* b, float sp) {
+  if (sp != 0.f) return (double)sp;
+  if (J == AS_BIN_EMPTY) return 0.0;
+  double v = 0.0;
+#pragma unroll
+  for (int k = 3; k >= 0; --k) v += ldexp((double)b[k], 16 * (J + k) - 1100);
+  return v;
+}
+__device__ __forceinline__ BinSlotP ld_cg_binsp(const BinSlotP* p) {
+  const Raw<16> a = ldg_cg(reinterpret_cast<const Raw<16>*>(p));
+  const Raw<16> c = ldg_cg(reinterpret_cast<const Raw<16>*>(p) + 1);
+  const Raw<8> d = ldg_cg(reinterpret_cast<const Raw<8>*>(p) + 4);
+  BinSlotP s;
+  s.J = static_cast<int>(a.x);
+  s.sp = __uint_as_float(a.y);
+  s.b[0] = static_cast<long long>((static_cast<u64>(a.w) << 32) | a.z);
+  s.b[1] = static_cast<long long>((static_cast<u64>(c.y) << 32) | c.x);
+  s.b[2] = static_cast<long long>((static_cast<u64>(c.w) << 32) | c.z);
+  s.b[3] = static_cast<long long>((static_cast<u64>(d.y) << 32) | d.x);
+  s.pad = 0;
+  return s;
+}
 // L2-coherent load of a slot written by another CTA earlier in the kernel
 __device__ __forceinline__ BinSlot ld_cg_bins(const BinSlot* p) {
   const Raw<16> a = ldg_cg(reinterpret_cast<const Raw<16>*>(p));

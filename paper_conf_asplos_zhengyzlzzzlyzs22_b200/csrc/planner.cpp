@@ -615,7 +615,8 @@ void select_mapping(Plan& p) {
       // barrier levels (dependent column reductions, values read after a
       // barrier) are swept one after the other by the same ring; sharded
       // plans keep one sweep per kernel (their level-1 sweep is a separate
-      // role), precise column sums (R7c) need more than the bins' 32 bits
+      // role); precise column sums (R7c) deposit fp64 tile partials into
+      // 4 x 16-bit bins (>= 48 bits, as::bins_add_p)
       bool one_sweep = true;
       for (size_t i = 0; i < g.nodes.size(); ++i) {
         if (!p.info[i].live) continue;
@@ -624,7 +625,7 @@ void select_mapping(Plan& p) {
       }
       const bool levels_ok = one_sweep || p.desc.shard_world <= 1;
       bool ok = tu.tma != 0 && !no_tma && has_colred && levels_ok && !has_rowred && !has_rowvec &&
-                !has_mask && !ragged && m.nslab == 1 && p.n_precise_colreds == 0 &&
+                !has_mask && !ragged && m.nslab == 1 &&
                 R < (1LL << 30) && (p.desc.flags & ASTITCH_FLAG_FORCE_GLOBAL) == 0 && es_max <= 4;
       int64_t rowbytes = 0;
       for (int id : g.inputs) {
@@ -652,8 +653,13 @@ void select_mapping(Plan& p) {
         const int64_t ring = S * TR * rowbytes;
         // the CTA combine of the teams' accumulators (one 32-byte as::BinSlot
         // per lane column) and the finalise scratch reuse the ring
-        const int64_t comb = std::max<int64_t>(static_cast<int64_t>(TM) * T * Et * 32, (TM * T + 32) * 32);
-        if (TR >= std::max(4, TM) && ring <= budget && ring >= comb) {
+        const int64_t comb = std::max<int64_t>(static_cast<int64_t>(TM) * T * Et * 48, (TM * T + 32) * 48);
+        // long sweeps only (>= 16 tiles per CTA): a short sweep is latency-
+        // bound and pays the ring's fill and the producer hop (measured on
+        // B200, BatchNorm fp32 [25088, 128]: 35.3 us vs 30.4 us static;
+        // [1M, 1024]: 2.54 ms vs 2.77 ms); tuning tma=1 forces it
+        const int64_t trips = ((R + TR - 1) / std::max<int64_t>(TR, 1) + sms - 1) / sms;
+        if (TR >= std::max(4, TM) && ring <= budget && ring >= comb && (trips >= 16 || tu.tma == 1)) {
           m.tma_sweep = true;
           m.vec_elems = E = Et;
           m.chunks = static_cast<int>(C / Et);
@@ -1075,8 +1081,8 @@ void plan_workspace(Plan& p) {
     const int64_t nparts = p.map.grid;
     // partial slots: one per column reduction + a lo slot per precise sum (R7c)
     const size_t nslots = p.colreds.size() + static_cast<size_t>(p.n_precise_colreds);
-    // (tma_sweep: a 32-byte binned accumulator per slot and column, as::BinSlot)
-    off = align(off + static_cast<size_t>(nparts) * nslots * C * (p.map.tma_sweep ? 32 : 4));
+    // (tma_sweep: a 48-byte binned accumulator per slot and column, as::BinSlot / as::BinSlotP)
+    off = align(off + static_cast<size_t>(nparts) * nslots * C * (p.map.tma_sweep ? 48 : 4));
     w.colvals = off;
     // [post COLVEC hi][rank-local column totals][post COLVEC lo (R7c)]
     bool any_precise_post = false;

@@ -379,7 +379,7 @@ def test_tma_sweep_selection():
     """tma_sweep (R23) for one-sweep element-wise + column-reduction graphs
     (C5 and its shapes); not for row reductions (fig7a), dependent column
     levels (BatchNorm), masks, or when switched off (tuning tma=0, NO_TMA)."""
-    def m(name, rows=4096, cols=None, **kw):
+    def m(name, rows=1 << 20, cols=None, **kw):
         s = specs.get(name, rows=rows, cols=cols)
         return A.Plan(A.Graph.from_spec(s), rows, s["cols"], device=-1, flags=kw.get("flags", A.FLAG_NO_COMPILE),
                       tune=kw.get("tune")).describe()["mapping"]
@@ -393,5 +393,7 @@ def test_tma_sweep_selection():
     assert not m("C5", cols=16384)["tma_sweep"]                      # column slabs instead
     assert not m("C5", tune="tma=0")["tma_sweep"]
     assert not m("C5", flags=A.FLAG_NO_COMPILE | A.FLAG_NO_TMA)["tma_sweep"]
-    assert not m("fig7a")["tma_sweep"] and not m("bn", rows=3000, cols=128)["tma_sweep"]
-    assert m("C5", rows=7)["grid"] == 1                              # never more CTAs than tiles
+    assert not m("fig7a")["tma_sweep"]                               # row reductions
+    assert not m("bn", rows=3000, cols=128)["tma_sweep"]             # short sweep (< 16 tiles per CTA)
+    assert m("bn", rows=1 << 20, cols=1024)["tma_sweep"]             # long BatchNorm: 3 levels, precise bins
+    assert m("C5", rows=7, tune="tma=1")["grid"] == 1                # never more CTAs than tiles

@@ -16,14 +16,17 @@ pytestmark = pytest.mark.gpu
 
 
 def _plan(spec, **kw):
+    """Plans default to tune tma=1: the planner takes tma_sweep by itself for
+    long sweeps only (>= 16 tiles per CTA); these tests use small shapes."""
     import torch
     import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    kw.setdefault("tune", "tma=1")
     return A.Plan(A.Graph.from_spec(spec), spec["rows"], spec["cols"], device=torch.cuda.current_device(), **kw)
 
 
 def test_tma_sweep_chosen_for_c5():
-    spec = specs.get("C5", rows=4096)
-    m = _plan(spec).describe()["mapping"]
+    spec = specs.get("C5", rows=1 << 20)
+    m = _plan(spec, tune=None).describe()["mapping"]
     assert m["tma_sweep"] and m["template"] == "global_sweep"
     assert m["threads"] == m["rows_per_block"] * m["team"] + 32   # + the producer warp
     assert m["blocks_per_sm"] == 1 and m["smem_bytes"] == m["tma_stages"] * m["tma_rows"] * 2 * 1024 * 2
@@ -189,7 +192,7 @@ def test_tma_sweep_barrier_levels(seed, rows, cols):
     from workloads.random_graphs import random_graph
     spec = random_graph(seed, rows, cols, rowwise=False)
     x = gen.generate("fig6a", spec)
-    got, plan = run_gpu(spec, x, return_plan=True)
+    got, plan = run_gpu(spec, x, return_plan=True, tune="tma=1")
     d = plan.describe()
     assert d["mapping"]["tma_sweep"]
     ref = evaluate(spec, x)
@@ -198,3 +201,26 @@ def test_tma_sweep_barrier_levels(seed, rows, cols):
     again = run_gpu(spec, x, plan=plan)
     for k in got:
         assert np.array_equal(got[k], again[k]), k
+
+
+@pytest.mark.parametrize("rows,cols", [(3, 1024), (777, 128), (20000, 256), (5, 4096)])
+@pytest.mark.parametrize("mean", [0.0, 1000.0, -3.0e4])
+def test_tma_sweep_precise_bins_batchnorm(rows, cols, mean):
+    """BatchNorm under tma_sweep: the column mean is a precise sum (R7c) whose
+    fp64 tile partials go to 4 x 16-bit bins (>= 48 bits): means up to 3e6x
+    the spread hold the fp32 1e-5 rule, and the totals are identical for
+    grids of 148 and 7 CTAs."""
+    spec = specs.get("bn", rows=rows, cols=cols)
+    x = gen.generate("bn", spec)
+    x["x"] = (mean + 0.01 * x["x"].astype(np.float64)).astype(np.float32)
+    ref = evaluate(spec, x)
+    outs = []
+    for sms in (0, 7):
+        p = _plan(spec, sm_count=sms)
+        assert p.describe()["mapping"]["tma_sweep"]
+        got = run_gpu(spec, x, plan=p)
+        for name, dt in spec["outputs"]:
+            check_close(got[name], ref[name], dt, spec_tol(spec), name=f"bn[{rows},{cols}] mean={mean}:{name}")
+        outs.append(got)
+    for k in outs[0]:
+        assert np.array_equal(outs[0][k], outs[1][k]), k
