@@ -37,7 +37,7 @@ def case(seed, argv):
 def main():
     seed = int(sys.argv[1])
     spec, flags = case(seed, sys.argv)
-    tunes = [a.split("=", 1)[1] for a in sys.argv if a.startswith("--tune=")] or [None]
+    tunes = [a.split("=", 1)[1] for a in sys.argv if a.startswith("--tune=")] or ["tma=1" if "--tma" in sys.argv else None]
     if "--show" in sys.argv:
         import json
         print(json.dumps(spec, indent=0)[:4000])

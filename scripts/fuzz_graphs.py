@@ -48,7 +48,9 @@ def main():
             flags = int(rng.choice([0, 0, 0, 0, 0, 2, 4, 64]))
         x = gen.generate("fig6a", spec)
         try:
-            got, plan = run_gpu(spec, x, return_plan=True, flags=flags)
+            # --tma: force the bulk-copy sweep where eligible (the planner takes
+            # it by itself only for long sweeps; fuzz shapes are small)
+            got, plan = run_gpu(spec, x, return_plan=True, flags=flags, tune="tma=1" if "--tma" in sys.argv else None)
             ref = evaluate(spec, x)
             errs = []
             for name, dt in spec["outputs"]:
