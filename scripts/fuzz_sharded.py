@@ -96,7 +96,7 @@ def main():
                 ranks = []
                 for r in range(world):
                     sp = ShardedPlan(g, rows, cols, world, r, 0, sm_count=sms // world if mode == "fused" else 0,
-                                     tune="bps=1" if mode == "fused" else None,
+                                     tune=(("bps=1," if mode == "fused" else "") + ("tma=1" if "--tma" in sys.argv else "")).strip(",") or None,
                                      row_range=rr[r])
                     b, nr = sp.row_begin, sp.row_count
                     ins = device_inputs(dict(spec, rows=nr), shard_inputs(spec, x, b, nr))
