@@ -1439,9 +1439,10 @@ struct Gen {
   bool binned(int id) const { return m.tma_sweep && N(id).sub != ASTITCH_RMAX; }
   // byte address of (CTA g, partial slot q, column col) in the tma_sweep
   // partial region (48-byte slots: as::BinSlot / as::BinSlotP / an fp32 max)
+  // (32-byte slots unless a precise sum needs as::BinSlotP's 48)
   std::string slot_at(const std::string& base, const std::string& gi, int q, const std::string& col) const {
     return "((const char*)(" + base + ") + (((long long)(" + gi + ") * " + std::to_string(nslots()) + " + " +
-           std::to_string(q) + ") * C + (" + col + ")) * 48LL)";
+           std::to_string(q) + ") * C + (" + col + ")) * " + (p.n_precise_colreds > 0 ? "48LL)" : "32LL)");
   }
   // prologue (once per kernel): ring, mbarriers, the running stage counters
   // of the producer (kt_p) and of the consumers (kt_c), which continue across

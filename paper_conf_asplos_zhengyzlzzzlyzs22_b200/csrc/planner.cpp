@@ -1081,8 +1081,10 @@ void plan_workspace(Plan& p) {
     const int64_t nparts = p.map.grid;
     // partial slots: one per column reduction + a lo slot per precise sum (R7c)
     const size_t nslots = p.colreds.size() + static_cast<size_t>(p.n_precise_colreds);
-    // (tma_sweep: a 48-byte binned accumulator per slot and column, as::BinSlot / as::BinSlotP)
-    off = align(off + static_cast<size_t>(nparts) * nslots * C * (p.map.tma_sweep ? 48 : 4));
+    // (tma_sweep: a binned accumulator per slot and column, as::BinSlot 32 B,
+    // as::BinSlotP 48 B when a precise sum needs it)
+    const size_t slot_bytes = !p.map.tma_sweep ? 4 : (p.n_precise_colreds > 0 ? 48 : 32);
+    off = align(off + static_cast<size_t>(nparts) * nslots * C * slot_bytes);
     w.colvals = off;
     // [post COLVEC hi][rank-local column totals][post COLVEC lo (R7c)]
     bool any_precise_post = false;
