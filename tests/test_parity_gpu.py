@@ -403,9 +403,13 @@ def test_parity_op_vocabulary(spec, template):
     _compare(spec, got, evaluate(spec, x))
 
 
-@pytest.mark.parametrize("cfg,rows,cols,world", [("C5", 3001, 1024, 2), ("C5", 4099, 256, 4), ("fig7a", 1001, 96, 2),
-                                                 ("C5int", 4096, 128, 2), ("bn", 1500, 64, 2)])
-def test_fused_exchange_virtual_ranks(cfg, rows, cols, world):
+@pytest.mark.parametrize("cfg,rows,cols,world,tune", [("C5", 3001, 1024, 2, None), ("C5", 4099, 256, 4, None),
+                                                      ("fig7a", 1001, 96, 2, None), ("C5int", 4096, 128, 2, None),
+                                                      ("bn", 1500, 64, 2, None),
+                                                      # the fused role under tma_sweep (R23 bins + peer exchange)
+                                                      ("C5", 3001, 1024, 2, "tma=1"), ("C5", 4099, 256, 4, "tma=1"),
+                                                      ("C5int", 4096, 128, 2, "tma=1")])
+def test_fused_exchange_virtual_ranks(cfg, rows, cols, world, tune):
     """astitch_run_fused (NEXT f1): every rank's ONE cooperative kernel pushes its
     column totals into all ranks' exchange slots, flags them and combines the
     slots in rank order.  Virtual ranks share one GPU (each plan sized for
@@ -426,7 +430,9 @@ def test_fused_exchange_virtual_ranks(cfg, rows, cols, world):
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     ranks = []
     for r in range(world):
-        sp = ShardedPlan(g, rows, cols, world, r, 0, sm_count=sms // world - 1)  # one SM of slack: the virtual ranks share one GPU
+        sp = ShardedPlan(g, rows, cols, world, r, 0, sm_count=sms // world - 1, tune=tune)  # one SM of slack: the virtual ranks share one GPU
+        if tune:
+            assert sp.plan.describe()["mapping"]["tma_sweep"]
         b, n = sp.row_begin, sp.row_count
         xs = {k: (v[b:b + n] if getattr(v, "ndim", 0) == 2 or k == "p2" else v) for k, v in x.items()}
         ins = device_inputs(dict(spec, rows=n), xs)
