@@ -1649,6 +1649,9 @@ struct Gen {
     o << "  __shared__ int tma_tile[NSTG];\n";
     o << "  unsigned int* tctr = (unsigned int*)((char*)p.ws + " << (p.ws.barrier + 64) << "LL);\n";
     o << "  unsigned int* tdone = (unsigned int*)((char*)p.ws + " << (p.ws.barrier + 68) << "LL);\n";
+    // (ragged) per stage: the segment pitch (elements) when the tile's rows
+    // were copied with ONE bulk copy (all in one segment: contiguous), else 0
+    if (ragged) o << "  __shared__ int tma_pk[NSTG];\n";
     o << "  const int NTILES = (int)((R + TR - 1) / TR);\n";
     o << "  const unsigned sbase_ = as::smem_addr(tma_smem);\n";
     o << "  if (threadIdx.x == 0) {\n    for (int s = 0; s < NSTG; ++s) { as::mbar_init(as::smem_addr(&tma_full[s]), 1u); "
@@ -1666,6 +1669,23 @@ struct Gen {
     o << "      const int prow = tile * TR + pl;\n";
     o << "      const bool pact = pl < TR && prow < R;\n";
     o << "      " << limdecl("plim", "pact", "prow") << "\n      (void)plim;\n";
+    if (ragged) {
+      // rows of one segment are contiguous at the segment's pitch (a multiple
+      // of 8 elements): the whole tile in one bulk copy per stream
+      o << "      const int fx_ = __shfl_sync(0xffffffffu, plim_s.x, 0);\n";
+      o << "      if (__all_sync(0xffffffffu, !pact || plim_s.x == fx_)) {\n";
+      o << "        const int nact_ = __popc(__ballot_sync(0xffffffffu, pact));\n";
+      o << "        if (pl == 0) {\n          tma_tile[st] = tile; tma_pk[st] = plim_s.z;\n";
+      long long tot = 0;
+      for (size_t s = 0; s < streams.size(); ++s) tot += dtype_size(streams[s].dt);
+      o << "          as::mbar_expect_tx(fb, (unsigned)(nact_ * plim_s.z * " << tot << "));\n";
+      for (size_t s = 0; s < streams.size(); ++s)
+        o << "          as::bulk_g2s(sbase_ + (unsigned)(" << soff[s] << "LL + (long long)st * TR * " << slot[s]
+          << "LL), (const char*)p.in[" << N(streams[s].node).input_index << "] + (long long)plim_b * " << nb(streams[s].dt)
+          << "LL, (unsigned)(nact_ * plim_s.z * " << dtype_size(streams[s].dt) << "), fb);\n";
+      o << "        }\n        continue;\n      }\n";
+      o << "      if (pl == 0) tma_pk[st] = 0;\n";
+    }
     o << "      unsigned nbytes_ = 0;\n";
     for (size_t s = 0; s < streams.size(); ++s) {
       const int es = dtype_size(streams[s].dt);
@@ -1701,8 +1721,13 @@ struct Gen {
       o << "      const long long c0 = " << chx("j") << " * E;\n";
       std::string cond = "act0";
       if (!exact || masked) cond += " && c0 < lim0";
-      o << "      if (" << cond << ") r" << s << "_u0[j] = as::lds_chunk<" << nb(stv.dt) << ">(sbase_ + (unsigned)(" << soff[s]
-        << "LL + ((long long)st * TR + rl_) * " << slot[s] << "LL + " << chx("j") << " * " << nb(stv.dt) << "LL));\n";
+      if (ragged)  // the row's offset: segment pitch when the tile came in one copy, else its slot
+        o << "      if (" << cond << ") r" << s << "_u0[j] = as::lds_chunk<" << nb(stv.dt) << ">(sbase_ + (unsigned)(" << soff[s]
+          << "LL + (long long)st * TR * " << slot[s] << "LL + (tma_pk[st] ? (long long)rl_ * tma_pk[st] * " << dtype_size(stv.dt)
+          << "LL : (long long)rl_ * " << slot[s] << "LL) + " << chx("j") << " * " << nb(stv.dt) << "LL));\n";
+      else
+        o << "      if (" << cond << ") r" << s << "_u0[j] = as::lds_chunk<" << nb(stv.dt) << ">(sbase_ + (unsigned)(" << soff[s]
+          << "LL + ((long long)st * TR + rl_) * " << slot[s] << "LL + " << chx("j") << " * " << nb(stv.dt) << "LL));\n";
       if (!absorb) o << "      else r" << s << "_u0[j] = " << raw_t(stv) << "{};\n";
       o << "    }\n";
     }
