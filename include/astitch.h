@@ -227,8 +227,12 @@ astitch_status astitch_plan(astitch_graph_t g, const astitch_plan_desc* desc, as
  * assume-relax-apply), vec_bytes (16|32), hoist (0|1), tile_stages, tile_rows,
  * tile_threads, split, split_threads, stream (1 force row_stream, 0 never),
  * stage (1: row_stream stages rows in smem), stage_kb, portable_clusters,
- * dyn_colred_rows (global sweep: counter-ordered row tiles).  Values a
- * template cannot use are ignored.  The plan is a pure function of
+ * sync (block barrier per row step), prefetch, persistent (0: one row group
+ * per CTA), waves (grid = waves x resident CTAs), remat (0: buffer values read
+ * after a barrier instead of recomputing, R22), tma (0: never tma_sweep, 1:
+ * whenever eligible, also short sweeps), tma_rows, tma_stages, tma_teams
+ * (bulk-copy ring shape), tma_team (1: row teams fed by bulk copies).  Values
+ * a template cannot use are ignored.  The plan is a pure function of
  * (graph, desc, tuning): the library reads no environment variables for
  * planning or code generation.  describe() reports the string.
  * Errors: as astitch_plan, plus ERR_INVALID_ARGUMENT for an unknown key or a
