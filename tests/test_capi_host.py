@@ -261,3 +261,22 @@ def test_disk_cubin_cache_and_plan_time(tmp_path):
     r3 = json.loads(subprocess.run([sys.executable, "-c", code], capture_output=True, text=True,
                                    check=True).stdout.strip().splitlines()[-1])
     assert r3["nvrtc_compiles"] >= 1
+
+
+def test_documented_tuning_keys_are_accepted():
+    """Every key astitch.h documents for astitch_plan_ex parses; an unknown
+    key is ERR_INVALID_ARGUMENT (keeps the header and the parser in step)."""
+    import os
+    import re
+    hdr = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include", "astitch.h")).read()
+    doc = hdr[hdr.index("keys: threads"):hdr.index("Values\n * a template cannot use")]
+    keys = {k for k in re.findall(r"\b([a-z_]+)\b(?=[ ,(.]|$)", doc.replace("\n *", " "))
+            if k in {"threads", "unroll", "team", "bps", "vec_bytes", "hoist", "tile_stages", "tile_rows", "tile_threads",
+                     "split", "split_threads", "stream", "stage", "stage_kb", "portable_clusters", "sync", "prefetch",
+                     "persistent", "waves", "remat", "tma", "tma_rows", "tma_stages", "tma_teams", "tma_team"}}
+    assert len(keys) == 25, sorted(keys)
+    spec = specs.get("C5", rows=64, cols=32)
+    for k in sorted(keys):
+        A.Plan(A.Graph.from_spec(spec), 64, 32, device=-1, flags=A.FLAG_NO_COMPILE, tune=f"{k}=1")
+    with pytest.raises(A.AstitchError):
+        A.Plan(A.Graph.from_spec(spec), 64, 32, device=-1, flags=A.FLAG_NO_COMPILE, tune="dyn_colred_rows=16")
