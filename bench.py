@@ -719,7 +719,9 @@ def main():
                        "l2": ("inputs > L2 (%.2f GB per rank vs %d MB L2)" % (nbytes / 1e9, l2 // 2**20)) if nsets == 1
                        else f"{nsets} rotating input sets >= 4x L2",
                        "timing": "cuda_graph_replay" if graph is not None else "eager",
-                       "template": desc["mapping"]["template"], "grid": desc["kernels"][0]["grid"],
+                       "template": desc["mapping"]["template"] + ("/tma_sweep" if desc["mapping"].get("tma_sweep") else "")
+                                   + ("/tma_team" if desc["mapping"].get("tma_team") else ""),
+                       "grid": desc["kernels"][0]["grid"],
                        "threads": desc["mapping"]["threads"], "regs": desc["kernels"][0]["regs"],
                        "tuning": desc.get("tuning") or None, "flags": args.flags or None},
             "us_per_subgraph": round(ms_step * 1e3, 3),
