@@ -5,7 +5,7 @@
 #   2 FORCE_GLOBAL  regional -> global demotion (row reductions via HBM + grid barrier)
 #   4 NO_PACK       no horizontal packing (one row per warp, XLA-style mapping)
 #   8 NO_SPLIT      no task splitting of long rows
-#  32 NO_TMA        no TMA-staged packed tiles
+#  32 NO_TMA        no bulk-copy (TMA) staging: packed tiles, tma_sweep, tma_team
 #  64 NO_PREFETCH   no software prefetch of the next row
 # Output: gpurun_out/ablation.jsonl (one bench.py line per run, "flags" added).
 mkdir -p gpurun_out
@@ -22,9 +22,9 @@ run() {  # config flags [extra bench args]
 }
 for f in 0 2 4; do run C1 $f; done
 for f in 0 2 4 64; do run C2 $f; done
-for f in 0 2 4 64; do run C3 $f; done
+for f in 0 2 4 32 64; do run C3 $f; done
 for f in 0 2 4 32; do run C4 $f; done
-for f in 0 4 64; do run C5 $f; done
+for f in 0 4 32 64; do run C5 $f; done
 for f in 0 4; do run fig6a $f; done
 for f in 0 8; do run fig6b $f --rows 64 --cols 300000; done
 python scripts/summarize_ablation.py $out
