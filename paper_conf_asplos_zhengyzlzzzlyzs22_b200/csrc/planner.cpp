@@ -651,8 +651,9 @@ void select_mapping(Plan& p) {
         if (tu.tma_rows > 0) TR = tu.tma_rows;
         TR -= TR % TM;
         const int64_t ring = S * TR * rowbytes;
-        // the CTA combine of the teams' accumulators (one 32-byte as::BinSlot
-        // per lane column) and the finalise scratch reuse the ring
+        // the CTA combine of the teams' accumulators (one as::BinSlot /
+        // as::BinSlotP, <= 48 bytes, per lane column) and the finalise
+        // scratch reuse the ring
         const int64_t comb = std::max<int64_t>(static_cast<int64_t>(TM) * T * Et * 48, (TM * T + 32) * 48);
         // long sweeps only (>= 16 tiles per CTA): a short sweep is latency-
         // bound and pays the ring's fill and the producer hop (measured on
@@ -944,8 +945,9 @@ void select_mapping(Plan& p) {
   // masked rows of >= 512 bytes (measured on B200, C3: 16-row tiles x 4
   // stages, 3 CTAs/SM, 135.8 us vs 140.4 us for the oversubscribed register
   // row teams; 1 CTA/SM with 128 KB rings 193 us); opt-in (tuning
-  // tma_team=1) elsewhere: packed varlen rows (C3v) measured equal (78.5 vs
-  // 78.1 us), unmasked rows are not better served than by register rows.
+  // tma_team=1) elsewhere: packed varlen rows (C3v: 80.9 us with 16-lane
+  // teams and one bulk copy per single-segment tile vs 78.9 us register
+  // rows), unmasked rows are not better served than by register rows.
   const bool tma_team_default = has_mask && !ragged && C * es_min >= 512;
   if (m.tmpl == Template::RowTeam && (tu.tma_team == 1 || (tu.tma_team != 0 && tma_team_default)) && !no_tma &&
       R < (1LL << 30) && es_max <= 4) {
