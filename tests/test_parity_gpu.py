@@ -286,6 +286,16 @@ def test_full_c5_sampled():
     b = x["b"].astype(np.float32)
     exp = (b - np.float32(0.0078125) * got["db"].astype(np.float32)).astype(np.float32)
     np.testing.assert_array_equal(got["b_new"].astype(np.float32), exp)
+    # R23 at full size: the bench plan (tma_sweep, address-ordered tiles,
+    # exact binned db) on a grid of 74 CTAs instead of 148 -- every tile taken
+    # by a different CTA in a different order -- gives the same bits
+    import torch
+    import paper_conf_asplos_zhengyzlzzzlyzs22_b200 as A
+    p74 = A.Plan(A.Graph.from_spec(spec), spec["rows"], spec["cols"], device=torch.cuda.current_device(), sm_count=74)
+    assert p74.describe()["mapping"]["tma_sweep"]
+    got74 = run_gpu(spec, x, plan=p74)
+    for k in ("db", "b_new", "dz"):
+        assert np.array_equal(got74[k], got[k]), k
 
 
 @pytest.mark.parametrize("cfg", ["C2", "C3", "C4", "C5"])
