@@ -275,7 +275,7 @@ def test_full_c5_sampled():
     check_close(got["db"][cols], refc["db"], "F32", 2e-3, "C5 db")
     check_close(got["b_new"][cols], refc["b_new"], "F32", 2e-3, "C5 b_new")
     # fp32-quality check for db (reading R4): 1e-5 relative to the RMS
-    # (measured 9.7e-7 at full size, profiles/r02_parity_report.json)
+    # (measured 3.1e-7 at full size through tma_sweep's exact bins, profiles/r02_parity_report.json)
     s = np.sqrt(np.mean(refc["db"] ** 2))
     assert np.max(np.abs(got["db"][cols] - refc["db"])) <= 1e-5 * s
     rows = np.unique(rng.integers(0, spec["rows"], 3000))
